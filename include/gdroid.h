@@ -1,0 +1,150 @@
+/*
+ * gdroid.h — C ABI of the B200-native IDFG construction library (libgdroid.so).
+ *
+ * What the library computes: the Inter-procedural Data-Flow Graph of Eq. (1)
+ * (PAPER.md:351-355), IDFG(E_C) = ((N,E), {fact(n) | n in N}), by the worklist
+ * fixed point of Alg. 1 re-designed as Alg. 3-style device
+ * rounds: matrix/bitset facts (MAT, §IV-A),
+ * class-grouped worklists (GRP, §IV-B) and de-duplicated
+ * merged worklists (MER, §IV-C).  fact(n) is the in-set
+ * IN(n) (DESIGN.md §3 reading A4); the exact semantics — node transfer
+ * functions, CALL/RET/C2R edge transforms with pool projection — are
+ * SURVEY.md §8(c) C1-C4 as restated in DESIGN.md §3.
+ *
+ * Every entry point is extern "C", takes plain pointers and sizes, never throws,
+ * and returns a gdroid_status (negative = error; gdroid_last_error() gives a
+ * message naming the first offending index).
+ *
+ * Ownership: all desc arrays are caller-owned HOST memory, read only during
+ * gdroid_load_*; the caller may free them on return.  A gdroid_app handle owns
+ * all device and pinned memory it allocates until gdroid_free (which accepts
+ * NULL).  Distinct handles may be used concurrently from different threads; a
+ * single handle is not thread-safe.
+ *
+ * Streams: all device work of a handle is issued on the cudaStream_t passed to
+ * gdroid_load_* (NULL = legacy default stream).  gdroid_build_idfg is
+ * synchronous unless opts->async is set (then gdroid_sync completes it).
+ */
+#ifndef GDROID_H
+#define GDROID_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GDROID_ABI_VERSION 1u
+
+typedef enum {
+  GDROID_OK = 0,
+  GDROID_E_INVALID = -1,  /* structural fault: CSR, ids, edge/node kinds (V5), arity (V6)    */
+  GDROID_E_POOL = -2,     /* pool closure violated (V1-V4)                     */
+  GDROID_E_OOM = -3,      /* device or pinned allocation failed                             */
+  GDROID_E_CUDA = -4,     /* CUDA runtime error (message has the CUDA error string)          */
+  GDROID_E_STATE = -5,    /* read before build / sync without a pending async build          */
+  GDROID_E_RANGE = -6,    /* node or app index out of range                                  */
+  GDROID_E_SMALLBUF = -7, /* caller buffer too small; *n_pairs holds the needed count        */
+  GDROID_E_LIMIT = -8     /* max_rounds exceeded (facts are an under-approximation), or a
+                             size limit (> 512 instances in one module pool, > 2^32 edges)  */
+} gdroid_status;
+
+/* Node kinds: SURVEY §8(c) C2; the paper's 9 statement + 17 expression kinds
+ * map onto these (DESIGN.md §3 table). */
+typedef enum {
+  GK_NOP = 0, GK_ENTRY, GK_EXIT, GK_RETSITE, GK_CALL, GK_PRIM, GK_CONST, GK_NEW,
+  GK_COPY, GK_SLOAD, GK_SSTORE, GK_RETV, GK_FLOAD, GK_FSTORE, GK_ALOAD, GK_ASTORE
+} gdroid_node_kind;
+
+/* Edge kinds: SURVEY §8(c) C3 ("blue arrow-lines", Fig. 2). */
+typedef enum { GE_INTRA = 0, GE_CALL, GE_RET, GE_C2R } gdroid_edge_kind;
+
+#define GDROID_F_ARR 0u   /* the array pseudo-field id */
+
+typedef struct gdroid_app gdroid_app;   /* opaque; owns device memory */
+
+/* One app's ICFG (Alg. 2 l.1 h_icfg/h_stmt) plus the
+ * pre-determined slot and instance pools.
+ * Slot gids: locals method-major (local_base[m] + i, params first, RET last),
+ * then statics (L_total + g), then heap slots
+ * (L_total + n_statics + heap_base[o] + ordinal of f in F(t(o))). */
+typedef struct {
+  uint32_t abi_version;      /* must be GDROID_ABI_VERSION */
+  uint32_t n_nodes, n_methods, n_modules, n_types, n_instances, n_statics, n_fields, n_entries;
+  uint64_t n_edges;
+  const uint64_t* row_ptr;   /* [n_nodes+1] CSR over node ids                               */
+  const uint32_t* col;       /* [n_edges]   successor node id                               */
+  const uint8_t*  edge_kind; /* [n_edges]   gdroid_edge_kind                                */
+  const uint8_t*  node_kind; /* [n_nodes]   gdroid_node_kind                                */
+  const uint32_t* node_method;/* [n_nodes]                                                  */
+  const int32_t*  node_ops;  /* [n_nodes*4] {op0 lhs slot gid, op1 rhs slot gid, op2 field,
+                                op3 instance gid | RETSITE: its CALL node}; -1 = none.
+                                FLOAD v=w.f: op0=v, op1=w.  FSTORE v.f=w: op0=v, op1=w.
+                                SSTORE g=w: op0=g.  RETV w: op1=w.  CALL/RETSITE: op0=lhs. */
+  const uint64_t* call_arg_ptr;/* [n_nodes+1] CSR of actual args per CALL node             */
+  const int32_t*  call_args; /* local slot gid of the actual, -1 = non-reference actual      */
+  const uint32_t* method_entry, *method_exit, *method_module, *method_n_locals, *method_n_params;
+  const uint64_t* module_inst_ptr; const uint32_t* module_insts;     /* sorted, contains 0 */
+  const uint64_t* module_static_ptr; const uint32_t* module_statics; /* sorted static ids  */
+  const int32_t*  inst_type;  /* [n_instances]; -1 only for instance 0 = NULL              */
+  const uint64_t* type_field_ptr; const uint32_t* type_fields;       /* sorted field ids   */
+  const uint32_t* entries;    /* [n_entries] ENTRY nodes of component environment methods  */
+} gdroid_icfg_desc;
+
+/* Build options; an all-zero struct (or NULL) means defaults. */
+typedef struct {
+  uint32_t async;        /* 1: enqueue only, complete with gdroid_sync                      */
+  uint32_t max_rounds;   /* 0 = unlimited                                                   */
+  uint32_t blocks;       /* persistent-kernel CTAs (0 = SMs x occupancy)                     */
+  uint32_t loop_mode;    /* 0 = persistent cooperative kernel (default), 1 = host-launched
+                            round kernels (one launch per round)                            */
+} gdroid_build_opts;
+
+/* Device-counted statistics of the last build (DESIGN.md §5 byte models). */
+typedef struct {
+  uint64_t rounds;        /* worklist iterations (device rounds)                            */
+  uint64_t node_visits;   /* nodes processed, summed over rounds (Alg. 1 pops)               */
+  uint64_t alg_bytes;     /* touched-word byte model, summed over visits     */
+  uint64_t dense_bytes;   /* dense MAT byte model, summed over visits                        */
+  uint64_t atomics;       /* 64-bit atomicOr issued into successor in-sets                   */
+  uint64_t hist[3];       /* rounds with frontier <= 32, 33..64, > 64 (Table II buckets)     */
+  uint64_t build_ns;      /* CUDA-event time of the build (zero + fixed point + digest)      */
+  uint64_t fixpoint_ns;   /* CUDA-event time of the fixed-point kernel(s) alone              */
+  uint64_t h2d_ns;        /* host time of the load's upload                                  */
+  uint64_t fact_bytes;    /* size of the device fact store                                   */
+  uint64_t kernel_launches; /* kernels launched by the last build                            */
+} gdroid_build_stats;
+
+/* Load one app (= a batch of one). */
+gdroid_status gdroid_load_icfg(const gdroid_icfg_desc* desc, int device, void* cuda_stream,
+                               gdroid_app** out);
+/* Load n_apps independent apps into ONE handle; they share every device round
+ * (IDFG-instance batching).  Node ids, slot gids and digests stay
+ * per app. */
+gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, int device,
+                                void* cuda_stream, gdroid_app** out);
+/* Zero the fact store, seed the entries, run the fixed point, compute digests. */
+gdroid_status gdroid_build_idfg(gdroid_app* app, const gdroid_build_opts* opts,
+                                gdroid_build_stats* stats);
+gdroid_status gdroid_sync(gdroid_app* app, gdroid_build_stats* stats);
+/* Facts of one node of app k as strictly ascending (slot_gid << 32 | inst_gid).
+ * pairs == NULL: size query.  cap < needed: GDROID_E_SMALLBUF with *n_pairs set. */
+gdroid_status gdroid_read_facts(const gdroid_app* app, uint32_t node, uint64_t* pairs,
+                                uint64_t cap, uint64_t* n_pairs);
+gdroid_status gdroid_read_facts_in(const gdroid_app* app, uint32_t k, uint32_t node,
+                                   uint64_t* pairs, uint64_t cap, uint64_t* n_pairs);
+/* All facts of app k: ptr[n_nodes+1] and pairs (two-call: pairs == NULL fills ptr only). */
+gdroid_status gdroid_read_all_facts(const gdroid_app* app, uint32_t k, uint64_t* ptr,
+                                    uint64_t* pairs, uint64_t cap);
+/* Per-node digests d(n) = sum over IN(n) of mix64(mix64(n) ^ pair),
+ * computed on the device at the end of the build; per_node may be NULL. */
+gdroid_status gdroid_node_digests(const gdroid_app* app, uint64_t* per_node, uint64_t* app_digest);
+gdroid_status gdroid_app_digests(const gdroid_app* app, uint64_t* per_app /* [n_apps] */);
+uint32_t      gdroid_n_apps(const gdroid_app* app);
+void          gdroid_free(gdroid_app* app);
+const char*   gdroid_last_error(void);   /* thread-local; valid until the next call */
+uint32_t      gdroid_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

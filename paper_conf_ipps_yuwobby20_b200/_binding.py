@@ -1,0 +1,193 @@
+"""ctypes binding of libgdroid.so — argument marshalling only.
+
+Every step of the IDFG construction runs in the CUDA kernels behind the C ABI
+(include/gdroid.h).  There is no CPU fallback: if the library is missing or no
+CUDA device is usable, the calls raise.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from typing import List, Optional, Sequence, Tuple, Union
+
+import numpy as np
+
+from ._build import LIB
+
+ABI_VERSION = 1
+STATUS = {0: "OK", -1: "E_INVALID", -2: "E_POOL", -3: "E_OOM", -4: "E_CUDA", -5: "E_STATE",
+          -6: "E_RANGE", -7: "E_SMALLBUF", -8: "E_LIMIT"}
+
+_ARRAYS = ("row_ptr", "col", "edge_kind", "node_kind", "node_method", "node_ops", "call_arg_ptr",
+           "call_args", "method_entry", "method_exit", "method_module", "method_n_locals",
+           "method_n_params", "module_inst_ptr", "module_insts", "module_static_ptr",
+           "module_statics", "inst_type", "type_field_ptr", "type_fields", "entries")
+
+
+class IcfgDesc(C.Structure):
+    _fields_ = [("abi_version", C.c_uint32)] + \
+        [(n, C.c_uint32) for n in ("n_nodes", "n_methods", "n_modules", "n_types", "n_instances",
+                                    "n_statics", "n_fields", "n_entries")] + \
+        [("n_edges", C.c_uint64)] + [(n, C.c_void_p) for n in _ARRAYS]
+
+
+class BuildOpts(C.Structure):
+    _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
+                ("loop_mode", C.c_uint32)]
+
+
+class BuildStats(C.Structure):
+    _fields_ = [("rounds", C.c_uint64), ("node_visits", C.c_uint64), ("alg_bytes", C.c_uint64),
+                ("dense_bytes", C.c_uint64), ("atomics", C.c_uint64), ("hist", C.c_uint64 * 3),
+                ("build_ns", C.c_uint64), ("fixpoint_ns", C.c_uint64), ("h2d_ns", C.c_uint64),
+                ("fact_bytes", C.c_uint64), ("kernel_launches", C.c_uint64)]
+
+    def as_dict(self) -> dict:
+        d = {k: int(getattr(self, k)) for k, _ in self._fields_ if k != "hist"}
+        d["hist"] = [int(x) for x in self.hist]
+        return d
+
+
+class GdroidError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"gdroid {STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+_lib = None
+
+
+def lib():
+    """Load the in-tree libgdroid.so (raises if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB):
+            raise RuntimeError(f"{LIB} is missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+        L = C.CDLL(LIB)
+        P = C.c_void_p
+        L.gdroid_load_batch.argtypes = [P, C.c_uint32, C.c_int, P, C.POINTER(P)]
+        L.gdroid_load_icfg.argtypes = [P, C.c_int, P, C.POINTER(P)]
+        L.gdroid_build_idfg.argtypes = [P, P, P]
+        L.gdroid_sync.argtypes = [P, P]
+        L.gdroid_read_facts.argtypes = [P, C.c_uint32, P, C.c_uint64, P]
+        L.gdroid_read_facts_in.argtypes = [P, C.c_uint32, C.c_uint32, P, C.c_uint64, P]
+        L.gdroid_read_all_facts.argtypes = [P, C.c_uint32, P, P, C.c_uint64]
+        L.gdroid_node_digests.argtypes = [P, P, P]
+        L.gdroid_app_digests.argtypes = [P, P]
+        L.gdroid_n_apps.argtypes = [P]
+        L.gdroid_n_apps.restype = C.c_uint32
+        L.gdroid_free.argtypes = [P]
+        L.gdroid_free.restype = None
+        L.gdroid_last_error.restype = C.c_char_p
+        L.gdroid_abi_version.restype = C.c_uint32
+        for f in ("gdroid_load_batch", "gdroid_load_icfg", "gdroid_build_idfg", "gdroid_sync",
+                  "gdroid_read_facts", "gdroid_read_facts_in", "gdroid_read_all_facts",
+                  "gdroid_node_digests", "gdroid_app_digests"):
+            getattr(L, f).restype = C.c_int
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise GdroidError(rc, lib().gdroid_last_error().decode())
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(C.c_void_p) if a.size else None
+
+
+def make_desc(g) -> Tuple[IcfgDesc, list]:
+    """Marshal an Icfg-like object (synth.Icfg) into a gdroid_icfg_desc; returns (desc, keepalive)."""
+    d = IcfgDesc()
+    d.abi_version = ABI_VERSION
+    d.n_nodes, d.n_methods, d.n_modules = g.n_nodes, g.n_methods, g.n_modules
+    d.n_types, d.n_instances, d.n_statics = g.n_types, g.n_instances, g.n_statics
+    d.n_fields, d.n_entries, d.n_edges = g.n_fields, g.n_entries, g.n_edges
+    keep = []
+    for nm in _ARRAYS:
+        a = np.ascontiguousarray(getattr(g, nm))
+        keep.append(a)
+        setattr(d, nm, _ptr(a))
+    return d, keep
+
+
+class App:
+    """A loaded batch of one or more apps on one device (owns device memory)."""
+
+    def __init__(self, icfgs: Union[object, Sequence[object]], device: int = 0, stream: int = 0):
+        if not isinstance(icfgs, (list, tuple)):
+            icfgs = [icfgs]
+        L = lib()
+        n = len(icfgs)
+        arr = (IcfgDesc * n)()
+        keep = []
+        for i, g in enumerate(icfgs):
+            d, k = make_desc(g)
+            arr[i] = d
+            keep.append(k)
+        self._h = C.c_void_p()
+        _check(L.gdroid_load_batch(C.cast(arr, C.c_void_p), n, device, C.c_void_p(stream),
+                                   C.byref(self._h)))
+        self.n_apps = n
+        self.n_nodes = [g.n_nodes for g in icfgs]
+        self.stats: Optional[dict] = None
+
+    def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
+              asynchronous: bool = False) -> Optional[dict]:
+        o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode)
+        s = BuildStats()
+        _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
+        if asynchronous:
+            return None
+        self.stats = s.as_dict()
+        return self.stats
+
+    def sync(self) -> dict:
+        s = BuildStats()
+        _check(lib().gdroid_sync(self._h, C.byref(s)))
+        self.stats = s.as_dict()
+        return self.stats
+
+    def read_facts(self, node: int, k: int = 0) -> np.ndarray:
+        L = lib()
+        cnt = C.c_uint64(0)
+        _check(L.gdroid_read_facts_in(self._h, k, node, None, 0, C.byref(cnt)))
+        out = np.zeros(max(cnt.value, 1), dtype=np.uint64)
+        _check(L.gdroid_read_facts_in(self._h, k, node, _ptr(out), cnt.value, C.byref(cnt)))
+        return out[:cnt.value]
+
+    def read_all_facts(self, k: int = 0) -> Tuple[np.ndarray, np.ndarray]:
+        L = lib()
+        ptr = np.zeros(self.n_nodes[k] + 1, dtype=np.uint64)
+        _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), None, 0))
+        tot = int(ptr[-1])
+        pairs = np.zeros(max(tot, 1), dtype=np.uint64)
+        _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), _ptr(pairs), tot))
+        return ptr, pairs[:tot]
+
+    def node_digests(self) -> Tuple[np.ndarray, int]:
+        per = np.zeros(self.n_nodes[0], dtype=np.uint64)
+        app = C.c_uint64(0)
+        _check(lib().gdroid_node_digests(self._h, _ptr(per), C.byref(app)))
+        return per, int(app.value)
+
+    def app_digests(self) -> np.ndarray:
+        out = np.zeros(self.n_apps, dtype=np.uint64)
+        _check(lib().gdroid_app_digests(self._h, _ptr(out)))
+        return out
+
+    def free(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            lib().gdroid_free(self._h)
+            self._h = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def load(icfgs, device: int = 0, stream: int = 0) -> App:
+    return App(icfgs, device=device, stream=stream)

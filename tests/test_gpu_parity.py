@@ -1,0 +1,128 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact per node.
+
+Exactly one result is correct (the least fixed point is unique, DESIGN.md §3 C4), so every
+node's fact set must equal the oracle's pair for pair; digests must match too.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_yuwobby20_b200 as gd
+from programs import fig2, load_expected, tiny, tiny2
+from synth import random_tiny
+from synth.reductions import random_inline_pair, random_rd, random_ssa_loop
+
+pytestmark = pytest.mark.gpu
+
+
+def _assert_same(app, k, g, r, label=""):
+    ptr, pairs = app.read_all_facts(k)
+    if not (np.array_equal(ptr, r.ptr) and np.array_equal(pairs, r.pairs)):
+        for n in range(g.n_nodes):
+            a = set(pairs[ptr[n]:ptr[n + 1]].tolist())
+            b = set(r.facts(n).tolist())
+            assert a == b, f"{label} node {n}: gpu-only {sorted(a - b)[:8]} oracle-only {sorted(b - a)[:8]}"
+        raise AssertionError(f"{label}: CSR layout differs")
+
+
+@pytest.mark.parametrize("which", ["tiny", "tiny_m2", "tiny2", "fig2"])
+def test_golden_programs(which):
+    if which == "fig2":
+        g = fig2()[0]
+    elif which == "tiny2":
+        g, L, slots, insts = tiny2()
+    else:
+        g, L, slots, insts = tiny(m2_entry=(which == "tiny_m2"))
+    app = gd.load(g)
+    st = app.build()
+    r = oracle.build_idfg(g)
+    _assert_same(app, 0, g, r, which)
+    per, dig = app.node_digests()
+    assert dig == r.app_digest and np.array_equal(per, r.node_digest)
+    assert st["rounds"] > 0 and st["node_visits"] > 0
+    if which != "fig2":      # and against the hand-computed fixture directly
+        exp = load_expected(which)
+        inv_s = {v: k for k, v in slots.items()}
+        inv_i = {v: k for k, v in insts.items()}
+        for lab, n in L.items():
+            got = {(inv_s[int(p) >> 32], inv_i[int(p) & 0xFFFFFFFF]) for p in app.read_facts(n)}
+            assert got == exp[lab], lab
+
+
+@pytest.mark.parametrize("chunk", range(4))
+def test_random_tiny_batches(chunk):
+    """600 seeded random tiny ICFGs (every node/edge kind, recursion, projection), batched
+    into one handle (shared device rounds), each compared with its own oracle run."""
+    seeds = range(chunk * 150, chunk * 150 + 150)
+    gs = [random_tiny(s) for s in seeds]
+    app = gd.load(gs)
+    app.build()
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        _assert_same(app, k, g, r, g.name)
+        assert int(digs[k]) == r.app_digest
+
+
+def test_reduction_programs_batch():
+    gs = [random_rd(s) for s in range(100)] + [random_ssa_loop(s)[0] for s in range(100)]
+    for s in range(60):
+        P, Q, _, _ = random_inline_pair(s)
+        gs += [P, Q]
+    app = gd.load(gs)
+    app.build()
+    for k, g in enumerate(gs):
+        _assert_same(app, k, g, oracle.build_idfg(g), g.name)
+
+
+def test_loop_modes_and_rebuild_identical():
+    gs = [random_tiny(s, max_stmts=7) for s in range(1000, 1100)]
+    app = gd.load(gs)
+    s0 = app.build(loop_mode=0)
+    d0 = app.app_digests().copy()
+    s1 = app.build(loop_mode=1)
+    d1 = app.app_digests().copy()
+    s2 = app.build(loop_mode=0, blocks=3)      # few CTAs: many nodes per warp per round
+    d2 = app.app_digests().copy()
+    assert np.array_equal(d0, d1) and np.array_equal(d0, d2)
+    assert s1["kernel_launches"] > s0["kernel_launches"]
+    for k in (0, 17, 99):
+        _assert_same(app, k, gs[k], oracle.build_idfg(gs[k]))
+
+
+def test_async_build_and_errors():
+    g = tiny()[0]
+    app = gd.load(g)
+    with pytest.raises(gd.GdroidError) as e:
+        app.read_facts(0)                    # before any build
+    assert e.value.code == -5
+    assert app.build(asynchronous=True) is None
+    with pytest.raises(gd.GdroidError):
+        app.build()                          # still pending
+    st = app.sync()
+    assert st["rounds"] > 0
+    with pytest.raises(gd.GdroidError) as e:
+        app.read_facts(g.n_nodes)
+    assert e.value.code == -6
+    with pytest.raises(gd.GdroidError) as e:
+        app.build(max_rounds=2)
+    assert e.value.code == -8
+
+
+def test_empty_and_degenerate():
+    """Degenerate inputs: a method whose entry has no successor; an app whose only entry
+    reaches nothing; unreachable methods (A5) keep empty sets."""
+    from synth import IcfgBuilder
+    b = IcfgBuilder(n_fields=1)
+    d = b.add_module()
+    m = b.add_method(d, 0, 1)           # entry and exit, no edge between them
+    b.add_entry(m)
+    g = b.build()
+    app = gd.load(g)
+    app.build()
+    ptr, pairs = app.read_all_facts(0)
+    assert len(pairs) == 0
+    r = oracle.build_idfg(g)
+    assert r.app_digest == app.node_digests()[1] == 0

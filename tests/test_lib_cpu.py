@@ -1,0 +1,77 @@
+"""CPU-side checks of the C-ABI library (no GPU needed): it loads, exports every symbol that
+include/gdroid.h declares, and its loader rejects invalid inputs with the documented status
+before touching the device."""
+from __future__ import annotations
+
+import copy
+import ctypes as C
+import os
+import re
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_yuwobby20_b200 as gd
+from paper_conf_ipps_yuwobby20_b200._binding import GdroidError
+from programs import tiny, tiny2
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    src = open(os.path.join(ROOT, "include", "gdroid.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(gdroid_[a-z_]+)\s*\(", src)))
+
+
+def test_header_symbols_exported():
+    L = gd.lib()
+    names = declared_functions()
+    assert len(names) >= 12
+    for nm in names:
+        assert hasattr(L, nm), nm
+    assert L.gdroid_abi_version() == 1
+
+
+def _load_status(g):
+    try:
+        gd.load(g)
+    except GdroidError as e:
+        return e.code
+    return 0
+
+
+def _mut(g, **kw):
+    h = copy.deepcopy(g)
+    for k, v in kw.items():
+        setattr(h, k, v)
+    return h
+
+
+def test_loader_rejects_invalid():
+    g = tiny()[0]
+    # arity mismatch (V6)
+    mp = g.method_n_params.copy(); mp[1] = 2
+    ml = g.method_n_locals.copy(); ml[1] = 4
+    assert _load_status(_mut(g, method_n_params=mp, method_n_locals=ml)) == -1
+    # NEW site outside its module pool (V1)
+    mi = g.module_insts[g.module_insts != 3].copy()
+    assert _load_status(_mut(g, module_insts=mi, module_inst_ptr=np.array([0, len(mi)], np.uint64))) == -2
+    # static not visible (V2)
+    assert _load_status(_mut(g, module_statics=np.zeros(0, np.uint32),
+                             module_static_ptr=np.array([0, 0], np.uint64))) == -2
+    # operand local of another method (V4)
+    ops = g.node_ops.copy(); ops[9, 1] = 6     # n5: z = x  ->  z = t (a local of m1)
+    assert _load_status(_mut(g, node_ops=ops)) == -2
+    # RET edge re-targeted to a non-RETSITE (V5)
+    ek = g.edge_kind.copy(); col = g.col.copy()
+    e = int(np.nonzero(ek == 2)[0][0]); col[e] = 7
+    assert _load_status(_mut(g, col=col)) == -1
+    # CSR not monotone
+    rp = g.row_ptr.copy(); rp[3], rp[4] = rp[4], rp[3]
+    if rp[3] > rp[4]:
+        assert _load_status(_mut(g, row_ptr=rp)) == -1
+    # pool without NULL
+    g2 = tiny2()[0]
+    mi2 = g2.module_insts.copy(); mi2[0] = 1
+    assert _load_status(_mut(g2, module_insts=mi2)) in (-1, -2)
