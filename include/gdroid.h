@@ -140,6 +140,11 @@ gdroid_status gdroid_read_all_facts(const gdroid_app* app, uint32_t k, uint64_t*
 gdroid_status gdroid_node_digests(const gdroid_app* app, uint64_t* per_node, uint64_t* app_digest);
 gdroid_status gdroid_app_digests(const gdroid_app* app, uint64_t* per_app /* [n_apps] */);
 uint32_t      gdroid_n_apps(const gdroid_app* app);
+/* Diagnostics: record a per-round trace in the next builds (cap rounds, 0 = off), then read
+ * it back as pairs {globaltimer ns at round start, items << 32 | nodes}; *n = rounds recorded
+ * (the last entry, with 0 items, marks the end of the fixed point). */
+gdroid_status gdroid_debug_trace(gdroid_app* app, uint32_t cap);
+gdroid_status gdroid_debug_read_trace(const gdroid_app* app, uint64_t* out, uint64_t cap, uint64_t* n);
 void          gdroid_free(gdroid_app* app);
 const char*   gdroid_last_error(void);   /* thread-local; valid until the next call */
 uint32_t      gdroid_abi_version(void);

@@ -14,6 +14,8 @@
 #include <cstdio>
 #include <cstring>
 #include <deque>
+#include <queue>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -404,12 +406,15 @@ int oracle_build(const oracle_icfg* g, int order, uint64_t seed, oracle_result**
   R->visited.assign(N, 0);
   std::vector<char> in_wl(N, 0);
   std::deque<uint32_t> wl;                     // l.8
+  std::priority_queue<uint32_t, std::vector<uint32_t>, std::greater<uint32_t>> pq;   // order 3
+  auto push = [&](uint32_t x) { if (order == 3) pq.push(x); else wl.push_back(x); in_wl[x] = 1; };
   for (uint32_t i = 0; i < g->n_entries; ++i)  // l.9: worklist <- entry
-    if (!in_wl[g->entries[i]]) { wl.push_back(g->entries[i]); in_wl[g->entries[i]] = 1; }
+    if (!in_wl[g->entries[i]]) push(g->entries[i]);
   uint64_t rng = seed * 0x9e3779b97f4a7c15ULL + 1;
-  while (!wl.empty()) {                        // l.10
+  while (!wl.empty() || !pq.empty()) {         // l.10
     uint32_t n;
-    if (order == 1) { n = wl.back(); wl.pop_back(); }
+    if (order == 3) { n = pq.top(); pq.pop(); }
+    else if (order == 1) { n = wl.back(); wl.pop_back(); }
     else if (order == 2) {
       rng ^= rng << 13; rng ^= rng >> 7; rng ^= rng << 17;
       size_t i = (size_t)(rng % wl.size());
@@ -423,7 +428,7 @@ int oracle_build(const oracle_icfg* g, int order, uint64_t seed, oracle_result**
       uint32_t s = g->col[e];
       PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
       bool grew = merge_union(R->IN[s], Z);    // union + update()
-      if ((grew || !R->visited[s]) && !in_wl[s]) { wl.push_back(s); in_wl[s] = 1; }  // l.13-14
+      if ((grew || !R->visited[s]) && !in_wl[s]) push(s);  // l.13-14
     }
   }
   R->seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();

@@ -39,7 +39,7 @@ typedef struct {
 
 typedef struct oracle_result oracle_result;
 
-/* order: 0 = FIFO (Alg. 1), 1 = LIFO, 2 = seeded uniform-random pop.
+/* order: 0 = FIFO (Alg. 1), 1 = LIFO, 2 = seeded uniform-random pop, 3 = smallest node id first.
  * Returns 0 on success, -1 invalid structure (V5/V6), -2 pool violation (V1-V4). */
 int oracle_build(const oracle_icfg* g, int order, uint64_t seed, oracle_result** out);
 void oracle_free(oracle_result* r);

@@ -76,6 +76,10 @@ def lib():
         L.gdroid_app_digests.argtypes = [P, P]
         L.gdroid_n_apps.argtypes = [P]
         L.gdroid_n_apps.restype = C.c_uint32
+        L.gdroid_debug_trace.argtypes = [P, C.c_uint32]
+        L.gdroid_debug_read_trace.argtypes = [P, P, C.c_uint64, P]
+        L.gdroid_debug_trace.restype = C.c_int
+        L.gdroid_debug_read_trace.restype = C.c_int
         L.gdroid_free.argtypes = [P]
         L.gdroid_free.restype = None
         L.gdroid_last_error.restype = C.c_char_p
@@ -176,6 +180,18 @@ class App:
         out = np.zeros(self.n_apps, dtype=np.uint64)
         _check(lib().gdroid_app_digests(self._h, _ptr(out)))
         return out
+
+    def set_trace(self, cap: int):
+        _check(lib().gdroid_debug_trace(self._h, cap))
+
+    def read_trace(self) -> np.ndarray:
+        """Per-round (start ns, items, nodes) of the last build (diagnostics)."""
+        n = C.c_uint64(0)
+        _check(lib().gdroid_debug_read_trace(self._h, None, 0, C.byref(n)))
+        buf = np.zeros(2 * max(n.value, 1), dtype=np.uint64)
+        _check(lib().gdroid_debug_read_trace(self._h, _ptr(buf), buf.size, C.byref(n)))
+        t = buf.reshape(-1, 2)[:n.value]
+        return np.stack([t[:, 0], t[:, 1] >> 32, t[:, 1] & 0xFFFFFFFF], axis=1)
 
     def free(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -11,25 +11,52 @@ namespace gd {
 constexpr int MAXW = 8;            // max 64-bit words per fact row: |Q_m| <= 512 instances
 constexpr int NCLS = 5;            // GRP classes + 2 interprocedural classes
 enum Cls : uint8_t { C_ONETIME = 0, C_SINGLE = 1, C_DOUBLE = 2, C_CALL = 3, C_EXIT = 4 };
-constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]
+constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]; slot CNT_NODES = nodes queued
+constexpr int CNT_NODES = 5;
 constexpr int THREADS = 256;       // fixed-point kernel block size
 constexpr int WARPS = THREADS / 32;
 
-// One ICFG node (32 B, one sector).  Row indices r* are relative to the node's fact block
-// (method-local rows first, then the module's global rows), resolved by the loader.
+// One ICFG node (64 B).  Row indices r* are relative to the node's fact block (method-local
+// rows first, then the module's global rows), resolved by the loader, and the block's layout
+// is copied in so a visit needs no method/module lookups.
 struct __align__(16) NodeRec {
   uint64_t off;      // word offset of IN(n) in the fact store
-  uint32_t method;   // global method index
+  uint32_t e0, e1;   // out-edge range [e0, e1) in the edge array
   uint8_t kind;      // gdroid_node_kind
   uint8_t cls;       // Cls
-  uint16_t app;      // index of the app inside a batch
+  uint8_t logW;      // log2 words per row
+  uint8_t pad;
   int32_t r0;        // lhs row (PRIM/CONST/NEW/COPY/SLOAD/RETV/FLOAD/ALOAD), static row (SSTORE),
                      // base row (FSTORE/ASTORE), lhs row of the call (CALL/RETSITE) or -1
-  int32_t r1;        // rhs row (COPY/SLOAD/SSTORE/RETV), w row (FLOAD/ALOAD/FSTORE/ASTORE)
+  int32_t r1;        // rhs row (COPY/SLOAD/SSTORE/RETV), w row (FLOAD/ALOAD/FSTORE/ASTORE),
+                     // n_params of the method (ENTRY), argument rows r1..r3 (CALL with <= 3 args)
   int32_t r2;        // field id (FLOAD/FSTORE; F_ARR for ALOAD/ASTORE)
-  int32_t r3;        // instance column (CONST/NEW)
+  int32_t r3;        // instance column (CONST/NEW); field-row table offset (FLOAD/ALOAD)
+  uint32_t B;        // words of the block = (L + n_glob) << logW
+  uint32_t L;        // method-local rows (params, temps, RET)
+  uint32_t n_stat;   // module static rows
+  uint32_t col_off;  // module column tables
+  uint32_t grow_off; // module global-row tables
+  uint16_t n_cols;   // |Q| of the module
+  uint16_t app;      // index of the app inside a batch
+  uint32_t module;   // global module index
 };
-static_assert(sizeof(NodeRec) == 32, "NodeRec must be 32 bytes");
+static_assert(sizeof(NodeRec) == 64, "NodeRec must be 64 bytes");
+
+// Work items.  A node's out-edges are split into chunks of ebs(deg) edges (at most 32 chunks
+// per node); a queue entry is (node << 5) | chunk.  High-degree nodes (method exits with many
+// return sites, virtual calls with many targets) thus spread over several warps.
+// INTRA/C2R edges share one transfer evaluation, so their chunks hold up to 4 edges; CALL
+// and RET edges each re-map the whole block, so CALL and EXIT nodes get one edge per chunk.
+constexpr uint32_t EDGES_PER_CHUNK = 4;
+__host__ __device__ __forceinline__ uint32_t chunk_edges(uint32_t deg, uint32_t cls) {
+  const uint32_t e = (deg + 31) >> 5;
+  const uint32_t lo = (cls == 3u || cls == 4u) ? 1u : EDGES_PER_CHUNK;   // C_CALL, C_EXIT
+  return e > lo ? e : lo;
+}
+__host__ __device__ __forceinline__ uint32_t n_chunks_of(uint32_t deg, uint32_t cls) {
+  return deg == 0 ? 1u : (deg + chunk_edges(deg, cls) - 1) / chunk_edges(deg, cls);
+}
 
 struct __align__(16) MethRec {
   uint32_t n_locals, n_params, module, local_base;   // local_base: app-local slot gid of local 0
@@ -45,16 +72,22 @@ struct __align__(16) ModRec {
   uint32_t pad;
 };
 
-struct Edge {
+// One out-edge (32 B) with the destination's layout copied in, so a CALL/RET edge needs no
+// lookup of the destination node.
+struct __align__(16) Edge {
   uint32_t dst;
-  uint32_t info;       // kind (2 bits) | xlate id << 2 (0 = same module / identity)
+  uint32_t info;       // kind (2 bits) | class of dst << 2 (3 bits) | (chunks of dst - 1) << 5
+  uint64_t off;        // fact-block word offset of dst
+  uint32_t B;          // dst block words
+  uint16_t L;          // dst method-local rows
+  uint8_t logW;        // dst log2 words per row
+  uint8_t pad;
+  int32_t aux;         // CALL: n_params of the callee; RET: lhs(c) row at the return site (-1)
+  uint32_t xoff;       // projection π: xmap offset (colmap |Q_src| then rowmap n_glob(dst)),
+                       // 0xffffffff = same module (identity)
 };
-
-struct XRec {          // cross-module projection π (CALL/RET edges between modules)
-  uint32_t colmap_off; // colmap[c_src] -> c_dst or -1, |Q_src| entries
-  uint32_t rowmap_off; // rowmap[g_dst] -> g_src or -1, n_glob(dst) entries
-  uint32_t src_mod, dst_mod;
-};
+static_assert(sizeof(Edge) == 32, "Edge must be 32 bytes");
+constexpr uint32_t NO_XMAP = 0xffffffffu;
 
 struct DevStats {
   unsigned long long rounds, visits, alg_bytes, dense_bytes, atomics, hist[3], limit_hit, pad;
@@ -64,7 +97,6 @@ struct Dev {
   const NodeRec* nodes;
   const MethRec* meths;
   const ModRec* mods;
-  const XRec* xrecs;
   const uint32_t* row_ptr;
   const Edge* edges;
   const uint32_t* arg_ptr;
@@ -77,13 +109,15 @@ struct Dev {
   const int32_t* grow_field;
   const uint32_t* tf_ptr;
   const uint32_t* tf;
-  const int32_t* colmap;
-  const int32_t* rowmap;
+  const int32_t* xmap;          // projection tables (see Edge::xoff)
   const uint32_t* app_node_base;
   const uint32_t* entries;      // global node ids of all component entries of all apps
+  const uint32_t* node_method;  // [N] (digest / readback only)
+  const int32_t* frow;          // field-row tables: frow[r3 + c] = global row of (col c, f) | -1
   uint64_t* facts;
   uint32_t* stamp;              // [N] last round a node was queued for (0 = never)
-  uint32_t* queue;              // [3][N] rotating class-segmented worklists
+  uint32_t* queue;              // [3][n_chunks] rotating class-segmented worklists of
+                                // (node << 5 | chunk) entries
   uint32_t* counts;             // [3][CNT_STRIDE]
   DevStats* stats;
   uint32_t* bar;                // grid barrier {count, generation}
@@ -91,9 +125,12 @@ struct Dev {
   unsigned long long* app_digest; // [n_apps]
   uint64_t n_words;             // fact store size in words
   uint32_t n_nodes;
+  uint32_t n_chunks;
   uint32_t n_entries;
   uint32_t seg[NCLS + 1];       // class segment starts inside one queue
   uint32_t max_rounds;
+  unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
+  uint32_t trace_cap;           // rounds recorded (0 = off)
 };
 
 // kernels.cu launch wrappers (return cudaError_t of the launch)

@@ -1,45 +1,62 @@
-// kernels.cu — sm_100a kernels of the IDFG fixed point (DESIGN.md §4).
+// kernels.cu — sm_100a kernels of the IDFG fixed point (DESIGN.md §4-5).
 //
-// One warp processes one worklist node (Alg. 3 l.9-15): it reads the
-// node's fact block IN(src) (MAT) with coalesced 8-byte-per-lane loads,
-// applies the node's transfer function on the fly (GEN_KILL, Alg. 3 l.10), maps the result
-// through each out-edge (SEARCH, l.11; edge transforms of DESIGN.md §3 C3) and ORs it into
-// IN(dst) with 64-bit atomicOr, skipping words whose bits are already present (a plain,
-// possibly stale load first: IN only grows, so a stale read never hides a needed OR).
-// update() (l.14) = "some word gained a bit" (warp vote).  Destinations that grew, or were
-// never queued (first-reach rule, DESIGN.md §3 A5), are appended to the next round's
-// class-segmented worklist (GRP, l.7) behind a per-node round stamp (atomicMax test-and-set),
-// which de-duplicates exactly like MER's merge (Fig. 7).
+// One warp processes one work item = (node, chunk of its out-edges) (Alg. 3 l.9-15,
+// PAPER.md:751-766): it reads the node's fact block IN(src) (MAT) with
+// coalesced 8-byte-per-lane loads issued together with the edge records, applies the node's
+// transfer function on the fly (GEN_KILL, Alg. 3 l.10), maps the result through each out-edge
+// (SEARCH, l.11; edge transforms of DESIGN.md §3 C3) and ORs it into IN(dst) with
+// fire-and-forget 64-bit RED.OR, only for words whose bits are missing (a plain, possibly
+// stale load first: IN only grows, so a stale read never hides a needed OR, it can only
+// over-report growth, which costs a duplicate push).  update() (l.14) = "some word had a
+// missing bit" (warp vote).  Destinations that grew, or were never queued (first-reach rule,
+// DESIGN.md §3 A5), are appended to the next round's class-segmented worklist (GRP, l.7)
+// behind a per-node round stamp (atomicMax test-and-set) that de-duplicates like MER's merge
+// (Fig. 7).  Appends are staged per CTA in shared memory and published
+// with one global atomic per class per CTA at the end of the round.
 //
 // The round loop runs inside one persistent cooperative kernel with a grid barrier per
 // round (no host round trip), or as one launch per round (loop_mode 1).
-#include <cooperative_groups.h>
-
 #include "internal.cuh"
 
 namespace gd {
 namespace {
 
-constexpr unsigned FULL = 0xffffffffu;
+#ifndef GD_MINB
+#define GD_MINB 3              // resident CTAs per SM the fixed-point kernels are compiled for
+#endif
 
-struct Acc {              // per-lane counters, reduced once per kernel
-  unsigned long long nz;  // non-zero edge words written (x16 bytes in the touched model)
-  unsigned long long nzx; // non-zero IN(src) words read (x8)
-  unsigned long long h;   // heap words gathered by DOUBLE kinds (x8)
-  unsigned long long atom;
-  unsigned long long dense;   // dense-model bytes (lane 0 only)
-  unsigned long long fixed;   // per-visit constant bytes (lane 0 only)
+constexpr unsigned FULL = 0xffffffffu;
+constexpr int KW = 4;          // words per lane per chunk of a fact block (loads issued together)
+constexpr int SCAP = 448;      // staged queue entries per class per CTA (overflow goes global)
+
+struct Acc {                   // per-warp counters (shared memory), flushed once per kernel
+  unsigned long long alg;      // touched-word model bytes
+  unsigned long long dense;    // dense-model bytes
+  unsigned long long atom;     // RED.OR issued
 };
 
 struct WarpScratch {
-  uint64_t gen[MAXW];     // generated row (replace / or-in)
-  uint64_t rv[MAXW];      // FSTORE base row v
-  uint64_t rw[MAXW];      // FSTORE / FLOAD value row w
+  uint64_t rv[MAXW];           // FSTORE base row v
+  uint64_t rw[MAXW];           // FSTORE / FLOAD value row w
+  int16_t cmap[64 * MAXW];     // projection column map of the current cross-module edge
+};
+
+// warp-uniform counter updates: lane 0 adds the warp's total
+__device__ __forceinline__ void acc_add(unsigned long long& slot, uint32_t per_lane) {
+  const uint32_t t = __reduce_add_sync(FULL, per_lane);
+  if ((threadIdx.x & 31) == 0) slot += t;
+}
+
+struct CtaStage {              // per-CTA staged worklist appends of the current round
+  uint32_t cnt[NCLS];
+  uint32_t nodes;
+  uint32_t gbase[NCLS];
+  uint32_t buf[NCLS][SCAP];
 };
 
 __device__ __forceinline__ uint64_t warp_or64(uint64_t v) {
-  uint32_t lo = __reduce_or_sync(FULL, (uint32_t)v);
-  uint32_t hi = __reduce_or_sync(FULL, (uint32_t)(v >> 32));
+  const uint32_t lo = __reduce_or_sync(FULL, (uint32_t)v);
+  const uint32_t hi = __reduce_or_sync(FULL, (uint32_t)(v >> 32));
   return ((uint64_t)hi << 32) | lo;
 }
 
@@ -55,236 +72,370 @@ __device__ __forceinline__ uint64_t mix64(uint64_t z) {   // splitmix64 finalise
   return z ^ (z >> 31);
 }
 
-// global-part-relative row of heap slot (instance in column c, field f) or -1 (C1)
-__device__ __forceinline__ int heap_row_rel(const Dev& D, const ModRec& md, uint32_t c, uint32_t f) {
-  int t = D.col_type[md.col_off + c];
-  if (t < 0) return -1;
-  uint32_t a = D.tf_ptr[t], b = D.tf_ptr[t + 1];
-  for (uint32_t k = a; k < b; ++k)
-    if (D.tf[k] == f) return (int)(D.col_hbase[md.col_off + c] + (k - a));
-  return -1;
+// ---------------------------------------------------------------------------------- pushes
+__device__ __forceinline__ void stage_init(CtaStage& st) {
+  if (threadIdx.x < NCLS) st.cnt[threadIdx.x] = 0;
+  if (threadIdx.x == NCLS) st.nodes = 0;
 }
 
-// IN(dst)[w] |= y; returns whether IN(dst) gained a bit (update(), A6)
-__device__ __forceinline__ bool or_into(uint64_t* p, uint64_t y, Acc& acc) {
-  if (!y) return false;
-  acc.nz++;
-  uint64_t cur = *p;                  // may be stale (subset of the truth): safe
-  if (!(y & ~cur)) return false;
-  uint64_t old = atomicOr((unsigned long long*)p, (unsigned long long)y);
-  acc.atom++;
-  return (y & ~old) != 0;
-}
-
-// Y[w] = f_src(X)[w] (DESIGN.md §3 C2), X[w] returned in x
-__device__ __forceinline__ uint64_t y_word(const Dev& D, const uint64_t* __restrict__ X, uint32_t w,
-                                           uint32_t logW, int mode, int t, uint32_t L,
-                                           const ModRec& md, uint32_t f, const WarpScratch& ws,
-                                           uint64_t& x) {
-  x = X[w];
-  if (mode == 0) return x;
-  const uint32_t r = w >> logW, j = w & ((1u << logW) - 1);
-  if (mode == 1) return (int)r == t ? ws.gen[j] : x;            // X \ K(v) ∪ gen
-  if (mode == 2) return (int)r == t ? (x | ws.gen[j]) : x;      // weak static store
-  if (r >= L + md.n_stat) {                                      // FSTORE: heap rows (o1, f)
-    const uint32_t g = r - L;
-    if (D.grow_field[md.grow_off + g] == (int)f) {
-      const int c = D.grow_col[md.grow_off + g];                 // o1 (never NULL)
-      if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) return x | ws.rw[j];
-    }
-  }
-  return x;
-}
-
-// Append the candidate destinations held by the warp's lanes to the next worklist.
-__device__ __forceinline__ void flush_pushes(const Dev& D, int lane, bool active, uint32_t dst,
-                                             bool grew, uint32_t round, uint32_t nxt) {
+// Append the candidate destinations held by the warp's lanes (every chunk of a pushed node)
+// to the CTA's staged worklist of the next round.
+__device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
+                                             uint32_t dst, uint32_t info, bool grew, uint32_t round,
+                                             uint32_t nxt) {
   bool push = false;
-  int cls = -1;
   if (active) {
-    bool want = grew || (D.stamp[dst] == 0);               // grew, or first reach (A5)
+    const bool want = grew || (D.stamp[dst] == 0);          // grew, or first reach (A5)
     if (want) {
-      uint32_t old = atomicMax(&D.stamp[dst], round + 1);  // test-and-set: de-duplicates (MER)
+      const uint32_t old = atomicMax(&D.stamp[dst], round + 1);  // test-and-set: de-duplicates (MER)
       push = old < round + 1;
     }
-    if (push) cls = D.nodes[dst].cls;
   }
+  const int cls = push ? (int)((info >> 2) & 7u) : -1;
+  const uint32_t nch = ((info >> 5) & 31u) + 1;
   unsigned pm = __ballot_sync(FULL, push);
-  while (pm) {                                             // warp-aggregated append per class
+  if (pm && lane == 0) atomicAdd(&st.nodes, (uint32_t)__popc(pm));
+  while (pm) {                                               // warp-aggregated append per class
     const int leader = __ffs(pm) - 1;
     const int c = __shfl_sync(FULL, cls, leader);
-    const unsigned same = __ballot_sync(FULL, push && cls == c);
+    const bool mine = push && cls == c;
+    const unsigned same = __ballot_sync(FULL, mine);
+    const uint32_t v = mine ? nch : 0u;
+    uint32_t incl = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(FULL, incl, o);
+      if (lane >= o) incl += t;
+    }
+    const uint32_t total = __shfl_sync(FULL, incl, 31);
     uint32_t base = 0;
-    if (lane == leader) base = atomicAdd(&D.counts[nxt * CNT_STRIDE + c], (uint32_t)__popc(same));
+    if (lane == leader) base = atomicAdd(&st.cnt[c], total);
     base = __shfl_sync(FULL, base, leader);
-    if (push && cls == c) {
-      const uint32_t rank = __popc(same & ((1u << lane) - 1));
-      D.queue[(size_t)nxt * D.n_nodes + D.seg[c] + base + rank] = dst;
+    if (mine) {
+      for (uint32_t q = 0; q < nch; ++q) {
+        const uint32_t idx = base + (incl - v) + q;
+        const uint32_t entry = (dst << 5) | q;
+        if (idx < (uint32_t)SCAP) st.buf[c][idx] = entry;
+        else {                                                 // stage full: publish directly
+          const uint32_t g = atomicAdd(&D.counts[nxt * CNT_STRIDE + c], 1u);
+          D.queue[(size_t)nxt * D.n_chunks + D.seg[c] + g] = entry;
+        }
+      }
     }
     pm &= ~same;
   }
 }
 
-// One worklist node, one warp (Alg. 3 l.9-15).
-__device__ void process_node(const Dev& D, uint32_t n, uint32_t round, uint32_t nxt, int lane,
-                             WarpScratch& ws, Acc& acc) {
-  const uint32_t e0 = D.row_ptr[n], e1 = D.row_ptr[n + 1];
-  if (lane == 0) acc.fixed += sizeof(NodeRec) + 8 + 8ull * (e1 - e0) + 8;
-  if (e0 == e1) return;                                    // no successor: nothing to propagate
+// Publish the CTA's staged appends (one global atomic per class), then reset the stage.
+__device__ __forceinline__ void stage_publish(const Dev& D, CtaStage& st, uint32_t nxt) {
+  __syncthreads();
+  if (threadIdx.x < NCLS) {
+    const uint32_t n = min(st.cnt[threadIdx.x], (uint32_t)SCAP);
+    st.gbase[threadIdx.x] = n ? atomicAdd(&D.counts[nxt * CNT_STRIDE + threadIdx.x], n) : 0u;
+  }
+  if (threadIdx.x == NCLS && st.nodes) atomicAdd(&D.counts[nxt * CNT_STRIDE + CNT_NODES], st.nodes);
+  __syncthreads();
+#pragma unroll
+  for (int c = 0; c < NCLS; ++c) {
+    const uint32_t n = min(st.cnt[c], (uint32_t)SCAP);
+    uint32_t* q = D.queue + (size_t)nxt * D.n_chunks + D.seg[c] + st.gbase[c];
+    for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) q[i] = st.buf[c][i];
+  }
+  __syncthreads();
+  stage_init(st);
+}
+
+// ---------------------------------------------------------------------------------- unions
+// OR KW words into IN(dst): a (possibly stale) load, then RED.OR only where bits are missing.
+// Words of row `kill` are dropped (C2R).  Returns the number of non-zero words in the low
+// 16 bits and the number of REDs issued in the high bits.
+__device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uint64_t (&y)[KW], uint32_t c0,
+                                             int lane, int kill, uint32_t logW) {
+  uint64_t cur[KW];
+#pragma unroll
+  for (int k = 0; k < KW; ++k) {
+    const uint32_t w = c0 + lane + 32 * k;
+    const bool keep = y[k] && !(kill >= 0 && (int)(w >> logW) == kill);
+    cur[k] = keep ? Z[w] : ~0ull;
+  }
+  uint32_t nz = 0, red = 0;
+#pragma unroll
+  for (int k = 0; k < KW; ++k) {
+    const uint32_t w = c0 + lane + 32 * k;
+    const uint64_t z = (kill >= 0 && (int)(w >> logW) == kill) ? 0ull : y[k];
+    nz += (z != 0);
+    if (z & ~cur[k]) {
+      atomicOr((unsigned long long*)(Z + w), (unsigned long long)z);
+      ++red;
+    }
+  }
+  return nz | (red << 16);
+}
+
+// ---------------------------------------------------------------------------------- one item
+__device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
+                             uint32_t nxt, int lane, WarpScratch& ws, Acc& acc) {
   const NodeRec R = D.nodes[n];
-  const MethRec mr = D.meths[R.method];
-  const ModRec md = D.mods[mr.module];
-  const uint32_t logW = md.logW, W = md.W, L = mr.n_locals;
-  const uint32_t B = (L + md.n_glob) << logW;
+  const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
+  const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
+  const bool first = ci == 0;
+  const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B;
+  uint32_t alg_l0 = (first ? (uint32_t)sizeof(NodeRec) : 0u) + (uint32_t)sizeof(Edge) * (e1 - e0) + 4u;
+  if (e0 >= e1) {                                           // no successor: nothing to propagate
+    if (lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
+    return;
+  }
   const uint64_t* __restrict__ X = D.facts + R.off;
 
-  // ---- GEN_KILL setup (a4): mode 0 identity, 1 replace row t, 2 or into row t, 3 FSTORE
-  int mode = 0, t = -1;
-  uint32_t f = 0;
-  switch (R.kind) {
-    case GK_PRIM:
-      mode = 1; t = R.r0;
-      if (lane < (int)W) ws.gen[lane] = 0;
-      break;
-    case GK_CONST: case GK_NEW:
-      mode = 1; t = R.r0;
-      if (lane < (int)W) ws.gen[lane] = ((R.r3 >> 6) == lane) ? (1ull << (R.r3 & 63)) : 0ull;
-      break;
-    case GK_COPY: case GK_SLOAD: case GK_RETV:
-      mode = 1; t = R.r0;
-      if (lane < (int)W) ws.gen[lane] = X[((uint64_t)R.r1 << logW) + lane];
-      break;
-    case GK_SSTORE:
-      mode = 2; t = R.r0;
-      if (lane < (int)W) ws.gen[lane] = X[((uint64_t)R.r1 << logW) + lane];
-      break;
-    case GK_FLOAD: case GK_ALOAD: {          // v = w.f: OR of heap rows (o1, f), o1 ∈ row w
-      mode = 1; t = R.r0; f = (uint32_t)R.r2;
-      if (lane < (int)W) ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
-      __syncwarp();
-      uint64_t a[MAXW];
+  // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
+  //      the rows the transfer function reads
+  const uint32_t ne0 = min(32u, e1 - e0);
+  Edge E{0, 0, 0};
+  if (lane < (int)ne0) E = D.edges[e0 + lane];
+  uint64_t y[KW];
 #pragma unroll
-      for (int j = 0; j < MAXW; ++j) a[j] = 0;
-      for (uint32_t c = lane; c < md.n_cols; c += 32) {
-        if (c == 0 || !((ws.rw[c >> 6] >> (c & 63)) & 1ull)) continue;   // NULL has no fields
-        const int hr = heap_row_rel(D, md, c, f);
-        if (hr < 0) continue;
-        const uint64_t* H = X + ((uint64_t)(L + hr) << logW);
-#pragma unroll
-        for (int j = 0; j < MAXW; ++j)
-          if (j < (int)W) a[j] |= H[j];
-        acc.h += W;
-      }
-#pragma unroll
-      for (int j = 0; j < MAXW; ++j) {
-        if (j < (int)W) {
-          const uint64_t v = warp_or64(a[j]);
-          if (lane == 0) ws.gen[j] = v;
-        }
-      }
-      break;
-    }
-    case GK_FSTORE: case GK_ASTORE:          // v.f = w (weak)
-      mode = 3; f = (uint32_t)R.r2;
-      if (lane < (int)W) {
-        ws.rv[lane] = X[((uint64_t)R.r0 << logW) + lane];
-        ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
-      }
-      break;
-    default:
-      break;                                 // NOP/ENTRY/EXIT/RETSITE/CALL: identity
+  for (int k = 0; k < KW; ++k) {
+    const uint32_t w = lane + 32 * k;
+    y[k] = (w < B) ? X[w] : 0ull;
   }
-  __syncwarp();
+  const uint32_t kind = R.kind;
+  int mode = 0, t = -1;                                     // 0 identity, 1 replace, 2 or-in, 3 FSTORE
+  uint32_t f = 0, hwords = 0;
+  uint64_t genv = 0;                                        // lane j < W: word j of the generated row
+  if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
+    mode = 1; t = R.r0;
+    if (kind != GK_PRIM && (R.r3 >> 6) == lane) genv = 1ull << (R.r3 & 63);
+  } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
+    mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
+    if (lane < (int)W) genv = X[((uint64_t)R.r1 << logW) + lane];
+  } else if (kind == GK_FLOAD || kind == GK_ALOAD) {       // v = w.f: OR of rows (o1,f), o1 ∈ w
+    mode = 1; t = R.r0;
+    if (lane < (int)W) ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
+    int hr[(64 * MAXW) / 32];                               // heap rows of this lane's columns
+#pragma unroll
+    for (int q = 0; q < (64 * MAXW) / 32; ++q) {
+      const uint32_t c = lane + 32 * q;
+      hr[q] = (c < R.n_cols) ? D.frow[R.r3 + c] : -1;
+    }
+    __syncwarp();
+    uint64_t a[MAXW];
+#pragma unroll
+    for (int j = 0; j < MAXW; ++j) a[j] = 0;
+#pragma unroll
+    for (int q = 0; q < (64 * MAXW) / 32; ++q) {
+      const uint32_t c = lane + 32 * q;
+      if (hr[q] < 0 || !((ws.rw[c >> 6] >> (c & 63)) & 1ull)) continue;   // NULL has no row
+      const uint64_t* H = X + ((uint64_t)(L + hr[q]) << logW);
+#pragma unroll
+      for (int j = 0; j < MAXW; ++j)
+        if (j < (int)W) a[j] |= H[j];
+      hwords += W;
+    }
+#pragma unroll
+    for (int j = 0; j < MAXW; ++j)
+      if (j < (int)W) {
+        const uint64_t v = warp_or64(a[j]);
+        if (lane == j) genv = v;
+      }
+  } else if (kind == GK_FSTORE || kind == GK_ASTORE) {     // v.f = w (weak)
+    mode = 3; f = (uint32_t)R.r2;
+    if (lane < (int)W) {
+      ws.rv[lane] = X[((uint64_t)R.r0 << logW) + lane];
+      ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
+    }
+    __syncwarp();
+  }
+  // every word w of this lane has column-word index j = w & (W-1) = lane & (W-1)
+  const uint64_t gsel = __shfl_sync(FULL, genv, lane & (W - 1));
+  const uint64_t rwsel = (mode == 3) ? ws.rw[lane & (W - 1)] : 0ull;
 
-  // ---- SEARCH + union/update over the out-edges (a5)
-  uint32_t cand_dst = 0;
-  bool cand_grew = false;
-  unsigned long long dense = 8ull * B + 8ull * acc.h;
-  for (uint32_t e = e0; e < e1; ++e) {
-    const Edge E = D.edges[e];
-    const uint32_t kind = E.info & 3u, xid = E.info >> 2;
-    const uint32_t dst = E.dst;
-    const NodeRec RD = D.nodes[dst];
-    uint64_t* Z = D.facts + RD.off;
-    const bool first = (e == e0);
-    bool grew = false;
-    if (kind == GE_INTRA || kind == GE_C2R) {
-      const int kill = (kind == GE_C2R) ? R.r0 : -1;       // C2R drops lhs(c)
-      for (uint32_t w = lane; w < B; w += 32) {
-        uint64_t x;
-        uint64_t y = y_word(D, X, w, logW, mode, t, L, md, f, ws, x);
-        if (first) acc.nzx += (x != 0);
-        if (kill >= 0 && (int)(w >> logW) == kill) y = 0;
-        grew |= or_into(Z + w, y, acc);
-      }
-      dense += 16ull * B;
-    } else if (xid == 0) {                                 // CALL / RET inside one module
-      const MethRec mt = D.meths[RD.method];
-      const uint32_t Lt = mt.n_locals, Bt = (Lt + md.n_glob) << logW;
-      const uint32_t a0 = (kind == GE_CALL) ? D.arg_ptr[n] : 0;
-      for (uint32_t w = lane; w < Bt; w += 32) {
-        const uint32_t r = w >> logW, j = w & (W - 1);
-        int src;
-        if (r < Lt) {
-          if (kind == GE_CALL) src = (r < mt.n_params) ? D.args[a0 + r] : -1;   // param_j <- arg_j
-          else src = ((int)r == RD.r0) ? (int)(L - 1) : -1;                   // lhs(c) <- RET
-        } else {
-          src = (int)(L + (r - Lt));                                           // globals
-        }
-        if (src < 0) continue;
-        const uint64_t y = X[((uint64_t)src << logW) + j];   // CALL/EXIT transfers are identity
-        if (first) acc.nzx += (y != 0);
-        grew |= or_into(Z + w, y, acc);
-      }
-      dense += 16ull * Bt;
-    } else {                                               // CALL / RET across modules: π
-      const XRec xr = D.xrecs[xid];
-      const MethRec mt = D.meths[RD.method];
-      const ModRec mdt = D.mods[mt.module];
-      const uint32_t Lt = mt.n_locals, rows_t = Lt + mdt.n_glob, logWt = mdt.logW;
-      const uint32_t a0 = (kind == GE_CALL) ? D.arg_ptr[n] : 0;
-      for (uint32_t r = lane; r < rows_t; r += 32) {
-        int src;
-        if (r < Lt) {
-          if (kind == GE_CALL) src = (r < mt.n_params) ? D.args[a0 + r] : -1;
-          else src = ((int)r == RD.r0) ? (int)(L - 1) : -1;
-        } else {
-          const int gs = D.rowmap[xr.rowmap_off + (r - Lt)];
-          src = gs < 0 ? -1 : (int)(L + gs);
-        }
-        if (src < 0) continue;
-        uint64_t out[MAXW];
+  uint32_t nzx = 0, nz = 0, red = 0;                        // per-lane counters of this item
+  unsigned long long dense_l0 = first ? 8ull * B : 0ull;
+  for (uint32_t eb = e0; eb < e1; eb += 32) {               // edges in batches of 32 (a5)
+    const uint32_t ne = min(32u, e1 - eb);
+    if (eb != e0) {
+      E = Edge{0, 0, 0};
+      if (lane < (int)ne) E = D.edges[eb + lane];
+    }
+    const uint32_t my_kind = E.info & 3u;
+    const unsigned live = __ballot_sync(FULL, lane < (int)ne);
+    const unsigned same = __ballot_sync(FULL, lane < (int)ne && (my_kind == GE_INTRA || my_kind == GE_C2R));
+    unsigned gmask = 0;
+    // -- INTRA / C2R: identical layouts; OUT computed once per chunk and reused by every edge
+    if (same) {
+      for (uint32_t c0 = 0; c0 < B; c0 += 32 * KW) {
+        if (c0 != 0 || eb != e0) {
 #pragma unroll
-        for (int q = 0; q < MAXW; ++q) out[q] = 0;
-        for (uint32_t j = 0; j < W; ++j) {
-          uint64_t v = X[((uint64_t)src << logW) + j];
-          if (first) acc.nzx += (v != 0);
-          while (v) {
-            const int b = __ffsll((long long)v) - 1;
-            v &= v - 1;
-            const int cd = D.colmap[xr.colmap_off + j * 64 + b];
-            if (cd < 0) continue;
-#pragma unroll
-            for (int q = 0; q < MAXW; ++q)
-              if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
+          for (int k = 0; k < KW; ++k) {
+            const uint32_t w = c0 + lane + 32 * k;
+            y[k] = (w < B) ? X[w] : 0ull;
           }
         }
 #pragma unroll
-        for (int q = 0; q < MAXW; ++q)
-          if (q < (int)mdt.W) grew |= or_into(Z + ((uint64_t)r << logWt) + q, out[q], acc);
+        for (int k = 0; k < KW; ++k) {
+          const uint32_t w = c0 + lane + 32 * k;
+          if (first && eb == e0) nzx += (y[k] != 0);
+          if (w < B && mode != 0) {
+            const int r = (int)(w >> logW);
+            if (mode == 1) { if (r == t) y[k] = gsel; }
+            else if (mode == 2) { if (r == t) y[k] |= gsel; }
+            else if ((uint32_t)r >= L + R.n_stat) {           // FSTORE: heap rows (o1, f)
+              const uint32_t g = (uint32_t)r - L;
+              if (D.grow_field[R.grow_off + g] == (int)f) {
+                const int c = D.grow_col[R.grow_off + g];     // o1 (never NULL)
+                if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) y[k] |= rwsel;
+              }
+            }
+          }
+        }
+        unsigned sm = same;
+        while (sm) {
+          const int i = __ffs(sm) - 1;
+          sm &= sm - 1;
+          const uint32_t info = __shfl_sync(FULL, E.info, i);
+          const uint64_t off = __shfl_sync(FULL, E.off, i);
+          const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;     // C2R drops lhs(c)
+          const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW);
+          nz += r & 0xffffu;
+          red += r >> 16;
+          if (r >> 16) gmask |= 1u << i;
+        }
       }
-      dense += 16ull * ((uint64_t)rows_t << logWt);
+      dense_l0 += 16ull * B * __popc(same);
     }
-    grew = __any_sync(FULL, grew);
-    const int slot = (int)((e - e0) & 31u);
-    if (lane == slot) { cand_dst = dst; cand_grew = grew; }
-    if (slot == 31 || e + 1 == e1) {
-      flush_pushes(D, lane, lane <= slot, cand_dst, cand_grew, round, nxt);
+    // -- CALL / RET: layout changes (params <- args / lhs <- RET, globals, projection π)
+    unsigned oth = live & ~same;
+    while (oth) {
+      const int i = __ffs(oth) - 1;
+      oth &= oth - 1;
+      const uint32_t ek = __shfl_sync(FULL, E.info, i) & 3u;
+      const uint64_t off = __shfl_sync(FULL, E.off, i);
+      const uint32_t Bt = __shfl_sync(FULL, E.B, i);
+      const uint32_t Lt = __shfl_sync(FULL, (uint32_t)E.L, i);
+      const uint32_t logWt = __shfl_sync(FULL, (uint32_t)E.logW, i);
+      const int aux = __shfl_sync(FULL, E.aux, i);
+      const uint32_t xoff = __shfl_sync(FULL, E.xoff, i);
+      uint64_t* Z = D.facts + off;
+      const uint32_t npar = (ek == GE_CALL) ? (uint32_t)aux : 0u;    // callee n_params
+      const int lhs = (ek == GE_RET) ? aux : -1;                      // lhs(c) at the return site
+      const uint32_t a0 = (ek == GE_CALL && npar > 3) ? D.arg_ptr[n] : 0u;
+      // source row of target local row r (params <- args, lhs <- RET_callee), -1 = none
+      auto local_src = [&](uint32_t r) -> int {
+        if (ek == GE_CALL) {
+          if (r >= npar) return -1;
+          if (npar > 3) return D.args[a0 + r];
+          return r == 0 ? R.r1 : (r == 1 ? R.r2 : R.r3);                // inline argument rows
+        }
+        return (int)r == lhs ? (int)(L - 1) : -1;
+      };
+      bool g = false;
+      if (xoff == NO_XMAP) {                                // same module: word-parallel
+        for (uint32_t c0 = 0; c0 < Bt; c0 += 32 * KW) {
+          uint64_t z[KW];
+#pragma unroll
+          for (int k = 0; k < KW; ++k) {
+            const uint32_t w = c0 + lane + 32 * k, r = w >> logW, j = w & (W - 1);
+            int src = -1;
+            if (w < Bt) src = (r < Lt) ? local_src(r) : (int)(L + (r - Lt));
+            z[k] = src >= 0 ? X[((uint64_t)src << logW) + j] : 0ull;   // CALL/EXIT: identity
+          }
+          const uint32_t r = or_chunk(Z, z, c0, lane, -1, logW);
+          nz += r & 0xffffu;
+          red += r >> 16;
+          if (r >> 16) g = true;
+        }
+        dense_l0 += 16ull * Bt;
+      } else {                                              // across modules: row-parallel π
+        for (uint32_t c = lane; c < R.n_cols; c += 32) ws.cmap[c] = (int16_t)D.xmap[xoff + c];
+        const int32_t* rowmap = D.xmap + xoff + R.n_cols;
+        const uint32_t rows_t = Bt >> logWt;
+        int src[KW];
+#pragma unroll
+        for (int k = 0; k < KW; ++k) src[k] = -1;
+        for (uint32_t r0 = 0; r0 < rows_t; r0 += 32 * KW) {
+#pragma unroll
+          for (int k = 0; k < KW; ++k) {                    // source row of each target row
+            const uint32_t r = r0 + lane + 32 * k;
+            src[k] = -1;
+            if (r < rows_t) {
+              if (r < Lt) src[k] = local_src(r);
+              else {
+                const int gs = rowmap[r - Lt];
+                src[k] = gs < 0 ? -1 : (int)(L + gs);
+              }
+            }
+          }
+          __syncwarp();
+          if (W == 1 && logWt == 0) {                       // one word per row on both sides
+            uint64_t v[KW], cur[KW];
+#pragma unroll
+            for (int k = 0; k < KW; ++k) v[k] = src[k] >= 0 ? X[src[k]] : 0ull;
+#pragma unroll
+            for (int k = 0; k < KW; ++k) {
+              uint64_t o = 0, b = v[k];
+              while (b) {
+                const int bit = __ffsll((long long)b) - 1;
+                b &= b - 1;
+                const int cd = ws.cmap[bit];
+                if (cd >= 0) o |= 1ull << cd;
+              }
+              v[k] = o;
+              cur[k] = o ? Z[r0 + lane + 32 * k] : ~0ull;
+            }
+#pragma unroll
+            for (int k = 0; k < KW; ++k) {
+              nz += (v[k] != 0);
+              if (v[k] & ~cur[k]) {
+                atomicOr((unsigned long long*)(Z + r0 + lane + 32 * k), (unsigned long long)v[k]);
+                ++red;
+                g = true;
+              }
+            }
+          } else {
+#pragma unroll 1
+            for (int k = 0; k < KW; ++k) {
+              if (src[k] < 0) continue;
+              const uint32_t r = r0 + lane + 32 * k;
+              uint64_t out[MAXW];
+#pragma unroll
+              for (int q = 0; q < MAXW; ++q) out[q] = 0;
+              for (uint32_t j = 0; j < W; ++j) {
+                uint64_t b = X[((uint64_t)src[k] << logW) + j];
+                while (b) {
+                  const int bit = __ffsll((long long)b) - 1;
+                  b &= b - 1;
+                  const int cd = ws.cmap[j * 64 + bit];
+                  if (cd < 0) continue;
+#pragma unroll
+                  for (int q = 0; q < MAXW; ++q)
+                    if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
+                }
+              }
+#pragma unroll
+              for (int q = 0; q < MAXW; ++q) {
+                if (q < (1 << logWt) && out[q]) {
+                  uint64_t* p = Z + ((uint64_t)r << logWt) + q;
+                  ++nz;
+                  if (out[q] & ~*p) { atomicOr((unsigned long long*)p, (unsigned long long)out[q]); ++red; g = true; }
+                }
+              }
+            }
+          }
+        }
+        __syncwarp();
+        dense_l0 += 16ull * Bt;
+      }
+      if (g) gmask |= 1u << i;
     }
+    const unsigned gall = __reduce_or_sync(FULL, gmask);
+    flush_pushes(D, st, lane, lane < (int)ne, E.dst, E.info, (gall >> lane) & 1u, round, nxt);
   }
-  if (lane == 0) acc.dense += dense;
+  acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
+  acc_add(acc.atom, red);
+  if (lane == 0) acc.dense += dense_l0 + alg_l0;
 }
 
+// ---------------------------------------------------------------------------------- rounds
 __device__ __forceinline__ void grid_sync(uint32_t* bar, uint32_t nblocks) {
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -304,85 +455,131 @@ __device__ __forceinline__ void grid_sync(uint32_t* bar, uint32_t nblocks) {
   __syncthreads();
 }
 
-__device__ __forceinline__ void flush_acc(const Dev& D, Acc& acc) {
-  unsigned long long ab = 16ull * acc.nz + 8ull * acc.nzx + 8ull * acc.h + acc.fixed;
-  ab = warp_sum64(ab);
-  const unsigned long long at = warp_sum64(acc.atom);
-  const unsigned long long de = warp_sum64(acc.dense + acc.fixed);
-  if ((threadIdx.x & 31) == 0 && (ab | at | de)) {
-    atomicAdd(&D.stats->alg_bytes, ab);
-    atomicAdd(&D.stats->atomics, at);
-    atomicAdd(&D.stats->dense_bytes, de);
+__device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
+  if ((threadIdx.x & 31) == 0 && (acc.alg | acc.atom | acc.dense)) {
+    atomicAdd(&D.stats->alg_bytes, acc.alg);
+    atomicAdd(&D.stats->atomics, acc.atom);
+    atomicAdd(&D.stats->dense_bytes, acc.dense);
   }
 }
 
-// Process every item of round `round` with warps gw, gw+nw, ...; returns total items.
-__device__ __forceinline__ uint32_t run_round(const Dev& D, uint32_t round, uint32_t gw, uint32_t nw,
-                                              int lane, WarpScratch& ws, Acc& acc) {
+// Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
+// the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
+__device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
+                                              uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
   if (D.bar[2]) return 0;                 // an earlier round found the worklist empty
-  uint32_t pre[NCLS + 1];
-  pre[0] = 0;
+  uint32_t cnt[NCLS];
+  uint32_t total = 0;
 #pragma unroll
-  for (int c = 0; c < NCLS; ++c) pre[c + 1] = pre[c] + D.counts[cur * CNT_STRIDE + c];
-  const uint32_t total = pre[NCLS];
-  if (total == 0) {                       // fixed point reached (Alg. 1 l.10)
-    if (blockIdx.x == 0 && threadIdx.x == 0) D.bar[2] = 1;
+  for (int c = 0; c < NCLS; ++c) { cnt[c] = D.counts[cur * CNT_STRIDE + c]; total += cnt[c]; }
+  if (total == 0) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      D.bar[2] = 1;
+      if (round <= D.trace_cap) {
+        unsigned long long ns;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
+        D.trace[2 * (round - 1)] = ns;
+        D.trace[2 * (round - 1) + 1] = 0;
+      }
+    }
     return 0;
   }
   if (D.max_rounds && round > D.max_rounds) return total;
   if (blockIdx.x == 0 && threadIdx.x == 0) {
+    const uint32_t nodes = D.counts[cur * CNT_STRIDE + CNT_NODES];
 #pragma unroll
-    for (int c = 0; c < NCLS; ++c) D.counts[clr * CNT_STRIDE + c] = 0;
+    for (int c = 0; c < CNT_STRIDE; ++c) D.counts[clr * CNT_STRIDE + c] = 0;
     D.stats->rounds += 1;
-    D.stats->visits += total;
-    D.stats->hist[total <= 32 ? 0 : (total <= 64 ? 1 : 2)] += 1;
+    D.stats->visits += nodes;
+    D.stats->hist[nodes <= 32 ? 0 : (nodes <= 64 ? 1 : 2)] += 1;
+    if (round <= D.trace_cap) {
+      unsigned long long ns;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
+      D.trace[2 * (round - 1)] = ns;
+      D.trace[2 * (round - 1) + 1] = ((unsigned long long)total << 32) | nodes;
+    }
   }
-  for (uint32_t item = gw; item < total; item += nw) {
-    int c = 0;
-    while (item >= pre[c + 1]) ++c;
-    const uint32_t n = D.queue[(size_t)cur * D.n_nodes + D.seg[c] + (item - pre[c])];
-    process_node(D, n, round, nxt, lane, ws, acc);
+  const uint32_t* Q = D.queue + (size_t)cur * D.n_chunks;
+  auto entry_of = [&](uint32_t item) -> uint32_t {          // item -> class segment -> entry
+    uint32_t c = 0, base = 0;
+#pragma unroll
+    for (int k = 0; k < NCLS - 1; ++k)
+      if (c == (uint32_t)k && item >= base + cnt[k]) { base += cnt[k]; c = k + 1; }
+    return Q[D.seg[c] + (item - base)];
+  };
+  uint32_t item = gw;
+  uint32_t entry = item < total ? entry_of(item) : 0u;
+  while (item < total) {
+    const uint32_t nitem = item + nw;
+    const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
+    if (nitem < total && lane < 4)                                     // and its NodeRec into L1
+      asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
+    process_item(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc);
+    item = nitem;
+    entry = nentry;
   }
   return total;
 }
 
-__global__ void __launch_bounds__(THREADS, 2) k_fixpoint(Dev D) {
+__global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   __shared__ WarpScratch ws_all[WARPS];
+  __shared__ Acc acc_all[WARPS];
+  __shared__ CtaStage st;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t gw = blockIdx.x * WARPS + wib, nw = gridDim.x * WARPS;
-  Acc acc = {};
+  Acc& acc = acc_all[wib];
+  if (lane == 0) acc = Acc{0, 0, 0};
+  stage_init(st);
+  __syncthreads();
   for (uint32_t round = 1;; ++round) {
-    const uint32_t total = run_round(D, round, gw, nw, lane, ws_all[wib], acc);
+    const uint32_t total = run_round(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == 0) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
       break;
     }
+    stage_publish(D, st, (round + 1) % 3);
     grid_sync(D.bar, gridDim.x);
   }
   flush_acc(D, acc);
 }
 
-__global__ void __launch_bounds__(THREADS, 2) k_round(Dev D, uint32_t round) {
+__global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t round) {
   __shared__ WarpScratch ws_all[WARPS];
+  __shared__ Acc acc_all[WARPS];
+  __shared__ CtaStage st;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t gw = blockIdx.x * WARPS + wib, nw = gridDim.x * WARPS;
-  Acc acc = {};
-  const uint32_t total = run_round(D, round, gw, nw, lane, ws_all[wib], acc);
+  Acc& acc = acc_all[wib];
+  if (lane == 0) acc = Acc{0, 0, 0};
+  stage_init(st);
+  __syncthreads();
+  const uint32_t total = run_round(D, st, round, gw, nw, lane, ws_all[wib], acc);
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
+  if (total) stage_publish(D, st, (round + 1) % 3);
   flush_acc(D, acc);
 }
 
 // (a2) seed round 1 with the component entries (Alg. 1 l.9)
 __global__ void k_seed(Dev D) {
+  __shared__ CtaStage st;
   const int lane = threadIdx.x & 31;
+  stage_init(st);
+  __syncthreads();
   for (uint32_t i0 = 0; i0 < D.n_entries; i0 += 32) {
     const uint32_t i = i0 + lane;
     const bool act = i < D.n_entries;
-    flush_pushes(D, lane, act, act ? D.entries[i] : 0, true, 0u, 1u);
+    const uint32_t e = act ? D.entries[i] : 0u;
+    uint32_t info = 0;
+    if (act) {
+      const NodeRec R = D.nodes[e];
+      info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls) - 1) << 5);
+    }
+    flush_pushes(D, st, lane, act, e, info, true, 0u, 1u);
   }
+  stage_publish(D, st, 1u);
 }
 
 // (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8)
@@ -391,9 +588,8 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
   for (uint32_t n = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < D.n_nodes; n += nw) {
     const NodeRec R = D.nodes[n];
-    const MethRec mr = D.meths[R.method];
-    const ModRec md = D.mods[mr.module];
-    const uint32_t logW = md.logW, L = mr.n_locals, B = (L + md.n_glob) << logW;
+    const uint32_t local_base = D.meths[D.node_method[n]].local_base;
+    const uint32_t logW = R.logW, L = R.L, B = R.B;
     const uint64_t* X = D.facts + R.off;
     const uint64_t hn = mix64((uint64_t)(n - D.app_node_base[R.app]));
     unsigned long long s = 0;
@@ -401,11 +597,11 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
       uint64_t x = X[w];
       if (!x) continue;
       const uint32_t r = w >> logW, j = w & ((1u << logW) - 1);
-      const uint64_t slot = r < L ? (uint64_t)(mr.local_base + r) : (uint64_t)D.grow_gid[md.grow_off + r - L];
+      const uint64_t slot = r < L ? (uint64_t)(local_base + r) : (uint64_t)D.grow_gid[R.grow_off + r - L];
       while (x) {
         const int b = __ffsll((long long)x) - 1;
         x &= x - 1;
-        const uint64_t o = D.col_gid[md.col_off + j * 64 + b];
+        const uint64_t o = D.col_gid[R.col_off + j * 64 + b];
         s += mix64(hn ^ ((slot << 32) | o));
       }
     }
@@ -422,11 +618,8 @@ __global__ void k_popc(Dev D, uint32_t n0, uint32_t n1, uint64_t* out) {
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
   for (uint32_t n = n0 + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < n1; n += nw) {
     const NodeRec R = D.nodes[n];
-    const MethRec mr = D.meths[R.method];
-    const ModRec md = D.mods[mr.module];
-    const uint32_t B = (mr.n_locals + md.n_glob) << md.logW;
     unsigned long long c = 0;
-    for (uint32_t w = lane; w < B; w += 32) c += __popcll(D.facts[R.off + w]);
+    for (uint32_t w = lane; w < R.B; w += 32) c += __popcll(D.facts[R.off + w]);
     c = warp_sum64(c);
     if (lane == 0) out[n - n0] = c;
   }
@@ -439,9 +632,8 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
   for (uint32_t n = n0 + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < n1; n += nw) {
     const NodeRec R = D.nodes[n];
-    const MethRec mr = D.meths[R.method];
-    const ModRec md = D.mods[mr.module];
-    const uint32_t logW = md.logW, L = mr.n_locals, B = (L + md.n_glob) << logW;
+    const uint32_t local_base = D.meths[D.node_method[n]].local_base;
+    const uint32_t logW = R.logW, L = R.L, B = R.B;
     uint64_t base = ptr[n - n0];
     for (uint32_t w0 = 0; w0 < B; w0 += 32) {
       const uint32_t w = w0 + lane;
@@ -456,11 +648,11 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
       uint64_t pos = base + incl - c;
       if (x) {
         const uint32_t r = w >> logW, j = w & ((1u << logW) - 1);
-        const uint64_t slot = r < L ? (uint64_t)(mr.local_base + r) : (uint64_t)D.grow_gid[md.grow_off + r - L];
+        const uint64_t slot = r < L ? (uint64_t)(local_base + r) : (uint64_t)D.grow_gid[R.grow_off + r - L];
         while (x) {
           const int b = __ffsll((long long)x) - 1;
           x &= x - 1;
-          pairs[pos++] = (slot << 32) | D.col_gid[md.col_off + j * 64 + b];
+          pairs[pos++] = (slot << 32) | D.col_gid[R.col_off + j * 64 + b];
         }
       }
       base += __shfl_sync(FULL, incl, 31);
@@ -493,28 +685,25 @@ cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStre
   return cudaGetLastError();
 }
 
-cudaError_t launch_digest(const Dev& D, cudaStream_t s) {
-  uint32_t blocks = (D.n_nodes + 7) / 8;
+static uint32_t grid_for(uint32_t items) {
+  uint32_t blocks = (items + 7) / 8;
   if (blocks > 148 * 16) blocks = 148 * 16;
-  if (blocks == 0) blocks = 1;
-  k_digest<<<blocks, 256, 0, s>>>(D);
+  return blocks ? blocks : 1;
+}
+
+cudaError_t launch_digest(const Dev& D, cudaStream_t s) {
+  k_digest<<<grid_for(D.n_nodes), 256, 0, s>>>(D);
   return cudaGetLastError();
 }
 
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s) {
-  uint32_t blocks = (n1 - n0 + 7) / 8;
-  if (blocks > 148 * 16) blocks = 148 * 16;
-  if (blocks == 0) blocks = 1;
-  k_popc<<<blocks, 256, 0, s>>>(D, n0, n1, out);
+  k_popc<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
                           cudaStream_t s) {
-  uint32_t blocks = (n1 - n0 + 7) / 8;
-  if (blocks > 148 * 16) blocks = 148 * 16;
-  if (blocks == 0) blocks = 1;
-  k_expand<<<blocks, 256, 0, s>>>(D, n0, n1, ptr, pairs);
+  k_expand<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, ptr, pairs);
   return cudaGetLastError();
 }
 

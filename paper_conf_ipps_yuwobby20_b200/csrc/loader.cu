@@ -61,7 +61,6 @@ struct HostImage {
   std::vector<NodeRec> nodes;
   std::vector<MethRec> meths;
   std::vector<ModRec> mods;
-  std::vector<XRec> xrecs{XRec{0, 0, 0, 0}};   // id 0 = identity (same module)
   std::vector<uint32_t> row_ptr{0};
   std::vector<Edge> edges;
   std::vector<uint32_t> arg_ptr{0};
@@ -71,9 +70,11 @@ struct HostImage {
   std::vector<uint32_t> grow_gid;
   std::vector<int32_t> grow_col, grow_field;
   std::vector<uint32_t> tf_ptr{0}, tf;
-  std::vector<int32_t> colmap, rowmap;
+  std::vector<int32_t> xmap;                   // projection tables: colmap then rowmap
+  std::vector<int32_t> frow;                   // per (module, field): column -> global heap row | -1
   std::vector<uint32_t> app_node_base;
   std::vector<uint32_t> entries;
+  std::vector<uint32_t> node_method;
   uint64_t fact_words = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
 };
@@ -191,6 +192,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     H.meths.push_back(MethRec{d->method_n_locals[m], d->method_n_params[m], db + d->method_module[m], (uint32_t)local_base[m]});
   // ---- nodes: operands -> rows (V1, V2, V4), fact offsets
   H.app_node_base.push_back(nb);
+  std::map<std::pair<uint32_t, uint32_t>, uint32_t> frow_map;
   auto local_idx = [&](int64_t gid, uint64_t m) -> int64_t {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
@@ -204,7 +206,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     const uint32_t L = d->method_n_locals[m];
     const int32_t* op = d->node_ops + 4 * n;
     NodeRec R{};
-    R.method = mb + (uint32_t)m; R.kind = kind; R.cls = (uint8_t)cls_of(kind); R.app = (uint16_t)k;
+    R.kind = kind; R.cls = (uint8_t)cls_of(kind); R.app = (uint16_t)k;
+    H.node_method.push_back(mb + (uint32_t)m);
     R.r0 = R.r1 = R.r2 = R.r3 = -1;
     auto need_local = [&](int32_t gid, int32_t& out, const char* what) -> bool {
       int64_t i = local_idx(gid, m);
@@ -243,6 +246,23 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           if (op[2] < 0 || (uint32_t)op[2] >= d->n_fields) return set_err(GDROID_E_INVALID, "app %u: node %llu: field out of range", k, (unsigned long long)n);
           R.r2 = op[2];
         }
+        if (kind == GK_FLOAD || kind == GK_ALOAD) {          // heap row of (o1, f) per column
+          auto key = std::make_pair((uint32_t)dd, (uint32_t)R.r2);
+          auto it = frow_map.find(key);
+          if (it == frow_map.end()) {
+            const uint32_t off = (uint32_t)H.frow.size();
+            for (uint32_t c = 0; c < md.n_cols; ++c) {
+              const int32_t ty = H.col_type[md.col_off + c];
+              int32_t row = -1;
+              if (c != 0 && ty >= 0)
+                for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
+                  if (H.tf[q] == (uint32_t)R.r2) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
+              H.frow.push_back(row);
+            }
+            it = frow_map.emplace(key, off).first;
+          }
+          R.r3 = (int32_t)it->second;
+        }
         break;
       case GK_SLOAD:
         if (!need_local(op[0], R.r0, "lhs")) return GDROID_E_POOL;
@@ -276,16 +296,22 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       int32_t row = -1;
       if (d->call_args[q] >= 0 && !need_local(d->call_args[q], row, "argument")) return GDROID_E_POOL;
       H.args.push_back(row);
+      if (kind == GK_CALL && a1 - a0 <= 3) (&R.r1)[q - a0] = row;   // inline argument rows
     }
     H.arg_ptr.push_back((uint32_t)H.args.size());
+    if (kind == GK_ENTRY) R.r1 = (int32_t)d->method_n_params[m];
     R.off = H.fact_words;
     const uint64_t words = (uint64_t)(L + md.n_glob) << md.logW;
+    if (words >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: node %llu: fact block too large", k, (unsigned long long)n);
+    R.B = (uint32_t)words; R.L = L; R.n_stat = md.n_stat;
+    R.e0 = (uint32_t)(H.edges.size() + d->row_ptr[n]); R.e1 = (uint32_t)(H.edges.size() + d->row_ptr[n + 1]);
+    R.col_off = md.col_off; R.grow_off = md.grow_off; R.n_cols = (uint16_t)md.n_cols;
+    R.logW = (uint8_t)md.logW; R.module = db + (uint32_t)dd;
     H.fact_words += (words + 3) & ~3ull;                        // 32-byte aligned blocks
     H.nodes.push_back(R);
-    H.cls_count[R.cls]++;
   }
   // ---- edges (V5, V6) + projection tables
-  std::map<std::pair<uint32_t, uint32_t>, uint32_t> xmap;
+  std::map<std::pair<uint32_t, uint32_t>, uint32_t> xmap;   // (src module, dst module) -> xoff
   for (uint64_t n = 0; n < N; ++n) {
     const uint8_t kind = d->node_kind[n];
     const uint64_t m = d->node_method[n];
@@ -293,7 +319,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     for (uint64_t e = d->row_ptr[n]; e < d->row_ptr[n + 1]; ++e) {
       const uint32_t s = d->col[e];
       const uint8_t ek = d->edge_kind[e];
-      uint32_t xid = 0;
+      uint32_t xoff = NO_XMAP;
       switch (ek) {
         case GE_INTRA:
           if (kind == GK_CALL || kind == GK_EXIT || d->node_method[s] != m) return set_err(GDROID_E_INVALID, "app %u: edge %llu: INTRA edge must stay in one method and not leave a CALL/EXIT (V5)", k, (unsigned long long)e);
@@ -323,39 +349,41 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
         if (sm != dm) {
           auto key = std::make_pair(db + sm, db + dm);
           auto it = xmap.find(key);
-          if (it != xmap.end()) xid = it->second;
+          if (it != xmap.end()) xoff = it->second;
           else {
-            xid = (uint32_t)H.xrecs.size();
-            xmap[key] = xid;
+            xoff = (uint32_t)H.xmap.size();
+            xmap[key] = xoff;
             const ModRec &ms = H.mods[db + sm], &mt = H.mods[db + dm];
-            XRec xr{(uint32_t)H.colmap.size(), (uint32_t)H.rowmap.size(), db + sm, db + dm};
             for (uint32_t c = 0; c < ms.n_cols; ++c) {      // columns: instance kept iff in Q_dst
               int64_t cd = bsearch_idx<uint32_t>(mi[dm].insts, mi[dm].n_insts, H.col_gid[ms.col_off + c]);
-              H.colmap.push_back((int32_t)cd);
+              H.xmap.push_back((int32_t)cd);
             }
             for (uint32_t g = 0; g < mt.n_glob; ++g) {      // global rows: slot kept iff in P_src
               const uint32_t gid = H.grow_gid[mt.grow_off + g];
               int32_t src = -1;
-              // statics: binary search; heap: owner column in the source pool + same ordinal
-              if (g < mt.n_stat) {
-                int64_t p = bsearch_idx<uint32_t>(mi[sm].stats, mi[sm].n_stats, gid - (uint32_t)Lt);
-                src = (int32_t)p;
-              } else {
+              if (g < mt.n_stat) {                          // statics: same static visible in src
+                src = (int32_t)bsearch_idx<uint32_t>(mi[sm].stats, mi[sm].n_stats, gid - (uint32_t)Lt);
+              } else {                                      // heap: owner in Q_src, same ordinal
                 const int32_t ct = H.grow_col[mt.grow_off + g];
                 const uint32_t o = H.col_gid[mt.col_off + ct];
                 int64_t cs = bsearch_idx<uint32_t>(mi[sm].insts, mi[sm].n_insts, o);
-                if (cs >= 0) {
-                  const uint32_t ord = g - H.col_hbase[mt.col_off + ct];
-                  src = (int32_t)(H.col_hbase[ms.col_off + cs] + ord);
-                }
+                if (cs >= 0) src = (int32_t)(H.col_hbase[ms.col_off + cs] + (g - H.col_hbase[mt.col_off + ct]));
               }
-              H.rowmap.push_back(src);
+              H.xmap.push_back(src);
             }
-            H.xrecs.push_back(xr);
           }
         }
       }
-      H.edges.push_back(Edge{nb + s, (uint32_t)ek | (xid << 2)});
+      const NodeRec& RS = H.nodes[nb + s];
+      const uint32_t nch = n_chunks_of((uint32_t)(d->row_ptr[s + 1] - d->row_ptr[s]), RS.cls);
+      if (RS.L > 0xffff) return set_err(GDROID_E_LIMIT, "app %u: method with > 65535 locals", k);
+      Edge E{};
+      E.dst = nb + s;
+      E.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5);
+      E.off = RS.off; E.B = RS.B; E.L = (uint16_t)RS.L; E.logW = RS.logW;
+      E.aux = (ek == GE_CALL) ? (int32_t)d->method_n_params[d->node_method[s]] : (ek == GE_RET ? RS.r0 : -1);
+      E.xoff = xoff;
+      H.edges.push_back(E);
     }
     if (kind == GK_CALL && n_c2r != 1) return set_err(GDROID_E_INVALID, "app %u: node %llu: a CALL needs exactly one C2R edge (V5)", k, (unsigned long long)n);
     H.row_ptr.push_back((uint32_t)H.edges.size());
@@ -402,6 +430,7 @@ void free_app(gdroid_app* a) {
   if (a->d_facts) cudaFree(a->d_facts);
   if (a->d_state) cudaFree(a->d_state);
   if (a->d_scratch) cudaFree(a->d_scratch);
+  if (a->D.trace) cudaFree(a->D.trace);
   if (a->h_stats) cudaFreeHost(a->h_stats);
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
@@ -466,10 +495,20 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   }
   const uint32_t N = (uint32_t)H.nodes.size();
   const uint32_t n_entries = (uint32_t)H.entries.size();
+  // work items: every node's out-edges in at most 32 chunks (queue entry = node << 5 | chunk)
+  if (N >= (1u << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
+  uint64_t nc64 = 0;
+  for (uint32_t n = 0; n < N; ++n) {
+    const uint32_t c = n_chunks_of(H.nodes[n].e1 - H.nodes[n].e0, H.nodes[n].cls);
+    H.cls_count[H.nodes[n].cls] += c;
+    nc64 += c;
+  }
+  if (nc64 >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
+  const uint32_t NC = (uint32_t)nc64;
   H.app_node_base.push_back(N);
   if (H.tf.empty()) H.tf.push_back(0);          // keep every table non-empty
-  if (H.colmap.empty()) H.colmap.push_back(-1);
-  if (H.rowmap.empty()) H.rowmap.push_back(-1);
+  if (H.xmap.empty()) H.xmap.push_back(-1);
+  if (H.frow.empty()) H.frow.push_back(-1);
   if (H.args.empty()) H.args.push_back(-1);
   if (H.entries.empty()) H.entries.push_back(0);
 
@@ -489,7 +528,6 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   size_t i_nodes = add(H.nodes.data(), H.nodes.size() * sizeof(NodeRec));
   size_t i_meths = add(H.meths.data(), H.meths.size() * sizeof(MethRec));
   size_t i_mods = add(H.mods.data(), H.mods.size() * sizeof(ModRec));
-  size_t i_x = add(H.xrecs.data(), H.xrecs.size() * sizeof(XRec));
   size_t i_rp = add(H.row_ptr.data(), H.row_ptr.size() * 4);
   size_t i_e = add(H.edges.data(), H.edges.size() * sizeof(Edge));
   size_t i_ap = add(H.arg_ptr.data(), H.arg_ptr.size() * 4);
@@ -502,10 +540,11 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   size_t i_gf = add(H.grow_field.data(), H.grow_field.size() * 4);
   size_t i_tp = add(H.tf_ptr.data(), H.tf_ptr.size() * 4);
   size_t i_tf = add(H.tf.data(), H.tf.size() * 4);
-  size_t i_cm = add(H.colmap.data(), H.colmap.size() * 4);
-  size_t i_rm = add(H.rowmap.data(), H.rowmap.size() * 4);
+  size_t i_xm = add(H.xmap.data(), H.xmap.size() * 4);
   size_t i_nb = add(H.app_node_base.data(), H.app_node_base.size() * 4);
   size_t i_en = add(H.entries.data(), H.entries.size() * 4);
+  size_t i_nm = add(H.node_method.data(), H.node_method.size() * 4);
+  size_t i_fr = add(H.frow.data(), H.frow.size() * 4);
 
   auto t0 = std::chrono::steady_clock::now();
   {
@@ -526,7 +565,6 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.nodes = (const NodeRec*)(T + parts[i_nodes].off);
   D.meths = (const MethRec*)(T + parts[i_meths].off);
   D.mods = (const ModRec*)(T + parts[i_mods].off);
-  D.xrecs = (const XRec*)(T + parts[i_x].off);
   D.row_ptr = (const uint32_t*)(T + parts[i_rp].off);
   D.edges = (const Edge*)(T + parts[i_e].off);
   D.arg_ptr = (const uint32_t*)(T + parts[i_ap].off);
@@ -539,11 +577,13 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.grow_field = (const int32_t*)(T + parts[i_gf].off);
   D.tf_ptr = (const uint32_t*)(T + parts[i_tp].off);
   D.tf = (const uint32_t*)(T + parts[i_tf].off);
-  D.colmap = (const int32_t*)(T + parts[i_cm].off);
-  D.rowmap = (const int32_t*)(T + parts[i_rm].off);
+  D.xmap = (const int32_t*)(T + parts[i_xm].off);
   D.app_node_base = (const uint32_t*)(T + parts[i_nb].off);
   D.entries = (const uint32_t*)(T + parts[i_en].off);
+  D.node_method = (const uint32_t*)(T + parts[i_nm].off);
+  D.frow = (const int32_t*)(T + parts[i_fr].off);
   D.n_nodes = N;
+  D.n_chunks = NC;
   D.n_entries = n_entries;
   uint32_t acc = 0;
   for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += H.cls_count[c]; }
@@ -555,7 +595,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     cudaError_t e = cudaMalloc(&a->d_facts, std::max<uint64_t>(H.fact_words, 4) * 8);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(H.fact_words * 8), cudaGetErrorString(e)));
     D.facts = a->d_facts;
-    size_t s_stamp = align256((size_t)N * 4), s_queue = align256((size_t)3 * N * 4), s_counts = align256(3 * CNT_STRIDE * 4);
+    size_t s_stamp = align256((size_t)N * 4), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t st = s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
     e = cudaMalloc(&a->d_state, st);
@@ -738,5 +778,31 @@ gdroid_status gdroid_app_digests(const gdroid_app* ca, uint64_t* per_app) {
 }
 
 void gdroid_free(gdroid_app* a) { free_app(a); }
+
+gdroid_status gdroid_debug_trace(gdroid_app* a, uint32_t cap) {
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  DeviceGuard guard(a->device);
+  if (a->D.trace) { cudaFree(a->D.trace); a->D.trace = nullptr; }
+  a->D.trace_cap = 0;
+  if (cap) {
+    CU(cudaMalloc(&a->D.trace, (size_t)cap * 16));
+    CU(cudaMemset(a->D.trace, 0, (size_t)cap * 16));
+    a->D.trace_cap = cap;
+  }
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_debug_read_trace(const gdroid_app* ca, uint64_t* out, uint64_t cap, uint64_t* n) {
+  gdroid_app* a = const_cast<gdroid_app*>(ca);
+  if (!a || !n) return set_err(GDROID_E_INVALID, "NULL argument");
+  if (!a->built) return set_err(GDROID_E_STATE, "trace read before a completed build");
+  DeviceGuard guard(a->device);
+  const uint64_t r = std::min<uint64_t>(a->last.rounds + 1, a->D.trace_cap);
+  *n = r;
+  if (!out) return GDROID_OK;
+  if (cap < 2 * r) return set_err(GDROID_E_SMALLBUF, "need %llu words", (unsigned long long)(2 * r));
+  CU(cudaMemcpy(out, a->D.trace, r * 16, cudaMemcpyDeviceToHost));
+  return GDROID_OK;
+}
 
 }  // extern "C"
