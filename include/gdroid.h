@@ -145,6 +145,9 @@ uint32_t      gdroid_n_apps(const gdroid_app* app);
  * (the last entry, with 0 items, marks the end of the fixed point). */
 gdroid_status gdroid_debug_trace(gdroid_app* app, uint32_t cap);
 gdroid_status gdroid_debug_read_trace(const gdroid_app* app, uint64_t* out, uint64_t cap, uint64_t* n);
+/* Diagnostics: per-phase cycle counters of the last build (only filled by a library compiled
+ * with -DGD_PHASES): setup, edges, pushes, round end (publish + grid barrier), items. */
+gdroid_status gdroid_debug_phases(const gdroid_app* app, uint64_t* out8);
 void          gdroid_free(gdroid_app* app);
 const char*   gdroid_last_error(void);   /* thread-local; valid until the next call */
 uint32_t      gdroid_abi_version(void);

@@ -484,33 +484,75 @@ uint64_t oracle_check_postfix(const oracle_icfg* g, const oracle_result* r) {
 }
 
 int64_t oracle_bsp_rounds(const oracle_icfg* g, uint32_t* seq, uint64_t cap, uint32_t* lens, uint64_t lens_cap) {
+  uint64_t visits = 0;
+  return oracle_bsp_rounds_policy(g, 0, seq, cap, lens, lens_cap, &visits);
+}
+
+// BSP rounds with a scheduling policy (experiments; results are policy-independent):
+// 0 = process the whole current list; 1 = defer a node to the next round when one of its
+// predecessors with a smaller node id is also in the current list (MER-style postponement,
+// PAPER.md:1039-1082; the smallest id of a list is never deferred, so progress is guaranteed).
+int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq, uint64_t cap, uint32_t* lens,
+                                 uint64_t lens_cap, uint64_t* visits) {
   Universe U;
   U.init(g);
   int rc = validate(U);
   if (rc) return rc;
   const uint32_t N = g->n_nodes;
+  std::vector<std::vector<uint32_t>> preds(N);
+  for (uint32_t p = 0; p < N; ++p)
+    for (uint64_t e = g->row_ptr[p]; e < g->row_ptr[p + 1]; ++e) preds[g->col[e]].push_back(p);
   std::vector<PairSet> IN(N);
-  std::vector<char> visited(N, 0), in_next(N, 0);
+  std::vector<char> visited(N, 0), in_next(N, 0), in_cur(N, 0);
   std::vector<uint32_t> cur, nxt;
   for (uint32_t i = 0; i < g->n_entries; ++i)
     if (std::find(cur.begin(), cur.end(), g->entries[i]) == cur.end()) cur.push_back(g->entries[i]);
   uint64_t k = 0;
   int64_t rounds = 0;
+  *visits = 0;
   while (!cur.empty()) {
     if ((uint64_t)rounds < lens_cap) lens[rounds] = (uint32_t)cur.size();
-    for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
+    if (policy != 2) for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
     ++rounds;
     nxt.clear();
-    for (uint32_t n : cur) {
-      visited[n] = 1;
-      PairSet Y = transfer(U, n, IN[n]);
-      for (uint64_t e = g->row_ptr[n]; e < g->row_ptr[n + 1]; ++e) {
-        uint32_t s = g->col[e];
-        PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
-        bool grew = merge_union(IN[s], Z);
-        if ((grew || !visited[s]) && !in_next[s]) { nxt.push_back(s); in_next[s] = 1; }
+    uint32_t max_depth = 0;
+    for (uint32_t n : cur) in_cur[n] = 1;
+    std::vector<uint32_t> cont_round(policy == 2 ? N : 0, 0);
+    for (uint32_t n0 : cur) {
+      bool defer = false;
+      if (policy == 1)
+        for (uint32_t p : preds[n0]) if (p < n0 && in_cur[p]) { defer = true; break; }
+      if (defer) {
+        if (!in_next[n0]) { nxt.push_back(n0); in_next[n0] = 1; }
+        continue;
+      }
+      // policy 2: continue depth-first into a grown successor of a single-successor node
+      uint32_t n = n0;
+      for (int depth = 0; depth < 64; ++depth) {
+        visited[n] = 1;
+        ++*visits;
+        PairSet Y = transfer(U, n, IN[n]);
+        int64_t cont = -1;
+        for (uint64_t e = g->row_ptr[n]; e < g->row_ptr[n + 1]; ++e) {
+          uint32_t s = g->col[e];
+          PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
+          bool grew = merge_union(IN[s], Z);
+          if (!(grew || !visited[s])) continue;
+          if (policy == 2 && g->row_ptr[n + 1] - g->row_ptr[n] == 1 && !in_cur[s] &&
+              cont_round[s] != (uint32_t)rounds) {
+            cont_round[s] = (uint32_t)rounds;
+            cont = s;
+            continue;
+          }
+          if (!in_next[s]) { nxt.push_back(s); in_next[s] = 1; }
+        }
+        if (depth + 1 > (int)max_depth) max_depth = depth + 1;
+        if (cont < 0) break;
+        n = (uint32_t)cont;
       }
     }
+    if (policy == 2 && (uint64_t)(rounds - 1) < cap) seq[rounds - 1] = max_depth;   // chain depth
+    for (uint32_t n : cur) in_cur[n] = 0;
     for (uint32_t s : nxt) in_next[s] = 0;
     cur.swap(nxt);
   }

@@ -80,6 +80,8 @@ def lib():
         L.gdroid_debug_read_trace.argtypes = [P, P, C.c_uint64, P]
         L.gdroid_debug_trace.restype = C.c_int
         L.gdroid_debug_read_trace.restype = C.c_int
+        L.gdroid_debug_phases.argtypes = [P, P]
+        L.gdroid_debug_phases.restype = C.c_int
         L.gdroid_free.argtypes = [P]
         L.gdroid_free.restype = None
         L.gdroid_last_error.restype = C.c_char_p
@@ -192,6 +194,11 @@ class App:
         _check(lib().gdroid_debug_read_trace(self._h, _ptr(buf), buf.size, C.byref(n)))
         t = buf.reshape(-1, 2)[:n.value]
         return np.stack([t[:, 0], t[:, 1] >> 32, t[:, 1] & 0xFFFFFFFF], axis=1)
+
+    def phases(self) -> np.ndarray:
+        out = np.zeros(8, dtype=np.uint64)
+        _check(lib().gdroid_debug_phases(self._h, _ptr(out)))
+        return out
 
     def free(self):
         if getattr(self, "_h", None) is not None and self._h.value:

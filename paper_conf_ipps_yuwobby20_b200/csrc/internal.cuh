@@ -91,6 +91,7 @@ constexpr uint32_t NO_XMAP = 0xffffffffu;
 
 struct DevStats {
   unsigned long long rounds, visits, alg_bytes, dense_bytes, atomics, hist[3], limit_hit, pad;
+  unsigned long long phase[8];  // GD_PHASES builds: cycles in setup / edges / push / round end, items
 };
 
 struct Dev {

@@ -54,6 +54,11 @@ struct CtaStage {              // per-CTA staged worklist appends of the current
   uint32_t buf[NCLS][SCAP];
 };
 
+// fire-and-forget 64-bit OR at L2 (RED; no return value, no scoreboard wait)
+__device__ __forceinline__ void red_or(uint64_t* p, uint64_t v) {
+  asm volatile("red.relaxed.gpu.global.or.b64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+
 __device__ __forceinline__ uint64_t warp_or64(uint64_t v) {
   const uint32_t lo = __reduce_or_sync(FULL, (uint32_t)v);
   const uint32_t hi = __reduce_or_sync(FULL, (uint32_t)(v >> 32));
@@ -165,7 +170,7 @@ __device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uin
     const uint64_t z = (kill >= 0 && (int)(w >> logW) == kill) ? 0ull : y[k];
     nz += (z != 0);
     if (z & ~cur[k]) {
-      atomicOr((unsigned long long*)(Z + w), (unsigned long long)z);
+      red_or(Z + w, z);
       ++red;
     }
   }
@@ -189,9 +194,6 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
 
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
   //      the rows the transfer function reads
-  const uint32_t ne0 = min(32u, e1 - e0);
-  Edge E{0, 0, 0};
-  if (lane < (int)ne0) E = D.edges[e0 + lane];
   uint64_t y[KW];
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
@@ -253,11 +255,8 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
   unsigned long long dense_l0 = first ? 8ull * B : 0ull;
   for (uint32_t eb = e0; eb < e1; eb += 32) {               // edges in batches of 32 (a5)
     const uint32_t ne = min(32u, e1 - eb);
-    if (eb != e0) {
-      E = Edge{0, 0, 0};
-      if (lane < (int)ne) E = D.edges[eb + lane];
-    }
-    const uint32_t my_kind = E.info & 3u;
+    const uint32_t my_info = lane < (int)ne ? D.edges[eb + lane].info : 0u;
+    const uint32_t my_kind = my_info & 3u;
     const unsigned live = __ballot_sync(FULL, lane < (int)ne);
     const unsigned same = __ballot_sync(FULL, lane < (int)ne && (my_kind == GE_INTRA || my_kind == GE_C2R));
     unsigned gmask = 0;
@@ -292,8 +291,9 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
         while (sm) {
           const int i = __ffs(sm) - 1;
           sm &= sm - 1;
-          const uint32_t info = __shfl_sync(FULL, E.info, i);
-          const uint64_t off = __shfl_sync(FULL, E.off, i);
+          const Edge* ep = D.edges + eb + i;
+          const uint32_t info = ep->info;
+          const uint64_t off = ep->off;
           const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;     // C2R drops lhs(c)
           const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW);
           nz += r & 0xffffu;
@@ -308,13 +308,14 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
     while (oth) {
       const int i = __ffs(oth) - 1;
       oth &= oth - 1;
-      const uint32_t ek = __shfl_sync(FULL, E.info, i) & 3u;
-      const uint64_t off = __shfl_sync(FULL, E.off, i);
-      const uint32_t Bt = __shfl_sync(FULL, E.B, i);
-      const uint32_t Lt = __shfl_sync(FULL, (uint32_t)E.L, i);
-      const uint32_t logWt = __shfl_sync(FULL, (uint32_t)E.logW, i);
-      const int aux = __shfl_sync(FULL, E.aux, i);
-      const uint32_t xoff = __shfl_sync(FULL, E.xoff, i);
+      const Edge* ep = D.edges + eb + i;
+      const uint32_t ek = ep->info & 3u;
+      const uint64_t off = ep->off;
+      const uint32_t Bt = ep->B;
+      const uint32_t Lt = ep->L;
+      const uint32_t logWt = ep->logW;
+      const int aux = ep->aux;
+      const uint32_t xoff = ep->xoff;
       uint64_t* Z = D.facts + off;
       const uint32_t npar = (ek == GE_CALL) ? (uint32_t)aux : 0u;    // callee n_params
       const int lhs = (ek == GE_RET) ? aux : -1;                      // lhs(c) at the return site
@@ -386,13 +387,13 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
             for (int k = 0; k < KW; ++k) {
               nz += (v[k] != 0);
               if (v[k] & ~cur[k]) {
-                atomicOr((unsigned long long*)(Z + r0 + lane + 32 * k), (unsigned long long)v[k]);
+                red_or(Z + r0 + lane + 32 * k, v[k]);
                 ++red;
                 g = true;
               }
             }
           } else {
-#pragma unroll 1
+#pragma unroll
             for (int k = 0; k < KW; ++k) {
               if (src[k] < 0) continue;
               const uint32_t r = r0 + lane + 32 * k;
@@ -416,7 +417,7 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
                 if (q < (1 << logWt) && out[q]) {
                   uint64_t* p = Z + ((uint64_t)r << logWt) + q;
                   ++nz;
-                  if (out[q] & ~*p) { atomicOr((unsigned long long*)p, (unsigned long long)out[q]); ++red; g = true; }
+                  if (out[q] & ~*p) { red_or(p, out[q]); ++red; g = true; }
                 }
               }
             }
@@ -428,7 +429,8 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
       if (g) gmask |= 1u << i;
     }
     const unsigned gall = __reduce_or_sync(FULL, gmask);
-    flush_pushes(D, st, lane, lane < (int)ne, E.dst, E.info, (gall >> lane) & 1u, round, nxt);
+    const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt);
   }
   acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
   acc_add(acc.atom, red);

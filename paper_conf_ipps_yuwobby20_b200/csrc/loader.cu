@@ -779,6 +779,12 @@ gdroid_status gdroid_app_digests(const gdroid_app* ca, uint64_t* per_app) {
 
 void gdroid_free(gdroid_app* a) { free_app(a); }
 
+gdroid_status gdroid_debug_phases(const gdroid_app* a, uint64_t* out8) {
+  if (!a || !out8) return set_err(GDROID_E_INVALID, "NULL argument");
+  for (int i = 0; i < 8; ++i) out8[i] = a->h_stats->phase[i];
+  return GDROID_OK;
+}
+
 gdroid_status gdroid_debug_trace(gdroid_app* a, uint32_t cap) {
   if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
   DeviceGuard guard(a->device);

@@ -23,6 +23,11 @@ app.set_trace(1 << 16)
 for _ in range(3):
     st = app.build(blocks=blocks)
 tr = app.read_trace()
+ph = app.phases().astype(float)
+if ph[4] > 0:
+    tot = ph[:4].sum()
+    print(f"phases (GD_PHASES): items {ph[4]:.0f}  setup {ph[0]/tot:.1%}  edges {ph[1]/tot:.1%}  push {ph[2]/tot:.1%}  "
+          f"round-end {ph[3]/tot:.1%};  cycles/item setup {ph[0]/ph[4]:.0f} edges {ph[1]/ph[4]:.0f} push {ph[2]/ph[4]:.0f}")
 dt = np.diff(tr[:, 0].astype(np.int64)) / 1e3   # us per round
 items = tr[:-1, 1]
 print(f"{wl}: rounds {len(dt)} fixpoint {st['fixpoint_ns']/1e6:.3f} ms, mean round {dt.mean():.2f} us")
