@@ -1,0 +1,99 @@
+"""GPU parity at BASELINE.json's full sizes against stored oracle results.
+
+tests/golden/oracle_digests.json is written by scripts/make_oracle_digests.py, which calls only
+oracle/ (never the CUDA path).  At these sizes the comparison is: the app digest (C8), an
+order-sensitive hash of the per-node digest array (so every node's set is checked), and the
+complete pair lists of sampled nodes.  Corpus apps are built in batches (shared rounds), in
+the same launch configuration bench.py times.
+"""
+from __future__ import annotations
+
+import json
+import os
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_yuwobby20_b200 as gd
+from synth import generator as G
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+FIX = os.path.join(HERE, "golden", "oracle_digests.json")
+M = (1 << 64) - 1
+
+
+def _mix64(z):
+    z &= M
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M
+    return z ^ (z >> 31)
+
+
+def _node_hash(per_node):
+    h = 0
+    for i, d in enumerate(per_node.tolist()):
+        h = (h + _mix64((i * 0x9E3779B97F4A7C15) ^ d)) & M
+    return h
+
+
+def _fixture():
+    if not os.path.exists(FIX):
+        pytest.skip("no stored oracle digests")
+    return json.load(open(FIX))
+
+
+def _check(app, k, g, ref):
+    assert ref["gen_version"] == G.GEN_VERSION and ref["n_nodes"] == g.n_nodes
+    for n, pairs in ref["samples"].items():
+        got = app.read_facts(int(n), k=k)
+        assert [str(int(p)) for p in got] == pairs, f"{ref['name']} node {n}"
+
+
+@pytest.mark.parametrize("name", ["small", "median", "worst"])
+def test_preset_full_size(name):
+    fx = _fixture()
+    if name not in fx:
+        pytest.skip(f"{name} not in fixture")
+    ref = fx[name]
+    g = G.preset(name)
+    app = gd.load(g)
+    app.build()
+    per, dig = app.node_digests()
+    assert str(dig) == ref["app_digest"]
+    assert str(_node_hash(per)) == ref["node_digest_hash"]
+    _check(app, 0, g, ref)
+
+
+def test_corpus_batches_full_size():
+    fx = _fixture()
+    ids = [i for i in range(16) if f"corpus{i}" in fx]
+    if not ids:
+        pytest.skip("no corpus apps in fixture")
+    for b0 in range(0, len(ids), 8):
+        batch = ids[b0:b0 + 8]
+        gs = [G.corpus_app(i) for i in batch]
+        app = gd.load(gs)
+        app.build()
+        digs = app.app_digests()
+        for k, (i, g) in enumerate(zip(batch, gs)):
+            ref = fx[f"corpus{i}"]
+            assert str(int(digs[k])) == ref["app_digest"], f"corpus{i}"
+            _check(app, k, g, ref)
+        app.free()
+
+
+def test_corpus_run_shard_pipeline():
+    """The corpus driver's per-rank pipeline (loader thread + batched builds) on 6 apps."""
+    from paper_conf_ipps_yuwobby20_b200 import corpus
+    fx = _fixture()
+    ids = [i for i in range(6) if f"corpus{i}" in fx]
+    sizes = G.corpus_sizes(16)
+    res = corpus.run_shard(ids, G.corpus_app, sizes, node_budget=600_000)
+    seen = {}
+    for br in res:
+        for k, i in enumerate(br.app_ids):
+            seen[i] = str(int(br.digests[k]))
+    assert sorted(seen) == ids and len(res) >= 2
+    for i in ids:
+        assert seen[i] == fx[f"corpus{i}"]["app_digest"]
