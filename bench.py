@@ -237,16 +237,20 @@ def run_ours(args):
     digests = app.app_digests()
 
     # e2e: the public C-ABI call with HOST buffers: load (H2D) + build + digest readback
-    e2e_ms = []
+    e2e_ms, e2e_parts = [], []
     for _ in range(args.e2e_steps):
         barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
-        a2 = gd.load(apps, device=local, stream=stream.cuda_stream)
+        a2 = gd.load(apps, device=local, stream=stream.cuda_stream)     # host tables + H2D
+        t1 = time.perf_counter()
         a2.build(loop_mode=args.loop_mode)
-        d2 = a2.app_digests()
-        e2e_ms.append((time.perf_counter() - t0) * 1e3)
+        t2 = time.perf_counter()
+        d2 = a2.app_digests()                                            # D2H of the result
+        t3 = time.perf_counter()
         a2.free()
+        e2e_ms.append((t3 - t0) * 1e3)
+        e2e_parts.append(((t1 - t0) * 1e3, (t2 - t1) * 1e3, (t3 - t2) * 1e3))
         assert np.array_equal(d2, digests)
     e2e_mine = statistics.median(e2e_ms) if e2e_ms else float("nan")
 
@@ -305,7 +309,10 @@ def run_ours(args):
                      "peak_source": peak_src, "traffic_workload": traffic_wl},
         "e2e": {"value": total_apps / (e2e_max / 1e3), "unit": "apps/s",
                 "h2d_bytes_per_step": input_bytes, "d2h_bytes_per_step": 8 * n_apps + 128,
-                "ms_per_step": e2e_max},
+                "ms_per_step": e2e_max,
+                "breakdown_ms": dict(zip(("load", "build", "readback"),
+                                         [round(statistics.median(x), 2) for x in zip(*e2e_parts)]))
+                                if e2e_parts else None},
         "clocks": clocks,
     }
     if not args.no_cpu_baseline:

@@ -6,11 +6,16 @@
 // buffer (the paper's dual-buffered copy, Alg. 2 l.2, is recast as the corpus driver's
 // double-buffered per-batch H2D).  (a2)-(a7) are enqueued by gdroid_build_idfg.
 #include <algorithm>
+#include <cstdlib>
 #include <chrono>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <atomic>
 #include <map>
+#include <mutex>
+#include <thread>
+#include <unordered_map>
 #include <string>
 #include <vector>
 
@@ -21,6 +26,21 @@ using namespace gd;
 namespace {
 
 thread_local std::string g_err;
+
+// GDROID_TIMING=1: print host-side phase times of gdroid_load_* to stderr
+struct PhaseTimer {
+  bool on;
+  std::chrono::steady_clock::time_point t;
+  PhaseTimer() : on(getenv("GDROID_TIMING") != nullptr), t(std::chrono::steady_clock::now()) {}
+  void mark(const char* what) {
+    if (!on) return;
+    auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "[gdroid] %-28s %8.2f ms\n", what, std::chrono::duration<double, std::milli>(now - t).count());
+    t = now;
+  }
+};
+thread_local PhaseTimer* g_pt = nullptr;
+#define PHASE(x) do { if (g_pt) g_pt->mark(x); } while (0)
 
 gdroid_status set_err(gdroid_status st, const char* fmt, ...) {
   char buf[600];
@@ -86,6 +106,42 @@ struct ModInfo {
   uint32_t gmod;   // global module index
 };
 
+// Run f(k) for k in [0, n) on up to hardware_concurrency threads.
+template <class F>
+void parallel_for(uint32_t n, F f) {
+  uint32_t T = std::max(1u, std::min<uint32_t>(n, std::thread::hardware_concurrency()));
+  if (T <= 1) { for (uint32_t k = 0; k < n; ++k) f(k); return; }
+  std::vector<std::thread> th;
+  std::atomic<uint32_t> next{0};
+  for (uint32_t t = 0; t < T; ++t)
+    th.emplace_back([&] { for (uint32_t k; (k = next.fetch_add(1)) < n;) f(k); });
+  for (auto& x : th) x.join();
+}
+
+// Run f(lo, hi) over [0, n) split into ranges of about `grain` items, in parallel.
+template <class F>
+void parallel_ranges(uint64_t n, uint64_t grain, F f) {
+  const uint64_t parts = (n + grain - 1) / grain;
+  if (parts <= 1) { if (n) f(0, n); return; }
+  parallel_for((uint32_t)parts, [&](uint32_t i) { f(i * grain, std::min(n, (i + 1) * grain)); });
+}
+
+// Deterministic error reporting from parallel validation: the lowest failing index wins.
+struct FirstErr {
+  std::mutex mu;
+  uint64_t idx = UINT64_MAX;
+  gdroid_status st = GDROID_OK;
+  std::string msg;
+  void offer(uint64_t i, gdroid_status s) {
+    std::lock_guard<std::mutex> l(mu);
+    if (i < idx) { idx = i; st = s; msg = g_err; }
+  }
+  gdroid_status result() {
+    if (st != GDROID_OK) g_err = msg;
+    return st;
+  }
+};
+
 gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   if (!d) return set_err(GDROID_E_INVALID, "app %u: NULL descriptor", k);
   if (d->abi_version != GDROID_ABI_VERSION)
@@ -95,6 +151,9 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   if (N == 0 || M == 0 || Dm == 0 || I == 0) return set_err(GDROID_E_INVALID, "app %u: empty ICFG", k);
   if ((uint64_t)H.nodes.size() + N >= (1ull << 32) || (uint64_t)H.edges.size() + E >= (1ull << 32))
     return set_err(GDROID_E_LIMIT, "app %u: batch exceeds 2^32 nodes or edges", k);
+  H.nodes.reserve(H.nodes.size() + N); H.node_method.reserve(H.node_method.size() + N);
+  H.edges.reserve(H.edges.size() + E); H.row_ptr.reserve(H.row_ptr.size() + N);
+  H.arg_ptr.reserve(H.arg_ptr.size() + N); H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
   const uint32_t nb = (uint32_t)H.nodes.size(), mb = (uint32_t)H.meths.size();
   const uint32_t db = (uint32_t)H.mods.size(), tb = (uint32_t)(H.tf_ptr.size() - 1);
   // ---- CSR (structure)
@@ -110,6 +169,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (d->node_kind[n] > GK_ASTORE) return set_err(GDROID_E_INVALID, "app %u: node %llu bad kind", k, (unsigned long long)n);
     if (d->node_method[n] >= M) return set_err(GDROID_E_INVALID, "app %u: node %llu method out of range", k, (unsigned long long)n);
   }
+  PHASE("csr checks");
   // ---- types
   for (uint64_t t = 0; t < T; ++t) {
     if (d->type_field_ptr[t + 1] < d->type_field_ptr[t]) return set_err(GDROID_E_INVALID, "app %u: type_field_ptr not monotone at %llu", k, (unsigned long long)t);
@@ -128,6 +188,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (t < -1 || t >= (int64_t)T) return set_err(GDROID_E_INVALID, "app %u: instance %llu type out of range", k, (unsigned long long)o);
     heap_base[o + 1] = heap_base[o] + (t < 0 ? 0 : d->type_field_ptr[t + 1] - d->type_field_ptr[t]);
   }
+  PHASE("types");
   // ---- methods / slot numbering
   std::vector<uint64_t> local_base(M + 1, 0);
   for (uint64_t m = 0; m < M; ++m) {
@@ -140,6 +201,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   }
   const uint64_t Lt = local_base[M];
   if (Lt + G + heap_base[I] >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: more than 2^32 slots", k);
+  PHASE("methods");
   // ---- modules: pools, rows, columns
   std::vector<ModInfo> mi(Dm);
   for (uint64_t dd = 0; dd < Dm; ++dd) {
@@ -190,14 +252,60 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   }
   for (uint64_t m = 0; m < M; ++m)
     H.meths.push_back(MethRec{d->method_n_locals[m], d->method_n_params[m], db + d->method_module[m], (uint32_t)local_base[m]});
-  // ---- nodes: operands -> rows (V1, V2, V4), fact offsets
+  PHASE("modules");
+  // ---- nodes: operands -> rows (V1, V2, V4), fact offsets (parallel over node ranges)
   H.app_node_base.push_back(nb);
-  std::map<std::pair<uint32_t, uint32_t>, uint32_t> frow_map;
+  for (uint64_t n = 0; n < N; ++n)
+    if (d->call_arg_ptr[n + 1] < d->call_arg_ptr[n]) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr not monotone at %llu", k, (unsigned long long)n);
+  const uint64_t n_args = d->call_arg_ptr[N] - d->call_arg_ptr[0];
+  if (d->call_arg_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr[0] != 0", k);
+  std::vector<uint64_t> foff(N + 1, 0);                      // fact-block offsets
+  parallel_ranges(N, 1 << 15, [&](uint64_t lo, uint64_t hi) {
+    for (uint64_t n = lo; n < hi; ++n) {
+      const uint64_t m = d->node_method[n];
+      const ModRec& md = H.mods[db + d->method_module[m]];
+      const uint64_t words = (uint64_t)(d->method_n_locals[m] + md.n_glob) << md.logW;
+      foff[n + 1] = (words + 3) & ~3ull;                        // 32-byte aligned blocks
+    }
+  });
+  for (uint64_t n = 0; n < N; ++n) foff[n + 1] += foff[n];
+  // field-row tables of FLOAD/ALOAD: one per (module, field) pair actually loaded from
+  std::vector<int32_t> frow_of(N, -1);
+  {
+    std::unordered_map<uint64_t, uint32_t> frow_map;
+    for (uint64_t n = 0; n < N; ++n) {
+      const uint8_t kind = d->node_kind[n];
+      if (kind != GK_FLOAD && kind != GK_ALOAD) continue;
+      const int32_t f = (kind == GK_ALOAD) ? (int32_t)GDROID_F_ARR : d->node_ops[4 * n + 2];
+      if (f < 0 || (uint32_t)f >= d->n_fields) continue;       // reported by the node pass
+      const uint64_t dd = d->method_module[d->node_method[n]];
+      const uint64_t key = (dd << 32) | (uint32_t)f;
+      auto it = frow_map.find(key);
+      if (it == frow_map.end()) {
+        const ModRec& md = H.mods[db + dd];
+        const uint32_t off = (uint32_t)H.frow.size();
+        for (uint32_t c = 0; c < md.n_cols; ++c) {
+          const int32_t ty = H.col_type[md.col_off + c];
+          int32_t row = -1;
+          if (c != 0 && ty >= 0)
+            for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
+              if (H.tf[q] == (uint32_t)f) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
+          H.frow.push_back(row);
+        }
+        it = frow_map.emplace(key, off).first;
+      }
+      frow_of[n] = (int32_t)it->second;
+    }
+  }
   auto local_idx = [&](int64_t gid, uint64_t m) -> int64_t {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
   };
-  for (uint64_t n = 0; n < N; ++n) {
+  H.nodes.resize(nb + N); H.node_method.resize(nb + N);
+  H.row_ptr.resize(nb + N + 1); H.arg_ptr.resize(nb + N + 1); H.args.resize(n_args);
+  FirstErr fe;
+  std::mutex cls_mu;
+  auto node_pass = [&](uint64_t n, uint32_t* cls_cnt) -> gdroid_status {
     const uint8_t kind = d->node_kind[n];
     const uint64_t m = d->node_method[n];
     const uint64_t dd = d->method_module[m];
@@ -207,7 +315,6 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     const int32_t* op = d->node_ops + 4 * n;
     NodeRec R{};
     R.kind = kind; R.cls = (uint8_t)cls_of(kind); R.app = (uint16_t)k;
-    H.node_method.push_back(mb + (uint32_t)m);
     R.r0 = R.r1 = R.r2 = R.r3 = -1;
     auto need_local = [&](int32_t gid, int32_t& out, const char* what) -> bool {
       int64_t i = local_idx(gid, m);
@@ -246,23 +353,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           if (op[2] < 0 || (uint32_t)op[2] >= d->n_fields) return set_err(GDROID_E_INVALID, "app %u: node %llu: field out of range", k, (unsigned long long)n);
           R.r2 = op[2];
         }
-        if (kind == GK_FLOAD || kind == GK_ALOAD) {          // heap row of (o1, f) per column
-          auto key = std::make_pair((uint32_t)dd, (uint32_t)R.r2);
-          auto it = frow_map.find(key);
-          if (it == frow_map.end()) {
-            const uint32_t off = (uint32_t)H.frow.size();
-            for (uint32_t c = 0; c < md.n_cols; ++c) {
-              const int32_t ty = H.col_type[md.col_off + c];
-              int32_t row = -1;
-              if (c != 0 && ty >= 0)
-                for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
-                  if (H.tf[q] == (uint32_t)R.r2) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
-              H.frow.push_back(row);
-            }
-            it = frow_map.emplace(key, off).first;
-          }
-          R.r3 = (int32_t)it->second;
-        }
+        if (kind == GK_FLOAD || kind == GK_ALOAD) R.r3 = frow_of[n];   // heap row of (o1, f) per column
         break;
       case GK_SLOAD:
         if (!need_local(op[0], R.r0, "lhs")) return GDROID_E_POOL;
@@ -290,29 +381,109 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
         break;
     }
     const uint64_t a0 = d->call_arg_ptr[n], a1 = d->call_arg_ptr[n + 1];
-    if (a1 < a0) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr not monotone at %llu", k, (unsigned long long)n);
     if (kind != GK_CALL && a1 != a0) return set_err(GDROID_E_INVALID, "app %u: node %llu: arguments on a non-CALL node", k, (unsigned long long)n);
     for (uint64_t q = a0; q < a1; ++q) {
       int32_t row = -1;
       if (d->call_args[q] >= 0 && !need_local(d->call_args[q], row, "argument")) return GDROID_E_POOL;
-      H.args.push_back(row);
+      H.args[q] = row;
       if (kind == GK_CALL && a1 - a0 <= 3) (&R.r1)[q - a0] = row;   // inline argument rows
     }
-    H.arg_ptr.push_back((uint32_t)H.args.size());
     if (kind == GK_ENTRY) R.r1 = (int32_t)d->method_n_params[m];
-    R.off = H.fact_words;
     const uint64_t words = (uint64_t)(L + md.n_glob) << md.logW;
     if (words >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: node %llu: fact block too large", k, (unsigned long long)n);
+    if (L > 0xffff) return set_err(GDROID_E_LIMIT, "app %u: node %llu: method with > 65535 locals", k, (unsigned long long)n);
+    R.off = H.fact_words + foff[n];
     R.B = (uint32_t)words; R.L = L; R.n_stat = md.n_stat;
-    R.e0 = (uint32_t)(H.edges.size() + d->row_ptr[n]); R.e1 = (uint32_t)(H.edges.size() + d->row_ptr[n + 1]);
+    R.e0 = (uint32_t)d->row_ptr[n]; R.e1 = (uint32_t)d->row_ptr[n + 1];
     R.col_off = md.col_off; R.grow_off = md.grow_off; R.n_cols = (uint16_t)md.n_cols;
     R.logW = (uint8_t)md.logW; R.module = db + (uint32_t)dd;
-    H.fact_words += (words + 3) & ~3ull;                        // 32-byte aligned blocks
-    H.nodes.push_back(R);
+    H.nodes[nb + n] = R;
+    H.node_method[nb + n] = mb + (uint32_t)m;
+    H.row_ptr[nb + n + 1] = (uint32_t)d->row_ptr[n + 1];
+    H.arg_ptr[nb + n + 1] = (uint32_t)a1;
+    cls_cnt[R.cls] += n_chunks_of(R.e1 - R.e0, R.cls);     // work items per GRP class
+    return GDROID_OK;
+  };
+  parallel_ranges(N, 1 << 14, [&](uint64_t lo, uint64_t hi) {
+    uint32_t cc[NCLS] = {0, 0, 0, 0, 0};
+    for (uint64_t n = lo; n < hi; ++n) {
+      const gdroid_status st = node_pass(n, cc);
+      if (st != GDROID_OK) { fe.offer(n, st); return; }
+    }
+    std::lock_guard<std::mutex> l(cls_mu);
+    for (int c = 0; c < NCLS; ++c) H.cls_count[c] += cc[c];
+  });
+  if (fe.st != GDROID_OK) return fe.result();
+  H.fact_words += foff[N];
+  PHASE("nodes");
+  // ---- projection tables: one per (source module, target module) pair with a CALL/RET edge
+  std::vector<uint64_t> pairs;
+  {
+    std::mutex pm;
+    parallel_ranges(N, 1 << 15, [&](uint64_t lo, uint64_t hi) {
+      std::vector<uint64_t> loc;
+      for (uint64_t n = lo; n < hi; ++n) {
+        const uint8_t kind = d->node_kind[n];
+        if (kind != GK_CALL && kind != GK_EXIT) continue;
+        const uint32_t sm = d->method_module[d->node_method[n]];
+        for (uint64_t e = d->row_ptr[n]; e < d->row_ptr[n + 1]; ++e) {
+          const uint8_t ek = d->edge_kind[e];
+          if (ek != GE_CALL && ek != GE_RET) continue;
+          const uint32_t dm = d->method_module[d->node_method[d->col[e]]];
+          if (dm != sm) loc.push_back(((uint64_t)sm << 32) | dm);
+        }
+      }
+      std::sort(loc.begin(), loc.end());
+      loc.erase(std::unique(loc.begin(), loc.end()), loc.end());
+      std::lock_guard<std::mutex> l(pm);
+      pairs.insert(pairs.end(), loc.begin(), loc.end());
+    });
+    std::sort(pairs.begin(), pairs.end());
+    pairs.erase(std::unique(pairs.begin(), pairs.end()), pairs.end());
   }
-  // ---- edges (V5, V6) + projection tables
-  std::map<std::pair<uint32_t, uint32_t>, uint32_t> xmap;   // (src module, dst module) -> xoff
-  for (uint64_t n = 0; n < N; ++n) {
+  std::vector<uint32_t> pair_off(pairs.size() + 1, 0);
+  for (size_t i = 0; i < pairs.size(); ++i) {
+    const ModRec &ms = H.mods[db + (pairs[i] >> 32)], &mt = H.mods[db + (uint32_t)pairs[i]];
+    pair_off[i + 1] = pair_off[i] + ms.n_cols + mt.n_glob;
+  }
+  const size_t xbase = H.xmap.size();
+  H.xmap.resize(xbase + pair_off[pairs.size()], -1);
+  parallel_ranges(pairs.size(), 64, [&](uint64_t lo, uint64_t hi) {
+    std::vector<int32_t> t2s;
+    for (uint64_t i = lo; i < hi; ++i) {
+      // π keeps a column iff its instance is in Q_dst and a global row iff
+      // its slot is in P_src; tables built by merging the sorted pools
+      const uint32_t sm = (uint32_t)(pairs[i] >> 32), dm = (uint32_t)pairs[i];
+      const ModRec &ms = H.mods[db + sm], &mt = H.mods[db + dm];
+      const ModInfo &Ps = mi[sm], &Pt = mi[dm];
+      int32_t* cmap = H.xmap.data() + xbase + pair_off[i];   // src column -> dst column
+      int32_t* rmap = cmap + ms.n_cols;                       // dst global row -> src global row
+      t2s.assign(Pt.n_insts, -1);
+      for (uint64_t a = 0, b2 = 0; a < Ps.n_insts && b2 < Pt.n_insts;) {
+        if (Ps.insts[a] == Pt.insts[b2]) { cmap[a] = (int32_t)b2; t2s[b2] = (int32_t)a; ++a; ++b2; }
+        else if (Ps.insts[a] < Pt.insts[b2]) ++a;
+        else ++b2;
+      }
+      for (uint64_t a = 0, b2 = 0; a < Ps.n_stats && b2 < Pt.n_stats;) {
+        if (Ps.stats[a] == Pt.stats[b2]) { rmap[b2] = (int32_t)a; ++a; ++b2; }
+        else if (Ps.stats[a] < Pt.stats[b2]) ++a;
+        else ++b2;
+      }
+      for (uint32_t ct = 1; ct < mt.n_cols; ++ct) {            // heap rows of shared instances
+        const int32_t cs = t2s[ct];
+        const int32_t ty = H.col_type[mt.col_off + ct];
+        if (cs < 0 || ty < 0) continue;
+        const uint32_t nf = H.tf_ptr[ty + 1] - H.tf_ptr[ty];
+        const uint32_t gt = H.col_hbase[mt.col_off + ct], gs = H.col_hbase[ms.col_off + cs];
+        for (uint32_t q = 0; q < nf; ++q) rmap[gt + q] = (int32_t)(gs + q);
+      }
+    }
+  });
+  PHASE("projection tables");
+  // ---- edges (V5, V6), parallel over source-node ranges
+  H.edges.resize(H.edges.size() + E);
+  Edge* out_edges = H.edges.data() + (H.edges.size() - E);
+  auto edge_pass = [&](uint64_t n) -> gdroid_status {
     const uint8_t kind = d->node_kind[n];
     const uint64_t m = d->node_method[n];
     int n_c2r = 0;
@@ -347,51 +518,209 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       if (ek == GE_CALL || ek == GE_RET) {
         const uint32_t sm = d->method_module[m], dm = d->method_module[d->node_method[s]];
         if (sm != dm) {
-          auto key = std::make_pair(db + sm, db + dm);
-          auto it = xmap.find(key);
-          if (it != xmap.end()) xoff = it->second;
-          else {
-            xoff = (uint32_t)H.xmap.size();
-            xmap[key] = xoff;
-            const ModRec &ms = H.mods[db + sm], &mt = H.mods[db + dm];
-            for (uint32_t c = 0; c < ms.n_cols; ++c) {      // columns: instance kept iff in Q_dst
-              int64_t cd = bsearch_idx<uint32_t>(mi[dm].insts, mi[dm].n_insts, H.col_gid[ms.col_off + c]);
-              H.xmap.push_back((int32_t)cd);
-            }
-            for (uint32_t g = 0; g < mt.n_glob; ++g) {      // global rows: slot kept iff in P_src
-              const uint32_t gid = H.grow_gid[mt.grow_off + g];
-              int32_t src = -1;
-              if (g < mt.n_stat) {                          // statics: same static visible in src
-                src = (int32_t)bsearch_idx<uint32_t>(mi[sm].stats, mi[sm].n_stats, gid - (uint32_t)Lt);
-              } else {                                      // heap: owner in Q_src, same ordinal
-                const int32_t ct = H.grow_col[mt.grow_off + g];
-                const uint32_t o = H.col_gid[mt.col_off + ct];
-                int64_t cs = bsearch_idx<uint32_t>(mi[sm].insts, mi[sm].n_insts, o);
-                if (cs >= 0) src = (int32_t)(H.col_hbase[ms.col_off + cs] + (g - H.col_hbase[mt.col_off + ct]));
-              }
-              H.xmap.push_back(src);
-            }
-          }
+          const uint64_t key = ((uint64_t)sm << 32) | dm;
+          const size_t i = std::lower_bound(pairs.begin(), pairs.end(), key) - pairs.begin();
+          xoff = (uint32_t)(xbase + pair_off[i]);
         }
       }
       const NodeRec& RS = H.nodes[nb + s];
       const uint32_t nch = n_chunks_of((uint32_t)(d->row_ptr[s + 1] - d->row_ptr[s]), RS.cls);
-      if (RS.L > 0xffff) return set_err(GDROID_E_LIMIT, "app %u: method with > 65535 locals", k);
-      Edge E{};
-      E.dst = nb + s;
-      E.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5);
-      E.off = RS.off; E.B = RS.B; E.L = (uint16_t)RS.L; E.logW = RS.logW;
-      E.aux = (ek == GE_CALL) ? (int32_t)d->method_n_params[d->node_method[s]] : (ek == GE_RET ? RS.r0 : -1);
-      E.xoff = xoff;
-      H.edges.push_back(E);
+      Edge E2{};
+      E2.dst = nb + s;
+      E2.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5);
+      E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = RS.logW;
+      E2.aux = (ek == GE_CALL) ? (int32_t)d->method_n_params[d->node_method[s]] : (ek == GE_RET ? RS.r0 : -1);
+      E2.xoff = xoff;
+      out_edges[e] = E2;
     }
     if (kind == GK_CALL && n_c2r != 1) return set_err(GDROID_E_INVALID, "app %u: node %llu: a CALL needs exactly one C2R edge (V5)", k, (unsigned long long)n);
-    H.row_ptr.push_back((uint32_t)H.edges.size());
-  }
+    return GDROID_OK;
+  };
+  parallel_ranges(N, 1 << 14, [&](uint64_t lo, uint64_t hi) {
+    for (uint64_t n = lo; n < hi; ++n) {
+      const gdroid_status st = edge_pass(n);
+      if (st != GDROID_OK) { fe.offer(n, st); return; }
+    }
+  });
+  if (fe.st != GDROID_OK) return fe.result();
+  PHASE("edges");
   for (uint64_t i = 0; i < d->n_entries; ++i) {
     if (d->entries[i] >= N || d->node_kind[d->entries[i]] != GK_ENTRY) return set_err(GDROID_E_INVALID, "app %u: entry %llu is not an ENTRY node", k, (unsigned long long)i);
     H.entries.push_back(nb + d->entries[i]);
   }
+  return GDROID_OK;
+}
+
+
+enum PartId { P_NODES, P_METHS, P_MODS, P_ROWPTR, P_EDGES, P_ARGPTR, P_ARGS, P_COLGID, P_COLTYPE,
+              P_COLHB, P_GROWGID, P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE, P_ENTRIES,
+              P_NODEMETH, P_FROW, NPART };
+
+// Device-table layout of a batch inside the staging buffer.
+struct Layout {
+  size_t off[NPART] = {};
+  size_t total = 0;
+  std::vector<uint32_t> app_base;
+  uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0;
+  uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
+};
+
+// Process-wide pinned staging buffer and per-app host images, reused by every load: in this
+// environment first-touch page faults (~1 GB/s) dominate host-side table building otherwise.
+struct LoadCache {
+  std::mutex mu;
+  void* stage = nullptr;
+  size_t cap = 0;
+  std::vector<HostImage> img;
+};
+LoadCache g_cache;
+
+void reset_image(HostImage& h) {
+  h.nodes.clear(); h.meths.clear(); h.mods.clear(); h.edges.clear(); h.args.clear();
+  h.col_gid.clear(); h.col_hbase.clear(); h.col_type.clear(); h.grow_gid.clear(); h.grow_col.clear();
+  h.grow_field.clear(); h.tf.clear(); h.xmap.clear(); h.frow.clear(); h.app_node_base.clear();
+  h.entries.clear(); h.node_method.clear();
+  h.row_ptr.assign(1, 0); h.arg_ptr.assign(1, 0); h.tf_ptr.assign(1, 0);
+  h.fact_words = 0;
+  for (auto& c : h.cls_count) c = 0;
+}
+
+size_t align256(size_t x);
+
+// Build every app's image (in parallel, app-local indices) and write the rebased batch tables
+// straight into the pinned staging buffer.  Caller holds g_cache.mu.
+gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout& Lo) {
+  if (g_cache.img.size() < n_apps) g_cache.img.resize(n_apps);
+  std::vector<HostImage>& img = g_cache.img;
+  std::vector<gdroid_status> st(n_apps, GDROID_OK);
+  std::vector<std::string> err(n_apps);
+  for (uint32_t k = 0; k < n_apps; ++k) {                  // each app is built in parallel inside
+    reset_image(img[k]);
+    st[k] = add_app(img[k], &descs[k], k);
+    if (st[k] != GDROID_OK) err[k] = g_err;
+  }
+  for (uint32_t k = 0; k < n_apps; ++k)
+    if (st[k] != GDROID_OK) { g_err = err[k]; return st[k]; }
+  PHASE("apps (parallel)");
+  struct Base { uint64_t node, edge, meth, mod, col, grow, type, tf, xmap, frow, args, fact, ent; };
+  std::vector<Base> b(n_apps + 1);
+  b[0] = Base{};
+  for (uint32_t k = 0; k < n_apps; ++k) {
+    const HostImage& h = img[k];
+    b[k + 1] = Base{b[k].node + h.nodes.size(), b[k].edge + h.edges.size(), b[k].meth + h.meths.size(),
+                    b[k].mod + h.mods.size(), b[k].col + h.col_gid.size(), b[k].grow + h.grow_gid.size(),
+                    b[k].type + (h.tf_ptr.size() - 1), b[k].tf + h.tf.size(), b[k].xmap + h.xmap.size(),
+                    b[k].frow + h.frow.size(), b[k].args + h.args.size(), b[k].fact + h.fact_words,
+                    b[k].ent + h.entries.size()};
+    for (int c = 0; c < NCLS; ++c) Lo.cls_count[c] += h.cls_count[c];
+  }
+  const Base& T = b[n_apps];
+  if (T.node >= (1ull << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
+  if (T.edge >= (1ull << 32) || T.xmap >= (1ull << 32) || T.frow >= (1ull << 31))
+    return set_err(GDROID_E_LIMIT, "batch tables exceed 32-bit indices");
+  uint64_t nc = 0;
+  for (int c = 0; c < NCLS; ++c) nc += Lo.cls_count[c];
+  if (nc >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
+  Lo.N = T.node; Lo.NC = nc; Lo.n_entries = T.ent; Lo.fact_words = T.fact;
+  Lo.app_base.resize(n_apps + 1);
+  for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
+  const size_t bytes[NPART] = {
+      T.node * sizeof(NodeRec), T.meth * sizeof(MethRec), T.mod * sizeof(ModRec), (T.node + 1) * 4,
+      T.edge * sizeof(Edge), (T.node + 1) * 4, std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4,
+      T.col * 4, T.grow * 4, T.grow * 4, T.grow * 4, (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4,
+      std::max<uint64_t>(T.xmap, 1) * 4, (n_apps + 1) * 4, std::max<uint64_t>(T.ent, 1) * 4, T.node * 4,
+      std::max<uint64_t>(T.frow, 1) * 4};
+  Lo.total = 0;
+  for (int p = 0; p < NPART; ++p) { Lo.off[p] = Lo.total; Lo.total += align256(bytes[p]); }
+  if (g_cache.cap < Lo.total) {
+    if (g_cache.stage) cudaFreeHost(g_cache.stage);
+    g_cache.stage = nullptr;
+    g_cache.cap = 0;
+    cudaError_t e = cudaMallocHost(&g_cache.stage, Lo.total + (Lo.total >> 2));
+    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "pinned staging (%zu B): %s", Lo.total, cudaGetErrorString(e));
+    g_cache.cap = Lo.total + (Lo.total >> 2);
+  }
+  char* S = (char*)g_cache.stage;
+  auto P = [&](int p) { return S + Lo.off[p]; };
+  NodeRec* g_nodes = (NodeRec*)P(P_NODES);
+  MethRec* g_meths = (MethRec*)P(P_METHS);
+  ModRec* g_mods = (ModRec*)P(P_MODS);
+  uint32_t* g_rowptr = (uint32_t*)P(P_ROWPTR);
+  Edge* g_edges = (Edge*)P(P_EDGES);
+  uint32_t* g_argptr = (uint32_t*)P(P_ARGPTR);
+  int32_t* g_args = (int32_t*)P(P_ARGS);
+  uint32_t* g_colgid = (uint32_t*)P(P_COLGID);
+  int32_t* g_coltype = (int32_t*)P(P_COLTYPE);
+  uint32_t* g_colhb = (uint32_t*)P(P_COLHB);
+  uint32_t* g_growgid = (uint32_t*)P(P_GROWGID);
+  int32_t* g_growcol = (int32_t*)P(P_GROWCOL);
+  int32_t* g_growfld = (int32_t*)P(P_GROWFLD);
+  uint32_t* g_tfptr = (uint32_t*)P(P_TFPTR);
+  uint32_t* g_tf = (uint32_t*)P(P_TF);
+  int32_t* g_xmap = (int32_t*)P(P_XMAP);
+  uint32_t* g_appbase = (uint32_t*)P(P_APPBASE);
+  uint32_t* g_entries = (uint32_t*)P(P_ENTRIES);
+  uint32_t* g_nodemeth = (uint32_t*)P(P_NODEMETH);
+  int32_t* g_frow = (int32_t*)P(P_FROW);
+  g_rowptr[0] = 0; g_argptr[0] = 0; g_tfptr[0] = 0;
+  g_args[0] = -1; g_tf[0] = 0; g_xmap[0] = -1; g_entries[0] = 0; g_frow[0] = -1;   // non-empty
+  for (uint32_t k = 0; k <= n_apps; ++k) g_appbase[k] = (uint32_t)b[k].node;
+  // work units: (app, slice of its nodes / edges) so one big app does not serialise the copy
+  constexpr size_t SLICE = 1 << 16;
+  struct Unit { uint32_t k, kind; size_t lo, hi; };
+  std::vector<Unit> units;
+  for (uint32_t k = 0; k < n_apps; ++k) {
+    const HostImage& h = img[k];
+    for (size_t lo = 0; lo < h.nodes.size(); lo += SLICE) units.push_back({k, 0, lo, std::min(h.nodes.size(), lo + SLICE)});
+    for (size_t lo = 0; lo < h.edges.size(); lo += SLICE) units.push_back({k, 1, lo, std::min(h.edges.size(), lo + SLICE)});
+    units.push_back({k, 2, 0, 0});
+  }
+  parallel_for((uint32_t)units.size(), [&](uint32_t u) {
+    const Unit U = units[u];
+    const HostImage& h = img[U.k];
+    const Base& B = b[U.k];
+    if (U.kind == 0) {
+      for (size_t i = U.lo; i < U.hi; ++i) {
+        NodeRec R = h.nodes[i];
+        R.off += B.fact; R.e0 += (uint32_t)B.edge; R.e1 += (uint32_t)B.edge;
+        R.col_off += (uint32_t)B.col; R.grow_off += (uint32_t)B.grow; R.module += (uint32_t)B.mod;
+        if (R.kind == GK_FLOAD || R.kind == GK_ALOAD) R.r3 += (int32_t)B.frow;
+        g_nodes[B.node + i] = R;
+        g_nodemeth[B.node + i] = h.node_method[i] + (uint32_t)B.meth;
+        g_rowptr[B.node + i + 1] = h.row_ptr[i + 1] + (uint32_t)B.edge;
+        g_argptr[B.node + i + 1] = h.arg_ptr[i + 1] + (uint32_t)B.args;
+      }
+      return;
+    }
+    if (U.kind == 1) {
+      for (size_t i = U.lo; i < U.hi; ++i) {
+        Edge E = h.edges[i];
+        E.dst += (uint32_t)B.node; E.off += B.fact;
+        if (E.xoff != NO_XMAP) E.xoff += (uint32_t)B.xmap;
+        g_edges[B.edge + i] = E;
+      }
+      return;
+    }
+    for (size_t i = 0; i < h.meths.size(); ++i) { MethRec M = h.meths[i]; M.module += (uint32_t)B.mod; g_meths[B.meth + i] = M; }
+    for (size_t i = 0; i < h.mods.size(); ++i) {
+      ModRec D = h.mods[i]; D.col_off += (uint32_t)B.col; D.grow_off += (uint32_t)B.grow; g_mods[B.mod + i] = D;
+    }
+    for (size_t i = 0; i < h.col_gid.size(); ++i) {
+      g_colgid[B.col + i] = h.col_gid[i];
+      g_coltype[B.col + i] = h.col_type[i] < 0 ? -1 : h.col_type[i] + (int32_t)B.type;
+      g_colhb[B.col + i] = h.col_hbase[i];
+    }
+    std::copy(h.grow_gid.begin(), h.grow_gid.end(), g_growgid + B.grow);
+    std::copy(h.grow_col.begin(), h.grow_col.end(), g_growcol + B.grow);
+    std::copy(h.grow_field.begin(), h.grow_field.end(), g_growfld + B.grow);
+    for (size_t i = 1; i < h.tf_ptr.size(); ++i) g_tfptr[B.type + i] = h.tf_ptr[i] + (uint32_t)B.tf;
+    std::copy(h.tf.begin(), h.tf.end(), g_tf + B.tf);
+    std::copy(h.xmap.begin(), h.xmap.end(), g_xmap + B.xmap);
+    std::copy(h.frow.begin(), h.frow.end(), g_frow + B.frow);
+    std::copy(h.args.begin(), h.args.end(), g_args + B.args);
+    for (size_t i = 0; i < h.entries.size(); ++i) g_entries[B.ent + i] = h.entries[i] + (uint32_t)B.node;
+  });
+  PHASE("rebase into staging");
   return GDROID_OK;
 }
 
@@ -426,9 +755,9 @@ void free_app(gdroid_app* a) {
   int cur = 0;
   cudaGetDevice(&cur);
   cudaSetDevice(a->device);
-  if (a->d_tables) cudaFree(a->d_tables);
-  if (a->d_facts) cudaFree(a->d_facts);
-  if (a->d_state) cudaFree(a->d_state);
+  if (a->d_tables) cudaFreeAsync(a->d_tables, a->stream);
+  if (a->d_facts) cudaFreeAsync(a->d_facts, a->stream);
+  if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
   if (a->d_scratch) cudaFree(a->d_scratch);
   if (a->D.trace) cudaFree(a->D.trace);
   if (a->h_stats) cudaFreeHost(a->h_stats);
@@ -488,117 +817,83 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   if (!out) return set_err(GDROID_E_INVALID, "out is NULL");
   *out = nullptr;
   if (!descs || n_apps == 0 || n_apps > 65535) return set_err(GDROID_E_INVALID, "need 1..65535 apps");
-  HostImage H;
-  for (uint32_t k = 0; k < n_apps; ++k) {
-    gdroid_status st = add_app(H, &descs[k], k);
-    if (st != GDROID_OK) return st;
-  }
-  const uint32_t N = (uint32_t)H.nodes.size();
-  const uint32_t n_entries = (uint32_t)H.entries.size();
-  // work items: every node's out-edges in at most 32 chunks (queue entry = node << 5 | chunk)
-  if (N >= (1u << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
-  uint64_t nc64 = 0;
-  for (uint32_t n = 0; n < N; ++n) {
-    const uint32_t c = n_chunks_of(H.nodes[n].e1 - H.nodes[n].e0, H.nodes[n].cls);
-    H.cls_count[H.nodes[n].cls] += c;
-    nc64 += c;
-  }
-  if (nc64 >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
-  const uint32_t NC = (uint32_t)nc64;
-  H.app_node_base.push_back(N);
-  if (H.tf.empty()) H.tf.push_back(0);          // keep every table non-empty
-  if (H.xmap.empty()) H.xmap.push_back(-1);
-  if (H.frow.empty()) H.frow.push_back(-1);
-  if (H.args.empty()) H.args.push_back(-1);
-  if (H.entries.empty()) H.entries.push_back(0);
-
+  PhaseTimer pt;
+  g_pt = &pt;
+  struct Reset { ~Reset() { g_pt = nullptr; } } reset_pt;
+  DeviceGuard guard(device);
   gdroid_app* a = new gdroid_app;
   a->device = device;
   a->stream = (cudaStream_t)cuda_stream;
   a->n_apps = n_apps;
-  a->app_base = H.app_node_base;
-  DeviceGuard guard(device);
   auto fail = [&](gdroid_status st) { free_app(a); return st; };
-
-  // ---- one table buffer, uploaded from one pinned staging buffer
-  struct Part { const void* src; size_t bytes; size_t off; };
-  std::vector<Part> parts;
-  size_t total = 0;
-  auto add = [&](const void* p, size_t bytes) { parts.push_back({p, bytes, total}); total += align256(bytes); return parts.size() - 1; };
-  size_t i_nodes = add(H.nodes.data(), H.nodes.size() * sizeof(NodeRec));
-  size_t i_meths = add(H.meths.data(), H.meths.size() * sizeof(MethRec));
-  size_t i_mods = add(H.mods.data(), H.mods.size() * sizeof(ModRec));
-  size_t i_rp = add(H.row_ptr.data(), H.row_ptr.size() * 4);
-  size_t i_e = add(H.edges.data(), H.edges.size() * sizeof(Edge));
-  size_t i_ap = add(H.arg_ptr.data(), H.arg_ptr.size() * 4);
-  size_t i_a = add(H.args.data(), H.args.size() * 4);
-  size_t i_cg = add(H.col_gid.data(), H.col_gid.size() * 4);
-  size_t i_ct = add(H.col_type.data(), H.col_type.size() * 4);
-  size_t i_ch = add(H.col_hbase.data(), H.col_hbase.size() * 4);
-  size_t i_gg = add(H.grow_gid.data(), H.grow_gid.size() * 4);
-  size_t i_gc = add(H.grow_col.data(), H.grow_col.size() * 4);
-  size_t i_gf = add(H.grow_field.data(), H.grow_field.size() * 4);
-  size_t i_tp = add(H.tf_ptr.data(), H.tf_ptr.size() * 4);
-  size_t i_tf = add(H.tf.data(), H.tf.size() * 4);
-  size_t i_xm = add(H.xmap.data(), H.xmap.size() * 4);
-  size_t i_nb = add(H.app_node_base.data(), H.app_node_base.size() * 4);
-  size_t i_en = add(H.entries.data(), H.entries.size() * 4);
-  size_t i_nm = add(H.node_method.data(), H.node_method.size() * 4);
-  size_t i_fr = add(H.frow.data(), H.frow.size() * 4);
-
+  {
+    // keep freed device memory cached in the stream-ordered pool (handles come and go per batch)
+    static bool pool_set[64] = {false};
+    if (device >= 0 && device < 64 && !pool_set[device]) {
+      cudaMemPool_t pool;
+      if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+      }
+      pool_set[device] = true;
+    }
+  }
+  Layout Lo;
   auto t0 = std::chrono::steady_clock::now();
   {
-    cudaError_t e = cudaMalloc(&a->d_tables, total);
-    if (e != cudaSuccess) return fail(set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", total, cudaGetErrorString(e)));
-    void* stage = nullptr;
-    e = cudaMallocHost(&stage, total);
-    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "pinned staging (%zu B): %s", total, cudaGetErrorString(e)));
-    for (auto& p : parts) if (p.bytes) std::memcpy((char*)stage + p.off, p.src, p.bytes);
-    e = cudaMemcpyAsync(a->d_tables, stage, total, cudaMemcpyHostToDevice, a->stream);
+    std::lock_guard<std::mutex> lock(g_cache.mu);
+    gdroid_status st = build_image(descs, n_apps, Lo);
+    if (st != GDROID_OK) return fail(st);
+    t0 = std::chrono::steady_clock::now();
+    cudaError_t e = cudaMallocAsync(&a->d_tables, Lo.total, a->stream);
+    if (e != cudaSuccess) return fail(set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", Lo.total, cudaGetErrorString(e)));
+    e = cudaMemcpyAsync(a->d_tables, g_cache.stage, Lo.total, cudaMemcpyHostToDevice, a->stream);
     cudaError_t e2 = cudaStreamSynchronize(a->stream);
-    cudaFreeHost(stage);
     if (e != cudaSuccess || e2 != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "H2D upload: %s", cudaGetErrorString(e != cudaSuccess ? e : e2)));
   }
   a->h2d_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
+  PHASE("upload");
+  a->app_base = Lo.app_base;
+  const uint32_t N = (uint32_t)Lo.N, NC = (uint32_t)Lo.NC;
   char* T = (char*)a->d_tables;
   Dev& D = a->D;
-  D.nodes = (const NodeRec*)(T + parts[i_nodes].off);
-  D.meths = (const MethRec*)(T + parts[i_meths].off);
-  D.mods = (const ModRec*)(T + parts[i_mods].off);
-  D.row_ptr = (const uint32_t*)(T + parts[i_rp].off);
-  D.edges = (const Edge*)(T + parts[i_e].off);
-  D.arg_ptr = (const uint32_t*)(T + parts[i_ap].off);
-  D.args = (const int32_t*)(T + parts[i_a].off);
-  D.col_gid = (const uint32_t*)(T + parts[i_cg].off);
-  D.col_type = (const int32_t*)(T + parts[i_ct].off);
-  D.col_hbase = (const uint32_t*)(T + parts[i_ch].off);
-  D.grow_gid = (const uint32_t*)(T + parts[i_gg].off);
-  D.grow_col = (const int32_t*)(T + parts[i_gc].off);
-  D.grow_field = (const int32_t*)(T + parts[i_gf].off);
-  D.tf_ptr = (const uint32_t*)(T + parts[i_tp].off);
-  D.tf = (const uint32_t*)(T + parts[i_tf].off);
-  D.xmap = (const int32_t*)(T + parts[i_xm].off);
-  D.app_node_base = (const uint32_t*)(T + parts[i_nb].off);
-  D.entries = (const uint32_t*)(T + parts[i_en].off);
-  D.node_method = (const uint32_t*)(T + parts[i_nm].off);
-  D.frow = (const int32_t*)(T + parts[i_fr].off);
+  D.nodes = (const NodeRec*)(T + Lo.off[P_NODES]);
+  D.meths = (const MethRec*)(T + Lo.off[P_METHS]);
+  D.mods = (const ModRec*)(T + Lo.off[P_MODS]);
+  D.row_ptr = (const uint32_t*)(T + Lo.off[P_ROWPTR]);
+  D.edges = (const Edge*)(T + Lo.off[P_EDGES]);
+  D.arg_ptr = (const uint32_t*)(T + Lo.off[P_ARGPTR]);
+  D.args = (const int32_t*)(T + Lo.off[P_ARGS]);
+  D.col_gid = (const uint32_t*)(T + Lo.off[P_COLGID]);
+  D.col_type = (const int32_t*)(T + Lo.off[P_COLTYPE]);
+  D.col_hbase = (const uint32_t*)(T + Lo.off[P_COLHB]);
+  D.grow_gid = (const uint32_t*)(T + Lo.off[P_GROWGID]);
+  D.grow_col = (const int32_t*)(T + Lo.off[P_GROWCOL]);
+  D.grow_field = (const int32_t*)(T + Lo.off[P_GROWFLD]);
+  D.tf_ptr = (const uint32_t*)(T + Lo.off[P_TFPTR]);
+  D.tf = (const uint32_t*)(T + Lo.off[P_TF]);
+  D.xmap = (const int32_t*)(T + Lo.off[P_XMAP]);
+  D.app_node_base = (const uint32_t*)(T + Lo.off[P_APPBASE]);
+  D.entries = (const uint32_t*)(T + Lo.off[P_ENTRIES]);
+  D.node_method = (const uint32_t*)(T + Lo.off[P_NODEMETH]);
+  D.frow = (const int32_t*)(T + Lo.off[P_FROW]);
   D.n_nodes = N;
   D.n_chunks = NC;
-  D.n_entries = n_entries;
+  D.n_entries = (uint32_t)Lo.n_entries;
   uint32_t acc = 0;
-  for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += H.cls_count[c]; }
+  for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += Lo.cls_count[c]; }
   D.seg[NCLS] = acc;
-  D.n_words = H.fact_words;
+  D.n_words = Lo.fact_words;
 
   // ---- fact store + mutable state
   {
-    cudaError_t e = cudaMalloc(&a->d_facts, std::max<uint64_t>(H.fact_words, 4) * 8);
-    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(H.fact_words * 8), cudaGetErrorString(e)));
+    cudaError_t e = cudaMallocAsync(&a->d_facts, std::max<uint64_t>(Lo.fact_words, 4) * 8, a->stream);
+    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(Lo.fact_words * 8), cudaGetErrorString(e)));
     D.facts = a->d_facts;
     size_t s_stamp = align256((size_t)N * 4), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t st = s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
-    e = cudaMalloc(&a->d_state, st);
+    e = cudaMallocAsync(&a->d_state, st, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "device state (%zu B): %s", st, cudaGetErrorString(e)));
     char* S = (char*)a->d_state;
     D.stamp = (uint32_t*)S; S += s_stamp;

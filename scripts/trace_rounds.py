@@ -14,6 +14,8 @@ if wl == "chain":   # a long NOP chain: one item per round -> barrier + one-item
     b = IcfgBuilder(n_fields=1); d = b.add_module(); m = b.add_method(d, 0, 2)
     nodes = [b.nop(m) for _ in range(4000)]
     b.chain(b.entry(m), *nodes, b.exit(m)); b.add_entry(m); gs = [b.build()]
+elif wl == "corpus27":
+    gs = [G.corpus_app(27)]
 elif wl == "corpus8":
     gs = [G.corpus_app(i) for i in range(8)]
 else:
