@@ -31,7 +31,7 @@ struct __align__(16) NodeRec {
   int32_t r1;        // rhs row (COPY/SLOAD/SSTORE/RETV), w row (FLOAD/ALOAD/FSTORE/ASTORE),
                      // n_params of the method (ENTRY), argument rows r1..r3 (CALL with <= 3 args)
   int32_t r2;        // field id (FLOAD/FSTORE; F_ARR for ALOAD/ASTORE)
-  int32_t r3;        // instance column (CONST/NEW); field-row table offset (FLOAD/ALOAD)
+  int32_t r3;        // instance column (CONST/NEW); field-row table offset (FLOAD/FSTORE/ALOAD/ASTORE)
   uint32_t B;        // words of the block = (L + n_glob) << logW
   uint32_t L;        // method-local rows (params, temps, RET)
   uint32_t n_stat;   // module static rows
@@ -42,6 +42,13 @@ struct __align__(16) NodeRec {
   uint32_t module;   // global module index
 };
 static_assert(sizeof(NodeRec) == 64, "NodeRec must be 64 bytes");
+
+// Wide blocks (modules with more than 64 instances, logW >= 1) carry a row-occupancy bitmap
+// after the rows: bit r set = row r may be non-zero.  Writers set it, readers visit only the
+// flagged rows (a fact written after the reader's bitmap load is re-processed next round,
+// because its writer also queued the node).
+__host__ __device__ __forceinline__ uint32_t occ_offset(uint32_t B) { return (B + 3u) & ~3u; }
+__host__ __device__ __forceinline__ uint32_t occ_words(uint32_t rows) { return (rows + 63u) >> 6; }
 
 // Work items.  A node's out-edges are split into chunks of ebs(deg) edges (at most 32 chunks
 // per node); a queue entry is (node << 5) | chunk.  High-degree nodes (method exits with many
@@ -130,6 +137,7 @@ struct Dev {
   uint32_t n_entries;
   uint32_t seg[NCLS + 1];       // class segment starts inside one queue
   uint32_t max_rounds;
+  uint32_t wide;                // 1 if some module has > 64 instances (row-occupancy path)
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
   uint32_t trace_cap;           // rounds recorded (0 = off)
 };
@@ -142,6 +150,6 @@ cudaError_t launch_digest(const Dev& D, cudaStream_t s);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,
                           uint64_t* pairs, cudaStream_t s);
-int fixpoint_max_blocks(int device);
+int fixpoint_max_blocks(int device, bool wide);
 
 }  // namespace gd

@@ -38,7 +38,9 @@ struct Acc {                   // per-warp counters (shared memory), flushed onc
 struct WarpScratch {
   uint64_t rv[MAXW];           // FSTORE base row v
   uint64_t rw[MAXW];           // FSTORE / FLOAD value row w
+  uint64_t gen[MAXW];          // generated row (wide path)
   int16_t cmap[64 * MAXW];     // projection column map of the current cross-module edge
+  uint16_t rowlist[1024];      // rows visited by the wide path
 };
 
 // warp-uniform counter updates: lane 0 adds the warp's total
@@ -177,7 +179,220 @@ __device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uin
   return nz | (red << 16);
 }
 
+// ---------------------------------------------------------------------------------- wide blocks
+// Row-sparse processing of a node whose block is wide (W >= 2 words per row): only the rows
+// flagged in its occupancy bitmap (plus the rows its transfer function generates) are read,
+// transformed and propagated; every row written into a wide target also sets the target's
+// occupancy bit.  Same results as the dense path, bytes proportional to non-zero rows.
+constexpr int WROWS = 1024;    // row-list capacity per warp (rows of one block)
+
+__device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_t logWt, uint32_t rt,
+                                               const uint64_t (&v)[MAXW], uint32_t& nz, uint32_t& red, bool& g) {
+  const uint32_t Wt = 1u << logWt;
+  uint64_t* row = Z + ((uint64_t)rt << logWt);
+  uint64_t cur[MAXW];
+  bool any = false, was_zero = true;
+#pragma unroll
+  for (int j = 0; j < MAXW; ++j) {
+    cur[j] = (j < (int)Wt && v[j]) ? row[j] : ~0ull;
+    any |= (j < (int)Wt && v[j] != 0);
+  }
+  if (!any) return;
+#pragma unroll
+  for (int j = 0; j < MAXW; ++j) {
+    if (j >= (int)Wt || !v[j]) continue;
+    ++nz;
+    if (cur[j]) was_zero = false;
+    if (v[j] & ~cur[j]) { red_or(row + j, v[j]); ++red; g = true; }
+  }
+  if (logWt >= 1 && was_zero) red_or(Z + occ_offset(Bt) + (rt >> 6), 1ull << (rt & 63));   // occupancy
+}
+
+__device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
+                             bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
+                             uint32_t alg_l0) {
+  const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B, rows = B >> logW;
+  const uint64_t* __restrict__ X = D.facts + R.off;
+  const uint64_t* __restrict__ OCC = X + occ_offset(B);
+  const uint32_t nocc = occ_words(rows);
+  const uint32_t kind = R.kind;
+  // ---- transfer setup: generated row t (mode 1 replace / 2 or-in) or FSTORE rows (mode 3)
+  int mode = 0, t = -1;
+  uint32_t hwords = 0;
+  if (lane < MAXW) ws.gen[lane] = 0;
+  if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
+    mode = 1; t = R.r0;
+    if (kind != GK_PRIM && lane == (R.r3 >> 6)) ws.gen[lane] = 1ull << (R.r3 & 63);
+  } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
+    mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
+    if (lane < (int)W) ws.gen[lane] = X[((uint64_t)R.r1 << logW) + lane];
+  } else if (kind == GK_FLOAD || kind == GK_ALOAD) {
+    mode = 1; t = R.r0;
+    if (lane < (int)W) ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
+    __syncwarp();
+    uint64_t a[MAXW];
+#pragma unroll
+    for (int j = 0; j < MAXW; ++j) a[j] = 0;
+    for (uint32_t c = lane; c < R.n_cols; c += 32) {
+      if (!((ws.rw[c >> 6] >> (c & 63)) & 1ull)) continue;
+      const int hr = D.frow[R.r3 + c];
+      if (hr < 0) continue;                                  // NULL / field not declared
+      const uint64_t* H = X + ((uint64_t)(L + hr) << logW);
+#pragma unroll
+      for (int j = 0; j < MAXW; ++j)
+        if (j < (int)W) a[j] |= H[j];
+      hwords += W;
+    }
+#pragma unroll
+    for (int j = 0; j < MAXW; ++j)
+      if (j < (int)W) {
+        const uint64_t v = warp_or64(a[j]);
+        if (lane == j) ws.gen[j] = v;
+      }
+  } else if (kind == GK_FSTORE || kind == GK_ASTORE) {
+    mode = 3;
+    if (lane < (int)W) {
+      ws.rv[lane] = X[((uint64_t)R.r0 << logW) + lane];
+      ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
+    }
+  }
+  __syncwarp();
+  // ---- row list: flagged rows, then the generated rows that are not flagged yet
+  const unsigned lt_mask = (1u << lane) - 1u;
+  const uint64_t my_occ = lane < (int)nocc ? OCC[lane] : 0ull;   // nocc <= 32 (loader: rows <= WROWS)
+  uint32_t cnt = 0;
+  for (uint32_t i = 0; i < nocc; ++i) {
+    const uint64_t wv = __shfl_sync(FULL, my_occ, i);
+    const uint32_t lo = (uint32_t)wv, hi = (uint32_t)(wv >> 32);
+    if ((lo >> lane) & 1u) ws.rowlist[cnt + __popc(lo & lt_mask)] = (uint16_t)(i * 64 + lane);
+    if ((hi >> lane) & 1u) ws.rowlist[cnt + __popc(lo) + __popc(hi & lt_mask)] = (uint16_t)(i * 64 + 32 + lane);
+    cnt += __popc(lo) + __popc(hi);
+  }
+  if (mode == 1 || mode == 2) {
+    const uint64_t wv = __shfl_sync(FULL, my_occ, (uint32_t)t >> 6);
+    if (!((wv >> (t & 63)) & 1ull)) { if (lane == 0) ws.rowlist[cnt] = (uint16_t)t; ++cnt; }
+  } else if (mode == 3) {                                    // heap rows (o1, f), o1 in row v
+    for (uint32_t c0 = 0; c0 < R.n_cols; c0 += 32) {
+      const uint32_t c = c0 + lane;
+      int hr = -1;
+      if (c < R.n_cols && ((ws.rv[c >> 6] >> (c & 63)) & 1ull)) hr = D.frow[R.r3 + c];
+      const uint32_t r = hr >= 0 ? L + (uint32_t)hr : 0u;
+      const uint64_t wv = __shfl_sync(FULL, my_occ, r >> 6);
+      const bool need = hr >= 0 && !((wv >> (r & 63)) & 1ull);
+      const unsigned m = __ballot_sync(FULL, need);
+      if (need) ws.rowlist[cnt + __popc(m & lt_mask)] = (uint16_t)r;
+      cnt += __popc(m);
+    }
+  }
+  __syncwarp();
+
+  uint32_t nzx = 0, nz = 0, red = 0;
+  unsigned long long dense_l0 = first ? 8ull * B : 0ull;
+  for (uint32_t eb = e0; eb < e1; eb += 32) {
+    const uint32_t ne = min(32u, e1 - eb);
+    const uint32_t my_info = lane < (int)ne ? D.edges[eb + lane].info : 0u;
+    unsigned gmask = 0;
+    for (uint32_t i = 0; i < ne; ++i) {
+      const Edge* ep = D.edges + eb + i;
+      const uint32_t ek = ep->info & 3u;
+      uint64_t* Z = D.facts + ep->off;
+      const uint32_t Bt = ep->B, Lt = ep->L, logWt = ep->logW;
+      const int aux = ep->aux;
+      const uint32_t xoff = ep->xoff;
+      const bool proj = (ek == GE_CALL || ek == GE_RET) && xoff != NO_XMAP;
+      if (proj) {
+        for (uint32_t c = lane; c < R.n_cols; c += 32) ws.cmap[c] = (int16_t)D.xmap[xoff + c];
+        __syncwarp();
+      }
+      const int32_t* rowinv = proj ? D.xmap + xoff + R.n_cols + ((Bt >> logWt) - Lt) : nullptr;
+      const uint32_t npar = (ek == GE_CALL) ? (uint32_t)aux : 0u;
+      const int lhs = (ek == GE_RET) ? aux : -1;
+      bool g = false;
+      for (uint32_t p = lane; p < cnt; p += 32) {
+        const uint32_t r = ws.rowlist[p];
+        // Y row r = f(X) row r
+        uint64_t y[MAXW];
+#pragma unroll
+        for (int j = 0; j < MAXW; ++j) y[j] = (j < (int)W) ? X[((uint64_t)r << logW) + j] : 0ull;
+        if (first && eb == e0 && i == 0) {
+#pragma unroll
+          for (int j = 0; j < MAXW; ++j) nzx += (j < (int)W && y[j] != 0);
+        }
+        if (mode == 1 && (int)r == t) {
+#pragma unroll
+          for (int j = 0; j < MAXW; ++j) y[j] = (j < (int)W) ? ws.gen[j] : 0ull;
+        } else if (mode == 2 && (int)r == t) {
+#pragma unroll
+          for (int j = 0; j < MAXW; ++j) if (j < (int)W) y[j] |= ws.gen[j];
+        } else if (mode == 3 && r >= L + R.n_stat) {
+          const uint32_t gg = r - L;
+          if (D.grow_field[R.grow_off + gg] == R.r2) {
+            const int c = D.grow_col[R.grow_off + gg];
+            if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) {
+#pragma unroll
+              for (int j = 0; j < MAXW; ++j) if (j < (int)W) y[j] |= ws.rw[j];
+            }
+          }
+        }
+        // target rows
+        int rt[3] = {-1, -1, -1};
+        if (ek == GE_INTRA) rt[0] = (int)r;
+        else if (ek == GE_C2R) rt[0] = ((int)r == R.r0) ? -1 : (int)r;
+        else if (r >= L) {
+          const uint32_t gs = r - L;
+          const int gt = proj ? rowinv[gs] : (int)gs;       // π: source global row -> target row
+          if (gt >= 0) rt[0] = (int)Lt + gt;
+        } else if (ek == GE_RET) {
+          if (r == L - 1 && lhs >= 0) rt[0] = lhs;
+        } else {
+          int k2 = 0;
+          for (uint32_t jj = 0; jj < npar && k2 < 3; ++jj) {
+            const int a = npar > 3 ? D.args[D.arg_ptr[n] + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
+            if (a == (int)r) rt[k2++] = (int)jj;
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+          if (rt[q] < 0) continue;
+          if (!proj) {
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], y, nz, red, g);
+          } else {
+            uint64_t out[MAXW];
+#pragma unroll
+            for (int s2 = 0; s2 < MAXW; ++s2) out[s2] = 0;
+            for (uint32_t j = 0; j < W; ++j) {
+              uint64_t b = 0;
+#pragma unroll
+              for (int jj = 0; jj < MAXW; ++jj) if ((uint32_t)jj == j) b = y[jj];
+              while (b) {
+                const int bit = __ffsll((long long)b) - 1;
+                b &= b - 1;
+                const int cd = ws.cmap[j * 64 + bit];
+                if (cd < 0) continue;
+#pragma unroll
+                for (int s2 = 0; s2 < MAXW; ++s2)
+                  if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
+              }
+            }
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], out, nz, red, g);
+          }
+        }
+      }
+      if (proj) __syncwarp();
+      g = __any_sync(FULL, g);
+      if (g) gmask |= 1u << i;
+      dense_l0 += 16ull * Bt;
+    }
+    const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt);
+  }
+  acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
+  acc_add(acc.atom, red);
+  if (lane == 0) acc.dense += dense_l0 + alg_l0;
+}
+
 // ---------------------------------------------------------------------------------- one item
+template <bool WIDE>
 __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                              uint32_t nxt, int lane, WarpScratch& ws, Acc& acc) {
   const NodeRec R = D.nodes[n];
@@ -189,6 +404,12 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
   if (e0 >= e1) {                                           // no successor: nothing to propagate
     if (lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
     return;
+  }
+  if constexpr (WIDE) {
+    if (logW >= 1) {                                        // wide block: row-sparse path
+      process_wide(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0);
+      return;
+    }
   }
   const uint64_t* __restrict__ X = D.facts + R.off;
 
@@ -367,7 +588,7 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
             }
           }
           __syncwarp();
-          if (W == 1 && logWt == 0) {                       // one word per row on both sides
+          if (!WIDE || (W == 1 && logWt == 0)) {            // one word per row on both sides
             uint64_t v[KW], cur[KW];
 #pragma unroll
             for (int k = 0; k < KW; ++k) v[k] = src[k] >= 0 ? X[src[k]] : 0ull;
@@ -392,7 +613,7 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
                 g = true;
               }
             }
-          } else {
+          } else if constexpr (WIDE) {
 #pragma unroll
             for (int k = 0; k < KW; ++k) {
               if (src[k] < 0) continue;
@@ -412,14 +633,7 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
                     if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
                 }
               }
-#pragma unroll
-              for (int q = 0; q < MAXW; ++q) {
-                if (q < (1 << logWt) && out[q]) {
-                  uint64_t* p = Z + ((uint64_t)r << logWt) + q;
-                  ++nz;
-                  if (out[q] & ~*p) { red_or(p, out[q]); ++red; g = true; }
-                }
-              }
+              emit_row_words(Z, Bt, logWt, r, out, nz, red, g);   // sets occupancy if wide
             }
           }
         }
@@ -467,6 +681,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 
 // Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
+template <bool WIDE>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
@@ -517,13 +732,14 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
     if (nitem < total && lane < 4)                                     // and its NodeRec into L1
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
-    process_item(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc);
+    process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc);
     item = nitem;
     entry = nentry;
   }
   return total;
 }
 
+template <bool WIDE>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -535,7 +751,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   stage_init(st);
   __syncthreads();
   for (uint32_t round = 1;; ++round) {
-    const uint32_t total = run_round(D, st, round, gw, nw, lane, ws_all[wib], acc);
+    const uint32_t total = run_round<WIDE>(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == 0) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
@@ -547,6 +763,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   flush_acc(D, acc);
 }
 
+template <bool WIDE>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t round) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -557,7 +774,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   if (lane == 0) acc = Acc{0, 0, 0};
   stage_init(st);
   __syncthreads();
-  const uint32_t total = run_round(D, st, round, gw, nw, lane, ws_all[wib], acc);
+  const uint32_t total = run_round<WIDE>(D, st, round, gw, nw, lane, ws_all[wib], acc);
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);
@@ -669,21 +886,26 @@ cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-int fixpoint_max_blocks(int device) {
+int fixpoint_max_blocks(int device, bool wide) {
   int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint, THREADS, 0);
+  if (wide) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<true>, THREADS, 0);
+  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<false>, THREADS, 0);
   return sms * (occ > 0 ? occ : 1);
 }
 
+// The wide (row-sparse) path is compiled into a separate instantiation so batches without wide
+// modules keep the dense path's register allocation.
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s) {
   Dev d = D;
   void* args[] = {&d};
-  return cudaLaunchCooperativeKernel((const void*)k_fixpoint, dim3(blocks), dim3(THREADS), args, 0, s);
+  const void* f = D.wide ? (const void*)k_fixpoint<true> : (const void*)k_fixpoint<false>;
+  return cudaLaunchCooperativeKernel(f, dim3(blocks), dim3(THREADS), args, 0, s);
 }
 
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s) {
-  k_round<<<blocks, THREADS, 0, s>>>(D, round);
+  if (D.wide) k_round<true><<<blocks, THREADS, 0, s>>>(D, round);
+  else k_round<false><<<blocks, THREADS, 0, s>>>(D, round);
   return cudaGetLastError();
 }
 

@@ -264,8 +264,10 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     for (uint64_t n = lo; n < hi; ++n) {
       const uint64_t m = d->node_method[n];
       const ModRec& md = H.mods[db + d->method_module[m]];
-      const uint64_t words = (uint64_t)(d->method_n_locals[m] + md.n_glob) << md.logW;
+      const uint64_t rows = d->method_n_locals[m] + md.n_glob;
+      const uint64_t words = rows << md.logW;
       foff[n + 1] = (words + 3) & ~3ull;                        // 32-byte aligned blocks
+      if (md.logW >= 1) foff[n + 1] += (((rows + 63) >> 6) + 3) & ~3ull;   // wide: row-occupancy words
     }
   });
   for (uint64_t n = 0; n < N; ++n) foff[n + 1] += foff[n];
@@ -275,8 +277,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     std::unordered_map<uint64_t, uint32_t> frow_map;
     for (uint64_t n = 0; n < N; ++n) {
       const uint8_t kind = d->node_kind[n];
-      if (kind != GK_FLOAD && kind != GK_ALOAD) continue;
-      const int32_t f = (kind == GK_ALOAD) ? (int32_t)GDROID_F_ARR : d->node_ops[4 * n + 2];
+      if (kind != GK_FLOAD && kind != GK_ALOAD && kind != GK_FSTORE && kind != GK_ASTORE) continue;
+      const int32_t f = (kind == GK_ALOAD || kind == GK_ASTORE) ? (int32_t)GDROID_F_ARR : d->node_ops[4 * n + 2];
       if (f < 0 || (uint32_t)f >= d->n_fields) continue;       // reported by the node pass
       const uint64_t dd = d->method_module[d->node_method[n]];
       const uint64_t key = (dd << 32) | (uint32_t)f;
@@ -353,7 +355,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           if (op[2] < 0 || (uint32_t)op[2] >= d->n_fields) return set_err(GDROID_E_INVALID, "app %u: node %llu: field out of range", k, (unsigned long long)n);
           R.r2 = op[2];
         }
-        if (kind == GK_FLOAD || kind == GK_ALOAD) R.r3 = frow_of[n];   // heap row of (o1, f) per column
+        R.r3 = frow_of[n];                                   // heap row of (o1, f) per column
         break;
       case GK_SLOAD:
         if (!need_local(op[0], R.r0, "lhs")) return GDROID_E_POOL;
@@ -392,6 +394,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     const uint64_t words = (uint64_t)(L + md.n_glob) << md.logW;
     if (words >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: node %llu: fact block too large", k, (unsigned long long)n);
     if (L > 0xffff) return set_err(GDROID_E_LIMIT, "app %u: node %llu: method with > 65535 locals", k, (unsigned long long)n);
+    if (md.logW >= 1 && L + md.n_glob > 1024) return set_err(GDROID_E_LIMIT, "app %u: node %llu: wide block with > 1024 rows", k, (unsigned long long)n);
     R.off = H.fact_words + foff[n];
     R.B = (uint32_t)words; R.L = L; R.n_stat = md.n_stat;
     R.e0 = (uint32_t)d->row_ptr[n]; R.e1 = (uint32_t)d->row_ptr[n + 1];
@@ -444,7 +447,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   std::vector<uint32_t> pair_off(pairs.size() + 1, 0);
   for (size_t i = 0; i < pairs.size(); ++i) {
     const ModRec &ms = H.mods[db + (pairs[i] >> 32)], &mt = H.mods[db + (uint32_t)pairs[i]];
-    pair_off[i + 1] = pair_off[i] + ms.n_cols + mt.n_glob;
+    pair_off[i + 1] = pair_off[i] + ms.n_cols + mt.n_glob + ms.n_glob;   // colmap, rowmap, rowinv
   }
   const size_t xbase = H.xmap.size();
   H.xmap.resize(xbase + pair_off[pairs.size()], -1);
@@ -477,6 +480,9 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
         const uint32_t gt = H.col_hbase[mt.col_off + ct], gs = H.col_hbase[ms.col_off + cs];
         for (uint32_t q = 0; q < nf; ++q) rmap[gt + q] = (int32_t)(gs + q);
       }
+      int32_t* rinv = rmap + mt.n_glob;                        // src global row -> dst global row
+      for (uint32_t g = 0; g < mt.n_glob; ++g)
+        if (rmap[g] >= 0) rinv[rmap[g]] = (int32_t)g;
     }
   });
   PHASE("projection tables");
@@ -563,6 +569,7 @@ struct Layout {
   std::vector<uint32_t> app_base;
   uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
+  bool wide = false;
 };
 
 // Process-wide pinned staging buffer and per-app host images, reused by every load: in this
@@ -613,6 +620,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
                     b[k].frow + h.frow.size(), b[k].args + h.args.size(), b[k].fact + h.fact_words,
                     b[k].ent + h.entries.size()};
     for (int c = 0; c < NCLS; ++c) Lo.cls_count[c] += h.cls_count[c];
+    for (const ModRec& md : h.mods) Lo.wide |= md.logW >= 1;
   }
   const Base& T = b[n_apps];
   if (T.node >= (1ull << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
@@ -684,7 +692,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
         NodeRec R = h.nodes[i];
         R.off += B.fact; R.e0 += (uint32_t)B.edge; R.e1 += (uint32_t)B.edge;
         R.col_off += (uint32_t)B.col; R.grow_off += (uint32_t)B.grow; R.module += (uint32_t)B.mod;
-        if (R.kind == GK_FLOAD || R.kind == GK_ALOAD) R.r3 += (int32_t)B.frow;
+        if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)B.frow;
         g_nodes[B.node + i] = R;
         g_nodemeth[B.node + i] = h.node_method[i] + (uint32_t)B.meth;
         g_rowptr[B.node + i + 1] = h.row_ptr[i + 1] + (uint32_t)B.edge;
@@ -884,6 +892,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += Lo.cls_count[c]; }
   D.seg[NCLS] = acc;
   D.n_words = Lo.fact_words;
+  D.wide = Lo.wide ? 1u : 0u;
 
   // ---- fact store + mutable state
   {
@@ -908,7 +917,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     for (auto& ev : a->ev)
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
-  a->max_blocks = fixpoint_max_blocks(device);
+  a->max_blocks = fixpoint_max_blocks(device, D.wide != 0);
   *out = a;
   return GDROID_OK;
 }
