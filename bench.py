@@ -132,24 +132,30 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def ncu_traffic():
-    """Per-launch DRAM bytes of k_fixpoint from the committed ncu summary, if any."""
+def ncu_traffic(workload, apps_per_rank):
+    """Per-launch DRAM bytes of k_fixpoint from the committed ncu summary of THIS workload
+    (profiles/ncu_summary.json, written by scripts/ncu_summary.py), else None."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as fh:
             d = json.load(fh)
-        return d.get("k_fixpoint", {}).get("dram_bytes_per_launch"), d.get("workload")
+        for cap in d.get("captures", [d]):
+            if cap.get("bench_workload") == workload and cap.get("apps_per_rank", apps_per_rank) == apps_per_rank:
+                return cap.get("k_fixpoint", {}).get("dram_bytes_per_launch"), cap.get("workload")
     except Exception:
-        return None, None
+        pass
+    return None, None
 
 
 # ------------------------------------------------------------------ CPU oracle legs
 def oracle_sample(apps, seconds):
-    """Time the oracle (as it stands, single-threaded) on apps of the workload until ~seconds."""
+    """Time the oracle (as it stands, single-threaded) on apps of the workload, cycling through
+    them until about `seconds` of CPU work (at most 64 runs)."""
     import oracle
     t0 = time.perf_counter()
     done, visits, app_s = 0, 0, []
-    for g in apps:
+    while done < 64:
+        g = apps[done % len(apps)]
         r = oracle.build_idfg(g)
         done += 1
         visits += r.visits
@@ -283,7 +289,7 @@ def run_ours(args):
     fix_ms = statistics.mean(fix_ns) / 1e6
     peak, peak_src = measured_peak()
     achieved = alg / (statistics.mean(fix_ns) / 1e9) / 1e9     # GB/s, touched-word model
-    traffic, traffic_wl = ncu_traffic()
+    traffic, traffic_wl = ncu_traffic(args.workload, desc["apps_per_rank"])
     clocks = clk.summary()
     line = {
         "metric": METRIC, "value": value, "unit": "apps/s", "n_gpus": world,
@@ -321,8 +327,8 @@ def run_ours(args):
         s = oracle_sample(apps, args.cpu_seconds)
         line["cpu_baseline"] = {"value": s["apps"] / s["wall_s"], "unit": "apps/s", "cores": 1,
                                 "kind": "oracle",
-                                "sample": f"{s['apps']} app(s) of rank 0's shard, single-threaded "
-                                          f"({s['wall_s']:.1f} s)",
+                                "sample": f"{s['apps']} oracle run(s) over rank 0's {len(apps)} app(s), "
+                                          f"single-threaded ({s['wall_s']:.1f} s)",
                                 "node_visits_per_s": s["visits"] / s["wall_s"]}
     print(json.dumps(line), flush=True)
     if world > 1:

@@ -18,6 +18,13 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "l1tex__t_sector_hit_rate.pct", "lts__t_sector_hit_rate.pct"]
 
 
+def kname(full):
+    """'void gd::<unnamed>::k_fixpoint<(bool)1>(gd::Dev)' -> 'k_fixpoint'"""
+    import re
+    m = re.search(r"(k_[a-z_]+)", full)
+    return m.group(1) if m else full.split("(")[0].split("::")[-1]
+
+
 def raw(rep):
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
@@ -53,7 +60,7 @@ def launches(path):
             v = float(r["Metric Value"].replace(",", ""))
             unit = r.get("Metric Unit", "ns")
             scale = {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "ns": 1e-6, "us": 1e-3, "ms": 1.0}.get(unit, 1e-6)
-            name = r["Kernel Name"].split("(")[0].split("::")[-1]
+            name = kname(r["Kernel Name"])
             per[name].append(v * scale)
     tot = sum(sum(v) for v in per.values())
     return {k: {"launches": len(v), "total_ms": round(sum(v), 4), "share": round(sum(v) / tot, 4)}
@@ -64,8 +71,11 @@ def main():
     rep, lcsv, prefix = sys.argv[1:4]
     wl = sys.argv[4] if len(sys.argv) > 4 else ""
     summary = {"workload": wl, "launch_list": launches(lcsv) if lcsv != "-" else None}
+    if len(sys.argv) > 5:
+        summary["bench_workload"] = sys.argv[5]
+        summary["apps_per_rank"] = int(sys.argv[6]) if len(sys.argv) > 6 else 1
     for d, u in raw(rep):
-        name = d.get("Kernel Name", "?").split("(")[0].split("::")[-1]
+        name = kname(d.get("Kernel Name", "?"))
         m = {k: d.get(k) for k in KEYS if k in d}
         m["units"] = {k: u.get(k) for k in KEYS if k in d}
         m["stall_pct"] = stalls(d)
