@@ -19,7 +19,10 @@ _STMT_KINDS = [NOP, PRIM, CONST, NEW, COPY, SLOAD, SSTORE, RETV, FLOAD, FSTORE,
 
 def random_tiny(seed: int, n_methods: int = None, n_modules: int = None,
                 max_stmts: int = 5, full_pools: bool = False,
-                kinds: List = None, allow_calls: bool = True) -> Icfg:
+                kinds: List = None, allow_calls: bool = True, wide_pad: int = 0) -> Icfg:
+    """wide_pad > 0 adds that many never-allocated instances to every module pool (half with
+    lower gids than the real sites, half higher), so pools exceed 64 instances and the CUDA
+    path takes its wide-block (row-occupancy) route with sites straddling word boundaries."""
     rng = random.Random(seed)
     n_fields = rng.randint(1, 3)                 # field 0 = F_ARR
     b = IcfgBuilder(n_fields=n_fields)
@@ -29,6 +32,7 @@ def random_tiny(seed: int, n_methods: int = None, n_modules: int = None,
     n_statics = rng.randint(0, 2)
     for _ in range(n_statics):
         b.add_static()
+    pad_lo = [b.add_instance(rng.choice(types)) for _ in range(wide_pad // 2)]
     M = n_methods or rng.randint(1, 3)
     D = n_modules or rng.randint(1, min(2, M))
     mods = [b.add_module() for _ in range(D)]
@@ -116,13 +120,14 @@ def random_tiny(seed: int, n_methods: int = None, n_modules: int = None,
             src = rng.choice(heads)[1]
             dst = rng.choice(heads + [(b.exit(m), b.exit(m))])[0]
             b.edge(src, dst, E_INTRA)
+    pad_hi = [b.add_instance(rng.choice(types)) for _ in range(wide_pad - wide_pad // 2)]
     all_insts = list(range(1, len(b.inst_type)))
     for d in mods:
         extra = [] if full_pools else [o for o in all_insts if rng.random() < 0.5]
         insts = all_insts if full_pools else mod_sites[d] + extra
         stats = list(range(n_statics)) if (full_pools or rng.random() < 0.5) else \
             sorted(mod_stat_used[d] | {g for g in range(n_statics) if rng.random() < 0.5})
-        b.set_module(d, insts=insts, statics=stats)
+        b.set_module(d, insts=list(insts) + pad_lo + pad_hi, statics=stats)
     b.add_entry(meths[0])
     if M > 1 and rng.random() < 0.3:
         b.add_entry(meths[-1])

@@ -126,3 +126,28 @@ def test_empty_and_degenerate():
     assert len(pairs) == 0
     r = oracle.build_idfg(g)
     assert r.app_digest == app.node_digests()[1] == 0
+
+
+@pytest.mark.parametrize("pad", [70, 150, 300])
+def test_wide_pool_batches(pad):
+    """Pools of > 64 instances (W = 2/4/8 words per row): the row-occupancy path, with the real
+    sites straddling word boundaries, against the oracle on 120 random tiny ICFGs."""
+    gs = [random_tiny(s, wide_pad=pad) for s in range(5000 + pad, 5120 + pad)]
+    app = gd.load(gs)
+    app.build()
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        _assert_same(app, k, g, r, g.name)
+        assert int(digs[k]) == r.app_digest
+    app.build(loop_mode=1)                       # same results through per-round launches
+    assert np.array_equal(app.app_digests(), digs)
+
+
+def test_wide_and_narrow_mixed_batch():
+    """Wide and narrow apps in one handle (the wide instantiation serves both layouts)."""
+    gs = [random_tiny(s, wide_pad=(100 if s % 2 else 0)) for s in range(7000, 7060)]
+    app = gd.load(gs)
+    app.build()
+    for k, g in enumerate(gs):
+        _assert_same(app, k, g, oracle.build_idfg(g), g.name)

@@ -289,3 +289,13 @@ def test_straight_line_closed_forms(case):
     heap = {Lt + g.n_statics + i: f"o{i + 1}.f" for i in range(3)}   # o1..o3 have field f
     got = {(names.get(s, heap.get(s)), o) for (s, o) in r.fact_set(ex)}
     assert got == expected
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_kleene_equals_worklist_wide_pools(seed):
+    """Same brute-force pin with > 64-instance pools (the padding instances never get facts)."""
+    g = random_tiny(seed + 50_000, wide_pad=130)
+    r = oracle.build_idfg(g)
+    S, K = kleene(g)
+    for n in range(g.n_nodes):
+        assert to_sym(S, r.facts(n)) == K[n], (seed, n)
