@@ -110,15 +110,20 @@ def run_shard(app_ids: Sequence[int], make_app: Callable[[int], object], sizes: 
               device: int = 0, stream: int = 0, node_budget: int = 4_000_000,
               prefetch: bool = True) -> List[BatchResult]:
     """Build every app of this rank's shard on `device`, batch by batch.  A loader thread
-    generates (host) the next batch while the GPU builds the current one — the paper's
-    dual-buffered transfer recast for a resident corpus."""
+    generates the next batch and uploads it (gdroid_load_batch on its own stream) while the GPU
+    builds the current one — the paper's dual-buffered transfer."""
+    import torch
     from . import _binding as gd
     plan = batches_under_budget(app_ids, sizes, node_budget)
-    q: "Queue" = Queue(maxsize=2 if prefetch else 1)
+    q: "Queue" = Queue(maxsize=1 if prefetch else 0)
+    streams = [torch.cuda.Stream(device=device), torch.cuda.Stream(device=device)]
 
     def loader():
-        for b in plan:
-            q.put((b, [make_app(i) for i in b]))
+        for j, b in enumerate(plan):
+            apps = [make_app(i) for i in b]
+            t0 = time.perf_counter()
+            h = gd.load(apps, device=device, stream=streams[j % 2].cuda_stream)
+            q.put((b, h, (time.perf_counter() - t0) * 1e3))
         q.put(None)
 
     th = threading.Thread(target=loader, daemon=True)
@@ -128,12 +133,11 @@ def run_shard(app_ids: Sequence[int], make_app: Callable[[int], object], sizes: 
         item = q.get()
         if item is None:
             break
-        ids, apps = item
+        ids, app, load_ms = item
         t0 = time.perf_counter()
-        app = gd.load(apps, device=device, stream=stream)
         st = app.build()
         dig = app.app_digests()
         app.free()
-        out.append(BatchResult(list(ids), dig, st, (time.perf_counter() - t0) * 1e3))
+        out.append(BatchResult(list(ids), dig, st, (time.perf_counter() - t0) * 1e3 + load_ms))
     th.join()
     return out

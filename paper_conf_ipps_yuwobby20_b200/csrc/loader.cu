@@ -12,6 +12,8 @@
 #include <cstdio>
 #include <cstring>
 #include <atomic>
+#include <condition_variable>
+#include <functional>
 #include <map>
 #include <mutex>
 #include <thread>
@@ -106,16 +108,70 @@ struct ModInfo {
   uint32_t gmod;   // global module index
 };
 
-// Run f(k) for k in [0, n) on up to hardware_concurrency threads.
+// Persistent worker pool for the host-side table build (spawning threads per parallel loop
+// costs more than the loops themselves on small apps).
+class Pool {
+ public:
+  static Pool& get() {
+    static Pool p;
+    return p;
+  }
+  uint32_t size() const { return (uint32_t)workers_.size() + 1; }
+  // Run job(k) for k in [0, n); the caller participates.  Not re-entrant.
+  void run(uint32_t n, const std::function<void(uint32_t)>& job) {
+    std::unique_lock<std::mutex> lk(mu_);
+    job_ = &job; n_ = n; next_.store(0); pending_ = (uint32_t)workers_.size(); ++gen_;
+    lk.unlock();
+    cv_.notify_all();
+    for (uint32_t k; (k = next_.fetch_add(1)) < n;) job(k);
+    lk.lock();
+    done_cv_.wait(lk, [&] { return pending_ == 0; });
+    job_ = nullptr;
+  }
+
+ private:
+  Pool() {
+    const uint32_t T = std::max(1u, std::thread::hardware_concurrency());
+    for (uint32_t t = 1; t < T; ++t) workers_.emplace_back([this] { loop(); });
+  }
+  ~Pool() {
+    { std::lock_guard<std::mutex> lk(mu_); stop_ = true; ++gen_; }
+    cv_.notify_all();
+    for (auto& w : workers_) w.join();
+  }
+  void loop() {
+    uint64_t seen = 0;
+    for (;;) {
+      std::unique_lock<std::mutex> lk(mu_);
+      cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
+      if (stop_) return;
+      seen = gen_;
+      const std::function<void(uint32_t)>* job = job_;
+      const uint32_t n = n_;
+      lk.unlock();
+      for (uint32_t k; (k = next_.fetch_add(1)) < n;) (*job)(k);
+      lk.lock();
+      if (--pending_ == 0) done_cv_.notify_one();
+    }
+  }
+  std::vector<std::thread> workers_;
+  std::mutex mu_;
+  std::condition_variable cv_, done_cv_;
+  const std::function<void(uint32_t)>* job_ = nullptr;
+  uint32_t n_ = 0, pending_ = 0;
+  uint64_t gen_ = 0;
+  bool stop_ = false;
+  std::atomic<uint32_t> next_{0};
+};
+std::mutex g_pool_mu;   // one parallel loop at a time (loads are serialised by g_cache.mu too)
+
+// Run f(k) for k in [0, n) on the worker pool.
 template <class F>
 void parallel_for(uint32_t n, F f) {
-  uint32_t T = std::max(1u, std::min<uint32_t>(n, std::thread::hardware_concurrency()));
-  if (T <= 1) { for (uint32_t k = 0; k < n; ++k) f(k); return; }
-  std::vector<std::thread> th;
-  std::atomic<uint32_t> next{0};
-  for (uint32_t t = 0; t < T; ++t)
-    th.emplace_back([&] { for (uint32_t k; (k = next.fetch_add(1)) < n;) f(k); });
-  for (auto& x : th) x.join();
+  if (n <= 1) { if (n) f(0); return; }
+  std::function<void(uint32_t)> job = [&](uint32_t k) { f(k); };
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  Pool::get().run(n, job);
 }
 
 // Run f(lo, hi) over [0, n) split into ranges of about `grain` items, in parallel.
@@ -255,50 +311,75 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   PHASE("modules");
   // ---- nodes: operands -> rows (V1, V2, V4), fact offsets (parallel over node ranges)
   H.app_node_base.push_back(nb);
-  for (uint64_t n = 0; n < N; ++n)
-    if (d->call_arg_ptr[n + 1] < d->call_arg_ptr[n]) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr not monotone at %llu", k, (unsigned long long)n);
-  const uint64_t n_args = d->call_arg_ptr[N] - d->call_arg_ptr[0];
   if (d->call_arg_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr[0] != 0", k);
-  std::vector<uint64_t> foff(N + 1, 0);                      // fact-block offsets
-  parallel_ranges(N, 1 << 15, [&](uint64_t lo, uint64_t hi) {
+  // per range: call_arg_ptr monotone, fact-block sizes, (module, field) keys of heap accesses
+  constexpr uint64_t RG = 1 << 15;
+  const uint64_t n_rg = (N + RG - 1) / RG;
+  std::vector<uint64_t> foff(N + 1, 0), rg_sum(n_rg + 1, 0);
+  std::vector<std::vector<uint64_t>> rg_keys(n_rg);
+  FirstErr fe0;
+  auto fkey = [&](uint64_t n) -> uint64_t {                 // UINT64_MAX: no field-row table
+    const uint8_t kind = d->node_kind[n];
+    if (kind != GK_FLOAD && kind != GK_ALOAD && kind != GK_FSTORE && kind != GK_ASTORE) return UINT64_MAX;
+    const int32_t f = (kind == GK_ALOAD || kind == GK_ASTORE) ? (int32_t)GDROID_F_ARR : d->node_ops[4 * n + 2];
+    if (f < 0 || (uint32_t)f >= d->n_fields) return UINT64_MAX;   // reported by the node pass
+    return ((uint64_t)d->method_module[d->node_method[n]] << 32) | (uint32_t)f;
+  };
+  parallel_ranges(N, RG, [&](uint64_t lo, uint64_t hi) {
+    uint64_t acc = 0;
+    std::vector<uint64_t>& keys = rg_keys[lo / RG];
     for (uint64_t n = lo; n < hi; ++n) {
+      if (d->call_arg_ptr[n + 1] < d->call_arg_ptr[n]) {
+        set_err(GDROID_E_INVALID, "app %u: call_arg_ptr not monotone at %llu", k, (unsigned long long)n);
+        fe0.offer(n, GDROID_E_INVALID);
+        return;
+      }
       const uint64_t m = d->node_method[n];
       const ModRec& md = H.mods[db + d->method_module[m]];
       const uint64_t rows = d->method_n_locals[m] + md.n_glob;
-      const uint64_t words = rows << md.logW;
-      foff[n + 1] = (words + 3) & ~3ull;                        // 32-byte aligned blocks
-      if (md.logW >= 1) foff[n + 1] += (((rows + 63) >> 6) + 3) & ~3ull;   // wide: row-occupancy words
+      uint64_t w = ((rows << md.logW) + 3) & ~3ull;            // 32-byte aligned blocks
+      if (md.logW >= 1) w += (((rows + 63) >> 6) + 3) & ~3ull;  // wide: row-occupancy words
+      acc += w;
+      foff[n + 1] = acc;                                       // range-local inclusive prefix
+      const uint64_t key = fkey(n);
+      if (key != UINT64_MAX) keys.push_back(key);
     }
+    rg_sum[lo / RG + 1] = acc;
+    std::sort(keys.begin(), keys.end());
+    keys.erase(std::unique(keys.begin(), keys.end()), keys.end());
   });
-  for (uint64_t n = 0; n < N; ++n) foff[n + 1] += foff[n];
-  // field-row tables of FLOAD/ALOAD: one per (module, field) pair actually loaded from
-  std::vector<int32_t> frow_of(N, -1);
-  {
-    std::unordered_map<uint64_t, uint32_t> frow_map;
-    for (uint64_t n = 0; n < N; ++n) {
-      const uint8_t kind = d->node_kind[n];
-      if (kind != GK_FLOAD && kind != GK_ALOAD && kind != GK_FSTORE && kind != GK_ASTORE) continue;
-      const int32_t f = (kind == GK_ALOAD || kind == GK_ASTORE) ? (int32_t)GDROID_F_ARR : d->node_ops[4 * n + 2];
-      if (f < 0 || (uint32_t)f >= d->n_fields) continue;       // reported by the node pass
-      const uint64_t dd = d->method_module[d->node_method[n]];
-      const uint64_t key = (dd << 32) | (uint32_t)f;
-      auto it = frow_map.find(key);
-      if (it == frow_map.end()) {
-        const ModRec& md = H.mods[db + dd];
-        const uint32_t off = (uint32_t)H.frow.size();
-        for (uint32_t c = 0; c < md.n_cols; ++c) {
-          const int32_t ty = H.col_type[md.col_off + c];
-          int32_t row = -1;
-          if (c != 0 && ty >= 0)
-            for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
-              if (H.tf[q] == (uint32_t)f) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
-          H.frow.push_back(row);
-        }
-        it = frow_map.emplace(key, off).first;
-      }
-      frow_of[n] = (int32_t)it->second;
+  if (fe0.st != GDROID_OK) return fe0.result();
+  const uint64_t n_args = d->call_arg_ptr[N];
+  for (uint64_t r = 0; r < n_rg; ++r) rg_sum[r + 1] += rg_sum[r];
+  parallel_ranges(N, RG, [&](uint64_t lo, uint64_t hi) {
+    const uint64_t base = rg_sum[lo / RG];
+    for (uint64_t n = lo; n < hi; ++n) foff[n + 1] += base;
+  });
+  // field-row tables of FLOAD/FSTORE/ALOAD/ASTORE: one per (module, field) pair used
+  std::vector<uint64_t> fkeys;
+  for (auto& v : rg_keys) fkeys.insert(fkeys.end(), v.begin(), v.end());
+  std::sort(fkeys.begin(), fkeys.end());
+  fkeys.erase(std::unique(fkeys.begin(), fkeys.end()), fkeys.end());
+  std::vector<uint32_t> fkey_off(fkeys.size());
+  for (size_t i = 0; i < fkeys.size(); ++i) {
+    const uint64_t dd = fkeys[i] >> 32;
+    const uint32_t f = (uint32_t)fkeys[i];
+    const ModRec& md = H.mods[db + dd];
+    fkey_off[i] = (uint32_t)H.frow.size();
+    for (uint32_t c = 0; c < md.n_cols; ++c) {
+      const int32_t ty = H.col_type[md.col_off + c];
+      int32_t row = -1;
+      if (c != 0 && ty >= 0)
+        for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
+          if (H.tf[q] == f) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
+      H.frow.push_back(row);
     }
   }
+  auto frow_of = [&](uint64_t n) -> int32_t {
+    const uint64_t key = fkey(n);
+    if (key == UINT64_MAX) return -1;
+    return (int32_t)fkey_off[std::lower_bound(fkeys.begin(), fkeys.end(), key) - fkeys.begin()];
+  };
   auto local_idx = [&](int64_t gid, uint64_t m) -> int64_t {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
@@ -355,7 +436,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           if (op[2] < 0 || (uint32_t)op[2] >= d->n_fields) return set_err(GDROID_E_INVALID, "app %u: node %llu: field out of range", k, (unsigned long long)n);
           R.r2 = op[2];
         }
-        R.r3 = frow_of[n];                                   // heap row of (o1, f) per column
+        R.r3 = frow_of(n);                                   // heap row of (o1, f) per column
         break;
       case GK_SLOAD:
         if (!need_local(op[0], R.r0, "lhs")) return GDROID_E_POOL;
@@ -768,7 +849,7 @@ void free_app(gdroid_app* a) {
   if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
   if (a->d_scratch) cudaFree(a->d_scratch);
   if (a->D.trace) cudaFree(a->D.trace);
-  if (a->h_stats) cudaFreeHost(a->h_stats);
+  delete a->h_stats;
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
   cudaSetDevice(cur);
@@ -912,8 +993,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     D.bar = (uint32_t*)S; S += s_bar;
     D.node_digest = (uint64_t*)S; S += s_nd;
     D.app_digest = (unsigned long long*)S;
-    e = cudaMallocHost(&a->h_stats, sizeof(DevStats));
-    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "pinned stats: %s", cudaGetErrorString(e)));
+    a->h_stats = new DevStats();
     for (auto& ev : a->ev)
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
