@@ -84,6 +84,7 @@ struct __align__(16) ModRec {
 struct __align__(16) Edge {
   uint32_t dst;
   uint32_t info;       // kind (2 bits) | class of dst << 2 (3 bits) | (chunks of dst - 1) << 5
+                       // | INFO_WIDE (dst block is wide)
   uint64_t off;        // fact-block word offset of dst
   uint32_t B;          // dst block words
   uint16_t L;          // dst method-local rows
@@ -94,6 +95,7 @@ struct __align__(16) Edge {
                        // 0xffffffff = same module (identity)
 };
 static_assert(sizeof(Edge) == 32, "Edge must be 32 bytes");
+constexpr uint32_t INFO_WIDE = 1u << 10;
 constexpr uint32_t NO_XMAP = 0xffffffffu;
 
 struct DevStats {
@@ -124,6 +126,7 @@ struct Dev {
   const int32_t* frow;          // field-row tables: frow[r3 + c] = global row of (col c, f) | -1
   uint64_t* facts;
   uint32_t* stamp;              // [N] last round a node was queued for (0 = never)
+  uint32_t* cont;               // [N] last round a warp continued into the node (0 = never)
   uint32_t* queue;              // [3][n_chunks] rotating class-segmented worklists of
                                 // (node << 5 | chunk) entries
   uint32_t* counts;             // [3][CNT_STRIDE]

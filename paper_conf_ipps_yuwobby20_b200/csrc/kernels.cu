@@ -28,11 +28,16 @@ namespace {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int KW = 4;          // words per lane per chunk of a fact block (loads issued together)
 constexpr int SCAP = 448;      // staged queue entries per class per CTA (overflow goes global)
+#ifndef GD_CONT_DEPTH
+#define GD_CONT_DEPTH 8        // longest depth-first continuation per queued wide item (0 = off)
+#endif
+constexpr uint32_t NO_CONT = 0xffffffffu;
 
 struct Acc {                   // per-warp counters (shared memory), flushed once per kernel
   unsigned long long alg;      // touched-word model bytes
   unsigned long long dense;    // dense-model bytes
   unsigned long long atom;     // RED.OR issued
+  unsigned long long cont;     // items processed by continuation (visits not in the queue)
 };
 
 struct WarpScratch {
@@ -87,12 +92,33 @@ __device__ __forceinline__ void stage_init(CtaStage& st) {
 
 // Append the candidate destinations held by the warp's lanes (every chunk of a pushed node)
 // to the CTA's staged worklist of the next round.
+//
+// Continuation (wide path only; cont != nullptr, warp-uniform *cont == NO_CONT on entry): the
+// first lane whose single-chunk wide destination wants a visit may instead hand it back to the
+// warp, which processes it at once in this round (a depth-first step).  That lane
+// does not queue it: the warp reads IN(dst) after its own ORs, and a later grower of dst sees a
+// stamp below round+1 and queues dst as usual, so no growth is lost.  cont[dst] == round keeps
+// a second warp from continuing into the same node in the same round (it queues it instead).
 __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
                                              uint32_t dst, uint32_t info, bool grew, uint32_t round,
-                                             uint32_t nxt) {
+                                             uint32_t nxt, uint32_t* cont = nullptr) {
   bool push = false;
+  bool want = false;
+  if (active) want = grew || (D.stamp[dst] == 0);           // grew, or first reach (A5)
+  if (cont && *cont == NO_CONT) {
+    const unsigned cand = __ballot_sync(FULL, want && (info & INFO_WIDE) && ((info >> 5) & 31u) == 0);
+    if (cand) {
+      const int l = __ffs(cand) - 1;
+      uint32_t ok = 0;
+      if (lane == l && D.stamp[dst] != round + 1 && atomicExch(&D.cont[dst], round) != round) {
+        atomicMax(&D.stamp[dst], round);                    // reached: no first-reach pushes
+        ok = 1;
+        want = false;
+      }
+      if (__shfl_sync(FULL, ok, l)) *cont = __shfl_sync(FULL, dst, l);
+    }
+  }
   if (active) {
-    const bool want = grew || (D.stamp[dst] == 0);          // grew, or first reach (A5)
     if (want) {
       const uint32_t old = atomicMax(&D.stamp[dst], round + 1);  // test-and-set: de-duplicates (MER)
       push = old < round + 1;
@@ -210,7 +236,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
 
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
-                             uint32_t alg_l0) {
+                             uint32_t alg_l0, uint32_t* cont) {
   const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B, rows = B >> logW;
   const uint64_t* __restrict__ X = D.facts + R.off;
   const uint64_t* __restrict__ OCC = X + occ_offset(B);
@@ -384,7 +410,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
       dense_l0 += 16ull * Bt;
     }
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt);
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt, cont);
   }
   acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
   acc_add(acc.atom, red);
@@ -393,8 +419,8 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
 
 // ---------------------------------------------------------------------------------- one item
 template <bool WIDE>
-__device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
-                             uint32_t nxt, int lane, WarpScratch& ws, Acc& acc) {
+__device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
+                                 uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont) {
   const NodeRec R = D.nodes[n];
   const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
@@ -403,12 +429,14 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
   uint32_t alg_l0 = (first ? (uint32_t)sizeof(NodeRec) : 0u) + (uint32_t)sizeof(Edge) * (e1 - e0) + 4u;
   if (e0 >= e1) {                                           // no successor: nothing to propagate
     if (lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
-    return;
+    return NO_CONT;
   }
   if constexpr (WIDE) {
     if (logW >= 1) {                                        // wide block: row-sparse path
-      process_wide(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0);
-      return;
+      uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
+      process_wide(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
+                   allow_cont ? &cont_v : nullptr);
+      return cont_v;
     }
   }
   const uint64_t* __restrict__ X = D.facts + R.off;
@@ -649,6 +677,7 @@ __device__ void process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci
   acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
   acc_add(acc.atom, red);
   if (lane == 0) acc.dense += dense_l0 + alg_l0;
+  return NO_CONT;
 }
 
 // ---------------------------------------------------------------------------------- rounds
@@ -672,7 +701,8 @@ __device__ __forceinline__ void grid_sync(uint32_t* bar, uint32_t nblocks) {
 }
 
 __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
-  if ((threadIdx.x & 31) == 0 && (acc.alg | acc.atom | acc.dense)) {
+  if ((threadIdx.x & 31) == 0 && (acc.alg | acc.atom | acc.dense | acc.cont)) {
+    atomicAdd(&D.stats->visits, acc.cont);
     atomicAdd(&D.stats->alg_bytes, acc.alg);
     atomicAdd(&D.stats->atomics, acc.atom);
     atomicAdd(&D.stats->dense_bytes, acc.dense);
@@ -732,7 +762,20 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
     if (nitem < total && lane < 4)                                     // and its NodeRec into L1
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
-    process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc);
+    if constexpr (!WIDE || GD_CONT_DEPTH == 0) {
+      process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
+    } else {
+      uint32_t n = entry >> 5, ci = entry & 31u;
+      for (int depth = 0;; ++depth) {
+        const uint32_t c = process_item<WIDE>(D, st, n, ci, round, nxt, lane, ws, acc, depth < GD_CONT_DEPTH);
+        if (c == NO_CONT) break;
+        __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
+        __threadfence_block();
+        n = c;
+        ci = 0;
+        if (lane == 0) acc.cont += 1;
+      }
+    }
     item = nitem;
     entry = nentry;
   }
@@ -747,7 +790,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t gw = blockIdx.x * WARPS + wib, nw = gridDim.x * WARPS;
   Acc& acc = acc_all[wib];
-  if (lane == 0) acc = Acc{0, 0, 0};
+  if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
   for (uint32_t round = 1;; ++round) {
@@ -771,7 +814,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const uint32_t gw = blockIdx.x * WARPS + wib, nw = gridDim.x * WARPS;
   Acc& acc = acc_all[wib];
-  if (lane == 0) acc = Acc{0, 0, 0};
+  if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
   const uint32_t total = run_round<WIDE>(D, st, round, gw, nw, lane, ws_all[wib], acc);

@@ -614,7 +614,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       const uint32_t nch = n_chunks_of((uint32_t)(d->row_ptr[s + 1] - d->row_ptr[s]), RS.cls);
       Edge E2{};
       E2.dst = nb + s;
-      E2.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5);
+      E2.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5) | (RS.logW >= 1 ? INFO_WIDE : 0u);
       E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = RS.logW;
       E2.aux = (ek == GE_CALL) ? (int32_t)d->method_n_params[d->node_method[s]] : (ek == GE_RET ? RS.r0 : -1);
       E2.xoff = xoff;
@@ -980,13 +980,14 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     cudaError_t e = cudaMallocAsync(&a->d_facts, std::max<uint64_t>(Lo.fact_words, 4) * 8, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(Lo.fact_words * 8), cudaGetErrorString(e)));
     D.facts = a->d_facts;
-    size_t s_stamp = align256((size_t)N * 4), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
+    size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t st = s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
     e = cudaMallocAsync(&a->d_state, st, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "device state (%zu B): %s", st, cudaGetErrorString(e)));
     char* S = (char*)a->d_state;
-    D.stamp = (uint32_t*)S; S += s_stamp;
+    D.stamp = (uint32_t*)S;
+    D.cont = D.stamp + N; S += s_stamp;
     D.queue = (uint32_t*)S; S += s_queue;
     D.counts = (uint32_t*)S; S += s_counts;
     D.stats = (DevStats*)S; S += s_stats;
@@ -1021,7 +1022,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   CU(cudaEventRecord(a->ev[0], s));
   // (a2) zero the fact matrices and the worklist state
   CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
-  CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 4, s));
+  CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));
   CU(cudaMemsetAsync(D.stats, 0, sizeof(DevStats), s));
   CU(cudaMemsetAsync(D.bar, 0, 16, s));

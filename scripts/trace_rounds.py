@@ -32,7 +32,8 @@ if ph[4] > 0:
           f"round-end {ph[3]/tot:.1%};  cycles/item setup {ph[0]/ph[4]:.0f} edges {ph[1]/ph[4]:.0f} push {ph[2]/ph[4]:.0f}")
 dt = np.diff(tr[:, 0].astype(np.int64)) / 1e3   # us per round
 items = tr[:-1, 1]
-print(f"{wl}: rounds {len(dt)} fixpoint {st['fixpoint_ns']/1e6:.3f} ms, mean round {dt.mean():.2f} us")
+print(f"{wl}: rounds {len(dt)} fixpoint {st['fixpoint_ns']/1e6:.3f} ms, mean round {dt.mean():.2f} us, "
+      f"queued items {int(items.sum())} node visits {st['node_visits']}")
 for lo, hi in [(0, 1), (1, 32), (32, 256), (256, 1024), (1024, 4096), (4096, 16384), (16384, 1 << 30)]:
     m = (items > lo) & (items <= hi) if lo else (items <= hi)
     if m.any():
