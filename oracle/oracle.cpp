@@ -502,6 +502,37 @@ int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq
   std::vector<std::vector<uint32_t>> preds(N);
   for (uint32_t p = 0; p < N; ++p)
     for (uint64_t e = g->row_ptr[p]; e < g->row_ptr[p + 1]; ++e) preds[g->col[e]].push_back(p);
+  // policy 3 (| window << 8): priority window.  prio(n) = reverse-postorder index of a DFS from
+  // the component entries; a round processes only the listed nodes with prio < min_c + window,
+  // min_c = smallest prio listed in the node's component; the rest are carried over.
+  const int pol = policy & 0xff;
+  const uint32_t window = (uint32_t)policy >> 8;
+  std::vector<uint32_t> prio((pol == 3 || pol == 4) ? N : 0, 0), comp((pol == 3 || pol == 4) ? N : 0, 0);
+  if ((pol == 3 || pol == 4)) {
+    std::vector<uint32_t> post;
+    std::vector<char> seen(N, 0);
+    std::vector<std::pair<uint32_t, uint64_t>> st;
+    for (uint32_t i = 0; i < g->n_entries; ++i) {
+      const uint32_t e = g->entries[i];
+      if (seen[e]) continue;
+      seen[e] = 1;
+      comp[e] = i;
+      st.push_back({e, g->row_ptr[e]});
+      while (!st.empty()) {
+        auto& top = st.back();
+        if (top.second < g->row_ptr[top.first + 1]) {
+          const uint32_t s = g->col[top.second++];
+          if (!seen[s]) { seen[s] = 1; comp[s] = i; st.push_back({s, g->row_ptr[s]}); }
+        } else {
+          post.push_back(top.first);
+          st.pop_back();
+        }
+      }
+    }
+    for (size_t k2 = 0; k2 < post.size(); ++k2) prio[post[k2]] = (uint32_t)(post.size() - 1 - k2);
+    if (pol == 4) for (uint32_t n = 0; n < N; ++n) prio[n] = n;   // policy 4: node id order
+  }
+  std::vector<uint32_t> cmin((pol == 3 || pol == 4) ? g->n_entries : 0, 0xffffffffu);
   std::vector<PairSet> IN(N);
   std::vector<char> visited(N, 0), in_next(N, 0), in_cur(N, 0);
   std::vector<uint32_t> cur, nxt;
@@ -512,23 +543,29 @@ int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq
   *visits = 0;
   while (!cur.empty()) {
     if ((uint64_t)rounds < lens_cap) lens[rounds] = (uint32_t)cur.size();
-    if (policy != 2) for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
+    if (pol != 2 && pol != 5) for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
     ++rounds;
     nxt.clear();
     uint32_t max_depth = 0;
     for (uint32_t n : cur) in_cur[n] = 1;
-    std::vector<uint32_t> cont_round(policy == 2 ? N : 0, 0);
+    std::vector<uint32_t> cont_round((pol == 2 || pol == 5) ? N : 0, 0);
+    if ((pol == 3 || pol == 4)) {
+      for (uint32_t n : cur) cmin[comp[n]] = 0xffffffffu;
+      for (uint32_t n : cur) cmin[comp[n]] = std::min(cmin[comp[n]], prio[n]);
+    }
     for (uint32_t n0 : cur) {
       bool defer = false;
-      if (policy == 1)
+      if (pol == 1)
         for (uint32_t p : preds[n0]) if (p < n0 && in_cur[p]) { defer = true; break; }
+      if ((pol == 3 || pol == 4)) defer = prio[n0] >= cmin[comp[n0]] + window;
       if (defer) {
         if (!in_next[n0]) { nxt.push_back(n0); in_next[n0] = 1; }
         continue;
       }
       // policy 2: continue depth-first into a grown successor of a single-successor node
       uint32_t n = n0;
-      for (int depth = 0; depth < 64; ++depth) {
+      const int max_dep = (pol == 2 || pol == 5) && window ? (int)window : 64;
+      for (int depth = 0; depth < max_dep; ++depth) {
         visited[n] = 1;
         ++*visits;
         PairSet Y = transfer(U, n, IN[n]);
@@ -538,7 +575,8 @@ int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq
           PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
           bool grew = merge_union(IN[s], Z);
           if (!(grew || !visited[s])) continue;
-          if (policy == 2 && g->row_ptr[n + 1] - g->row_ptr[n] == 1 && !in_cur[s] &&
+          if ((pol == 2 || pol == 5) && cont < 0 && depth + 1 < max_dep &&
+              (pol == 5 || g->row_ptr[n + 1] - g->row_ptr[n] == 1) && !in_cur[s] &&
               cont_round[s] != (uint32_t)rounds) {
             cont_round[s] = (uint32_t)rounds;
             cont = s;
@@ -551,7 +589,7 @@ int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq
         n = (uint32_t)cont;
       }
     }
-    if (policy == 2 && (uint64_t)(rounds - 1) < cap) seq[rounds - 1] = max_depth;   // chain depth
+    if ((pol == 2 || pol == 5) && (uint64_t)(rounds - 1) < cap) seq[rounds - 1] = max_depth;   // chain depth
     for (uint32_t n : cur) in_cur[n] = 0;
     for (uint32_t s : nxt) in_next[s] = 0;
     cur.swap(nxt);

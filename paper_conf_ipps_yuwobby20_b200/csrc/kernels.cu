@@ -29,7 +29,13 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int KW = 4;          // words per lane per chunk of a fact block (loads issued together)
 constexpr int SCAP = 448;      // staged queue entries per class per CTA (overflow goes global)
 #ifndef GD_CONT_DEPTH
-#define GD_CONT_DEPTH 8        // longest depth-first continuation per queued wide item (0 = off)
+#define GD_CONT_DEPTH 8        // longest depth-first continuation per queued item (0 = off)
+#endif
+#ifndef GD_CONT_LOAD
+#define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
+#endif
+#ifndef GD_CONT_DENSE
+#define GD_CONT_DENSE 0        // continue into narrow (one word per row) destinations too (light rounds)
 #endif
 constexpr uint32_t NO_CONT = 0xffffffffu;
 
@@ -93,24 +99,24 @@ __device__ __forceinline__ void stage_init(CtaStage& st) {
 // Append the candidate destinations held by the warp's lanes (every chunk of a pushed node)
 // to the CTA's staged worklist of the next round.
 //
-// Continuation (wide path only; cont != nullptr, warp-uniform *cont == NO_CONT on entry): the
-// first lane whose single-chunk wide destination wants a visit may instead hand it back to the
+// Continuation (cont != nullptr, warp-uniform *cont == NO_CONT on entry): the first lane whose
+// single-chunk destination (not queued for this round or the next) wants a visit may instead hand it back to the
 // warp, which processes it at once in this round (a depth-first step).  That lane
 // does not queue it: the warp reads IN(dst) after its own ORs, and a later grower of dst sees a
 // stamp below round+1 and queues dst as usual, so no growth is lost.  cont[dst] == round keeps
 // a second warp from continuing into the same node in the same round (it queues it instead).
 __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
                                              uint32_t dst, uint32_t info, bool grew, uint32_t round,
-                                             uint32_t nxt, uint32_t* cont = nullptr) {
+                                             uint32_t nxt, uint32_t* cont = nullptr, bool cont_dense = false) {
   bool push = false;
   bool want = false;
   if (active) want = grew || (D.stamp[dst] == 0);           // grew, or first reach (A5)
   if (cont && *cont == NO_CONT) {
-    const unsigned cand = __ballot_sync(FULL, want && (info & INFO_WIDE) && ((info >> 5) & 31u) == 0);
+    const unsigned cand = __ballot_sync(FULL, want && (cont_dense || (info & INFO_WIDE)) && ((info >> 5) & 31u) == 0);
     if (cand) {
       const int l = __ffs(cand) - 1;
       uint32_t ok = 0;
-      if (lane == l && D.stamp[dst] != round + 1 && atomicExch(&D.cont[dst], round) != round) {
+      if (lane == l && D.stamp[dst] < round && atomicExch(&D.cont[dst], round) != round) {
         atomicMax(&D.stamp[dst], round);                    // reached: no first-reach pushes
         ok = 1;
         want = false;
@@ -236,7 +242,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
 
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
-                             uint32_t alg_l0, uint32_t* cont) {
+                             uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
   const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B, rows = B >> logW;
   const uint64_t* __restrict__ X = D.facts + R.off;
   const uint64_t* __restrict__ OCC = X + occ_offset(B);
@@ -410,7 +416,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
       dense_l0 += 16ull * Bt;
     }
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt, cont);
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt, cont, cont_dense);
   }
   acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
   acc_add(acc.atom, red);
@@ -420,7 +426,8 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
 // ---------------------------------------------------------------------------------- one item
 template <bool WIDE>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
-                                 uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont) {
+                                 uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
+                                 bool light = false) {
   const NodeRec R = D.nodes[n];
   const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
@@ -435,11 +442,12 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     if (logW >= 1) {                                        // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
       process_wide(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
-                   allow_cont ? &cont_v : nullptr);
+                   allow_cont ? &cont_v : nullptr, GD_CONT_DENSE && light);
       return cont_v;
     }
   }
   const uint64_t* __restrict__ X = D.facts + R.off;
+  uint32_t cont_v = NO_CONT;                                // node to continue into (warp-uniform)
 
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
   //      the rows the transfer function reads
@@ -672,12 +680,13 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     }
     const unsigned gall = __reduce_or_sync(FULL, gmask);
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt);
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt,
+                 (GD_CONT_DENSE && allow_cont && light) ? &cont_v : nullptr, true);
   }
   acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
   acc_add(acc.atom, red);
   if (lane == 0) acc.dense += dense_l0 + alg_l0;
-  return NO_CONT;
+  return cont_v;
 }
 
 // ---------------------------------------------------------------------------------- rounds
@@ -755,6 +764,9 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       if (c == (uint32_t)k && item >= base + cnt[k]) { base += cnt[k]; c = k + 1; }
     return Q[D.seg[c] + (item - base)];
   };
+  // Continuation into narrow destinations (GD_CONT_DENSE) only while the round leaves warps
+  // idle (total items below GD_CONT_LOAD/4 x warps); wide destinations always continue.
+  const bool cont_ok = (uint64_t)total * 4u < (uint64_t)nw * GD_CONT_LOAD;
   uint32_t item = gw;
   uint32_t entry = item < total ? entry_of(item) : 0u;
   while (item < total) {
@@ -762,12 +774,13 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
     if (nitem < total && lane < 4)                                     // and its NodeRec into L1
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
-    if constexpr (!WIDE || GD_CONT_DEPTH == 0) {
+    if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
       process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
     } else {
       uint32_t n = entry >> 5, ci = entry & 31u;
       for (int depth = 0;; ++depth) {
-        const uint32_t c = process_item<WIDE>(D, st, n, ci, round, nxt, lane, ws, acc, depth < GD_CONT_DEPTH);
+        const uint32_t c = process_item<WIDE>(D, st, n, ci, round, nxt, lane, ws, acc,
+                                              depth < GD_CONT_DEPTH, cont_ok);
         if (c == NO_CONT) break;
         __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
         __threadfence_block();
