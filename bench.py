@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--apps-per-rank", type=int, default=8)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--loop-mode", type=int, default=0)
+    ap.add_argument("--variant", default="default", choices=["default", "mat", "mat_grp", "gdroid", "plain"],
+                    help="ablation variant (SURVEY §8(f) 1); plain needs one app per rank")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--e2e-steps", type=int, default=3)
@@ -219,9 +221,11 @@ def run_ours(args):
     nodes = sum(g.n_nodes for g in apps)
     input_bytes = sum(g.nbytes() for g in apps)
 
-    app = gd.load(apps, device=local, stream=stream.cuda_stream)     # inputs resident in HBM
+    plain = args.variant == "plain"
+    assert not plain or len(apps) == 1, "--variant plain takes one app per rank (--apps-per-rank 1)"
+    app = gd.load(apps, device=local, stream=stream.cuda_stream, plain=plain)   # inputs resident in HBM
     for _ in range(args.warmup):
-        app.build(loop_mode=args.loop_mode)
+        app.build(loop_mode=args.loop_mode, variant=args.variant)
     torch.cuda.synchronize()
 
     def barrier():
@@ -235,7 +239,7 @@ def run_ours(args):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         ev0.record(stream)
         for _ in range(args.steps):
-            stats.append(app.build(loop_mode=args.loop_mode))
+            stats.append(app.build(loop_mode=args.loop_mode, variant=args.variant))
         ev1.record(stream)
         torch.cuda.synchronize()
         barrier()
@@ -257,7 +261,7 @@ def run_ours(args):
         def loader():
             for i in range(args.e2e_steps + 1):          # +1: the first load primes the pipeline
                 t = time.perf_counter()
-                a = gd.load(apps, device=local, stream=streams[i % 2].cuda_stream)
+                a = gd.load(apps, device=local, stream=streams[i % 2].cuda_stream, plain=plain)
                 load_ms.append((time.perf_counter() - t) * 1e3)
                 q.put(a)
 
@@ -266,14 +270,14 @@ def run_ours(args):
         torch.cuda.synchronize()
         th.start()
         first = q.get()                                  # not timed: pipeline fill
-        first.build(loop_mode=args.loop_mode)
+        first.build(loop_mode=args.loop_mode, variant=args.variant)
         assert np.array_equal(first.app_digests(), digests)
         first.free()
         t0 = time.perf_counter()
         for i in range(args.e2e_steps):
             tb = time.perf_counter()
             a2 = q.get()
-            a2.build(loop_mode=args.loop_mode)
+            a2.build(loop_mode=args.loop_mode, variant=args.variant)
             tc = time.perf_counter()
             d2 = a2.app_digests()                        # D2H of the result
             a2.free()
@@ -326,7 +330,7 @@ def run_ours(args):
                    "fact_store_bytes_per_rank": stats[-1]["fact_bytes"],
                    "l2": "fact store > L2 (126 MB) per step; re-zeroed each step",
                    "parallelism": f"apps sharded over {world} GPU(s), no data-path collective",
-                   "loop_mode": args.loop_mode},
+                   "loop_mode": args.loop_mode, "variant": args.variant},
         "ms_per_app": ms_step / (total_apps / world),
         "node_visits_per_s": float(recs[:, 3].sum()) * args.steps / (max_ms / 1e3),
         "rounds_per_step": stats[-1]["rounds"],

@@ -97,7 +97,24 @@ typedef struct {
   uint32_t blocks;       /* persistent-kernel CTAs (0 = SMs x occupancy)                     */
   uint32_t loop_mode;    /* 0 = persistent cooperative kernel (default), 1 = host-launched
                             round kernels (one launch per round)                            */
+  uint32_t variant;      /* gdroid_variant: ablation of the paper's optimisations (SURVEY
+                            §8(f) 1).  Every variant computes the same
+                            least fixed point; only the schedule / data structure differ.  */
 } gdroid_build_opts;
+
+/* Variants (Fig. 8-12), recast on B200:
+ *   DEFAULT  the B200 path: MAT + GRP + round-stamp dedupe + continuation into wide successors
+ *   MAT      matrix store (MAT); one worklist segment in arrival order; no
+ *            head/tail merging; no continuation
+ *   MAT_GRP  + class-segmented worklists (GRP)
+ *   GDROID   + MER: each round processes the head list (whole waves of the grid's warps) and
+ *            merges the tail into the next worklist (Fig. 7)
+ *   PLAIN    the set-based plain implementation (Alg. 2): per-node sorted
+ *            pair arrays with regrowth from a device bump allocator, one thread per node,
+ *            per-thread switch over node kinds; needs a handle loaded with
+ *            gdroid_load_icfg_plain (one app)                                               */
+typedef enum { GDROID_V_DEFAULT = 0, GDROID_V_MAT = 1, GDROID_V_MAT_GRP = 2, GDROID_V_GDROID = 3,
+               GDROID_V_PLAIN = 4 } gdroid_variant;
 
 /* Device-counted statistics of the last build (DESIGN.md §5 byte models). */
 typedef struct {
@@ -122,6 +139,13 @@ gdroid_status gdroid_load_icfg(const gdroid_icfg_desc* desc, int device, void* c
  * per app. */
 gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, int device,
                                 void* cuda_stream, gdroid_app** out);
+/* Load ONE app for every variant including GDROID_V_PLAIN: the MAT handle of
+ * gdroid_load_icfg plus device copies of the descriptor arrays and the set-based
+ * state of the plain variant (per-node pair arrays in a bump-allocated heap sized
+ * from the pools' dense bound, per-thread scratch).
+ * Readback after a PLAIN build returns the sets; digests are computed from them. */
+gdroid_status gdroid_load_icfg_plain(const gdroid_icfg_desc* desc, int device, void* cuda_stream,
+                                     gdroid_app** out);
 /* Zero the fact store, seed the entries, run the fixed point, compute digests. */
 gdroid_status gdroid_build_idfg(gdroid_app* app, const gdroid_build_opts* opts,
                                 gdroid_build_stats* stats);

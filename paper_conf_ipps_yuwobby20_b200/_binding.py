@@ -33,7 +33,7 @@ class IcfgDesc(C.Structure):
 
 class BuildOpts(C.Structure):
     _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
-                ("loop_mode", C.c_uint32)]
+                ("loop_mode", C.c_uint32), ("variant", C.c_uint32)]
 
 
 class BuildStats(C.Structure):
@@ -46,6 +46,13 @@ class BuildStats(C.Structure):
         d = {k: int(getattr(self, k)) for k, _ in self._fields_ if k != "hist"}
         d["hist"] = [int(x) for x in self.hist]
         return d
+
+
+VARIANTS = {"default": 0, "mat": 1, "mat_grp": 2, "gdroid": 3, "plain": 4}   # gdroid_variant
+
+
+def variant_id(v) -> int:
+    return VARIANTS[v] if isinstance(v, str) else int(v)
 
 
 class GdroidError(RuntimeError):
@@ -67,6 +74,9 @@ def lib():
         P = C.c_void_p
         L.gdroid_load_batch.argtypes = [P, C.c_uint32, C.c_int, P, C.POINTER(P)]
         L.gdroid_load_icfg.argtypes = [P, C.c_int, P, C.POINTER(P)]
+        if hasattr(L, "gdroid_load_icfg_plain"):          # (absent in older builds used for A/B)
+            L.gdroid_load_icfg_plain.argtypes = [P, C.c_int, P, C.POINTER(P)]
+            L.gdroid_load_icfg_plain.restype = C.c_int
         L.gdroid_build_idfg.argtypes = [P, P, P]
         L.gdroid_sync.argtypes = [P, P]
         L.gdroid_read_facts.argtypes = [P, C.c_uint32, P, C.c_uint64, P]
@@ -121,11 +131,14 @@ def make_desc(g) -> Tuple[IcfgDesc, list]:
 class App:
     """A loaded batch of one or more apps on one device (owns device memory)."""
 
-    def __init__(self, icfgs: Union[object, Sequence[object]], device: int = 0, stream: int = 0):
+    def __init__(self, icfgs: Union[object, Sequence[object]], device: int = 0, stream: int = 0,
+                 plain: bool = False):
         if not isinstance(icfgs, (list, tuple)):
             icfgs = [icfgs]
         L = lib()
         n = len(icfgs)
+        if plain and n != 1:
+            raise ValueError("the PLAIN variant takes one app per handle")
         arr = (IcfgDesc * n)()
         keep = []
         for i, g in enumerate(icfgs):
@@ -133,15 +146,19 @@ class App:
             arr[i] = d
             keep.append(k)
         self._h = C.c_void_p()
-        _check(L.gdroid_load_batch(C.cast(arr, C.c_void_p), n, device, C.c_void_p(stream),
-                                   C.byref(self._h)))
+        if plain:
+            _check(L.gdroid_load_icfg_plain(C.cast(arr, C.c_void_p), device, C.c_void_p(stream),
+                                            C.byref(self._h)))
+        else:
+            _check(L.gdroid_load_batch(C.cast(arr, C.c_void_p), n, device, C.c_void_p(stream),
+                                       C.byref(self._h)))
         self.n_apps = n
         self.n_nodes = [g.n_nodes for g in icfgs]
         self.stats: Optional[dict] = None
 
     def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
-              asynchronous: bool = False) -> Optional[dict]:
-        o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode)
+              asynchronous: bool = False, variant=0) -> Optional[dict]:
+        o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant))
         s = BuildStats()
         _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
         if asynchronous:
@@ -212,5 +229,6 @@ class App:
             pass
 
 
-def load(icfgs, device: int = 0, stream: int = 0) -> App:
-    return App(icfgs, device=device, stream=stream)
+def load(icfgs, device: int = 0, stream: int = 0, plain: bool = False) -> App:
+    """gdroid_load_batch (or gdroid_load_icfg_plain with plain=True: one app, every variant)."""
+    return App(icfgs, device=device, stream=stream, plain=plain)

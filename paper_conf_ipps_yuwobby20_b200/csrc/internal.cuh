@@ -13,7 +13,10 @@ constexpr int NCLS = 5;            // GRP classes + 2 interpr
 enum Cls : uint8_t { C_ONETIME = 0, C_SINGLE = 1, C_DOUBLE = 2, C_CALL = 3, C_EXIT = 4 };
 constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]; slot CNT_NODES = nodes queued
 constexpr int CNT_NODES = 5;
-constexpr int THREADS = 256;       // fixed-point kernel block size
+#ifndef GD_THREADS
+#define GD_THREADS 256
+#endif
+constexpr int THREADS = GD_THREADS; // fixed-point kernel block size
 constexpr int WARPS = THREADS / 32;
 
 // One ICFG node (64 B).  Row indices r* are relative to the node's fact block (method-local
@@ -98,6 +101,11 @@ static_assert(sizeof(Edge) == 32, "Edge must be 32 bytes");
 constexpr uint32_t INFO_WIDE = 1u << 10;
 constexpr uint32_t NO_XMAP = 0xffffffffu;
 
+// Scheduling switches (gdroid_build_opts.variant).  GRP off = one worklist
+// segment in arrival order; MER = head/tail split with the tail merged into the next worklist
+// (Fig. 7); CONT = depth-first continuation into wide successors.
+constexpr uint32_t F_GRP = 1u, F_MER = 2u, F_CONT = 4u;
+
 struct DevStats {
   unsigned long long rounds, visits, alg_bytes, dense_bytes, atomics, hist[3], limit_hit, pad;
   unsigned long long phase[8];  // GD_PHASES builds: cycles in setup / edges / push / round end, items
@@ -141,9 +149,45 @@ struct Dev {
   uint32_t seg[NCLS + 1];       // class segment starts inside one queue
   uint32_t max_rounds;
   uint32_t wide;                // 1 if some module has > 64 instances (row-occupancy path)
+  uint32_t flags;               // F_* scheduling switches of the build (ablation variants)
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
   uint32_t trace_cap;           // rounds recorded (0 = off)
 };
+
+// ---- PLAIN variant (plain.cu): set-based facts, thread per node (Alg. 2)
+struct __align__(16) SetDesc {
+  uint64_t off;      // word offset of the node's sorted pair array in the heap
+  uint32_t size;     // pairs stored
+  uint32_t cap;      // pairs allocated
+};
+static_assert(sizeof(SetDesc) == 16, "SetDesc must be 16 bytes");
+
+struct PlainDev {
+  // input: device copies of one app's gdroid_icfg_desc arrays (+ two host-computed prefixes)
+  const uint64_t* row_ptr; const uint32_t* col; const uint8_t* ekind; const uint8_t* nkind;
+  const uint32_t* nmeth; const int32_t* ops; const uint64_t* arg_ptr; const int32_t* args;
+  const uint64_t* local_base;   // [M+1] prefix of method_n_locals
+  const uint32_t* n_params; const uint32_t* mmod;
+  const uint64_t* inst_ptr; const uint32_t* insts; const uint64_t* stat_ptr; const uint32_t* statics;
+  const int32_t* inst_type; const uint64_t* tf_ptr; const uint32_t* tfields;
+  const uint64_t* heap_base;    // [I+1] prefix of |F(t(o))|
+  const uint32_t* entries;
+  uint64_t L_total, G;
+  uint32_t n_nodes, n_instances, n_entries, max_rounds;
+  // state
+  SetDesc* sets; uint32_t* locks; uint64_t* heap; unsigned long long* heap_top; uint64_t heap_cap;
+  uint64_t* scratch; uint64_t maxset;   // per thread: 3 buffers of maxset pairs
+  uint32_t* stamp; uint32_t* queue; uint32_t* counts; uint32_t* bar; uint32_t* err;
+  DevStats* stats;
+  uint64_t* node_digest; unsigned long long* app_digest;
+};
+
+int plain_max_blocks(int device);
+cudaError_t launch_plain(const PlainDev& P, uint32_t blocks, cudaStream_t s);
+cudaError_t launch_plain_digest(const PlainDev& P, cudaStream_t s);
+cudaError_t launch_plain_sizes(const PlainDev& P, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
+cudaError_t launch_plain_gather(const PlainDev& P, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
+                                cudaStream_t s);
 
 // kernels.cu launch wrappers (return cudaError_t of the launch)
 cudaError_t launch_seed(const Dev& D, cudaStream_t s);

@@ -27,12 +27,15 @@ namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int KW = 4;          // words per lane per chunk of a fact block (loads issued together)
-constexpr int SCAP = 448;      // staged queue entries per class per CTA (overflow goes global)
+constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class per CTA (overflow goes global)
 #ifndef GD_CONT_DEPTH
 #define GD_CONT_DEPTH 8        // longest depth-first continuation per queued item (0 = off)
 #endif
 #ifndef GD_CONT_LOAD
 #define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
+#endif
+#ifndef GD_PF
+#define GD_PF 0                // prefetch the next item's fact lines / edges into L2 (two-ahead NodeRec)
 #endif
 #ifndef GD_CONT_DENSE
 #define GD_CONT_DENSE 0        // continue into narrow (one word per row) destinations too (light rounds)
@@ -111,7 +114,7 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
   bool push = false;
   bool want = false;
   if (active) want = grew || (D.stamp[dst] == 0);           // grew, or first reach (A5)
-  if (cont && *cont == NO_CONT) {
+  if (cont && *cont == NO_CONT && (D.flags & F_CONT)) {
     const unsigned cand = __ballot_sync(FULL, want && (cont_dense || (info & INFO_WIDE)) && ((info >> 5) & 31u) == 0);
     if (cand) {
       const int l = __ffs(cand) - 1;
@@ -130,7 +133,7 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
       push = old < round + 1;
     }
   }
-  const int cls = push ? (int)((info >> 2) & 7u) : -1;
+  const int cls = push ? ((D.flags & F_GRP) ? (int)((info >> 2) & 7u) : 0) : -1;   // GRP segment
   const uint32_t nch = ((info >> 5) & 31u) + 1;
   unsigned pm = __ballot_sync(FULL, push);
   if (pm && lane == 0) atomicAdd(&st.nodes, (uint32_t)__popc(pm));
@@ -767,13 +770,42 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   // Continuation into narrow destinations (GD_CONT_DENSE) only while the round leaves warps
   // idle (total items below GD_CONT_LOAD/4 x warps); wide destinations always continue.
   const bool cont_ok = (uint64_t)total * 4u < (uint64_t)nw * GD_CONT_LOAD;
+  // MER (Fig. 7): process the head list — whole waves of nw items — and
+  // merge the tail into the next worklist (the round stamp removes repetitions).
+  const uint32_t head = ((D.flags & F_MER) && total > nw) ? (total / nw) * nw : total;
   uint32_t item = gw;
   uint32_t entry = item < total ? entry_of(item) : 0u;
+  if (GD_PF && item + nw < total && lane < 4)                           // first look-ahead NodeRec
+    asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (entry_of(item + nw) >> 5)) + 16 * lane));
   while (item < total) {
+    if (item >= head) {                                                // tail: defer to round+1
+      const uint32_t n = entry >> 5;
+      uint32_t info = 0;
+      if (lane == 0) {
+        const NodeRec R = D.nodes[n];
+        info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls) - 1) << 5);
+      }
+      flush_pushes(D, st, lane, lane == 0, n, info, true, round, nxt);
+      item += nw;
+      entry = item < total ? entry_of(item) : 0u;
+      continue;
+    }
     const uint32_t nitem = item + nw;
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
-    if (nitem < total && lane < 4)                                     // and its NodeRec into L1
+    if (GD_PF) {
+      // two ahead: NodeRec of item + 2nw into L1; the next item's fact lines and edge records
+      // into L2 (its NodeRec was prefetched one item ago)
+      const uint32_t n2 = nitem + nw;
+      if (n2 < total && lane < 4)
+        asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (entry_of(n2) >> 5)) + 16 * lane));
+      if (nitem < total && lane < 9) {
+        const NodeRec* RN = D.nodes + (nentry >> 5);
+        const char* a = lane < 8 ? (const char*)(D.facts + RN->off) + 128 * lane : (const char*)(D.edges + RN->e0);
+        if (lane == 8 || (uint32_t)(16 * lane) < RN->B) asm volatile("prefetch.global.L2 [%0];" :: "l"(a));
+      }
+    } else if (nitem < total && lane < 4) {                            // NodeRec into L1
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
+    }
     if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
       process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
     } else {

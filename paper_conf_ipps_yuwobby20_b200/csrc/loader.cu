@@ -826,6 +826,7 @@ struct gdroid_app {
   void* d_tables = nullptr;
   uint64_t* d_facts = nullptr;
   void* d_state = nullptr;            // stamp, queue, counts, stats, bar, digests
+  uint32_t cls_count[NCLS] = {};      // work items per GRP class (queue segment sizes)
   DevStats* h_stats = nullptr;        // pinned
   uint64_t* d_scratch = nullptr;
   size_t scratch_bytes = 0;
@@ -835,6 +836,11 @@ struct gdroid_app {
   uint64_t launches = 0;
   bool built = false, pending = false;
   int max_blocks = 0;
+  // PLAIN variant (plain.cu): set-based state, present when loaded with gdroid_load_icfg_plain
+  PlainDev P{};
+  void* d_plain = nullptr;            // uploaded inputs + sets, locks, stamps, queues, scratch, heap
+  int plain_blocks = 0;
+  bool last_plain = false;            // the last build ran the PLAIN variant (readback from sets)
 };
 
 namespace {
@@ -848,6 +854,7 @@ void free_app(gdroid_app* a) {
   if (a->d_facts) cudaFreeAsync(a->d_facts, a->stream);
   if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
   if (a->d_scratch) cudaFree(a->d_scratch);
+  if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
   delete a->h_stats;
   for (auto& e : a->ev)
@@ -894,9 +901,155 @@ gdroid_status finish_stats(gdroid_app* a, gdroid_build_stats* out) {
   return GDROID_OK;
 }
 
+// ---------------------------------------------------------------------------------- PLAIN
+// Upload one app's descriptor arrays for the set-based plain variant (plain.cu) and size its
+// state: per-thread scratch of 3 x maxset pairs (maxset bounds every set a thread holds:
+// IN(n), f(IN(n)), an edge image, FSTORE's generated pairs) and the bump-allocated heap.
+gdroid_status load_plain(gdroid_app* a, const gdroid_icfg_desc* d) {
+  const uint64_t N = d->n_nodes, E = d->n_edges, M = d->n_methods, Dm = d->n_modules, I = d->n_instances,
+                 T = d->n_types;
+  const uint64_t n_args = d->call_arg_ptr[N], n_insts = d->module_inst_ptr[Dm], n_stat = d->module_static_ptr[Dm],
+                 n_tf = d->type_field_ptr[T];
+  std::vector<uint64_t> local_base(M + 1, 0), heap_base(I + 1, 0);
+  for (uint64_t m = 0; m < M; ++m) local_base[m + 1] = local_base[m] + d->method_n_locals[m];
+  for (uint64_t o = 0; o < I; ++o) {
+    const int32_t t = d->inst_type[o];
+    heap_base[o + 1] = heap_base[o] + (t < 0 ? 0 : d->type_field_ptr[t + 1] - d->type_field_ptr[t]);
+  }
+  // |P_m| x |Q_m| (+ |Q_m|^2 for FSTORE's generated pairs), max over methods
+  std::vector<uint64_t> mod_heap(Dm, 0);
+  for (uint64_t q = 0; q < Dm; ++q)
+    for (uint64_t k = d->module_inst_ptr[q]; k < d->module_inst_ptr[q + 1]; ++k)
+      mod_heap[q] += heap_base[d->module_insts[k] + 1] - heap_base[d->module_insts[k]];
+  uint64_t maxset = 8, dense_bound = 0;
+  for (uint64_t m = 0; m < M; ++m) {
+    const uint32_t q = d->method_module[m];
+    const uint64_t Q = d->module_inst_ptr[q + 1] - d->module_inst_ptr[q];
+    const uint64_t Pm = d->method_n_locals[m] + (d->module_static_ptr[q + 1] - d->module_static_ptr[q]) + mod_heap[q];
+    maxset = std::max(maxset, (Pm + Q) * Q);
+  }
+  for (uint64_t n = 0; n < N; ++n) {
+    const uint32_t q = d->method_module[d->node_method[n]];
+    const uint64_t Q = d->module_inst_ptr[q + 1] - d->module_inst_ptr[q];
+    dense_bound += (d->method_n_locals[d->node_method[n]] + (d->module_static_ptr[q + 1] - d->module_static_ptr[q]) +
+                    mod_heap[q]) * Q;
+  }
+  // layout of one device allocation
+  size_t off = 0;
+  auto take = [&](size_t bytes) { size_t o = off; off = align256(off + bytes); return o; };
+  const size_t o_rp = take((N + 1) * 8), o_col = take(E * 4), o_ek = take(E), o_nk = take(N), o_nm = take(N * 4),
+               o_ops = take(N * 16), o_ap = take((N + 1) * 8), o_args = take(n_args * 4), o_lb = take((M + 1) * 8),
+               o_np = take(M * 4), o_mm = take(M * 4), o_ip = take((Dm + 1) * 8), o_is = take(n_insts * 4),
+               o_sp = take((Dm + 1) * 8), o_ss = take(n_stat * 4), o_it = take(I * 4), o_tp = take((T + 1) * 8),
+               o_tf = take(n_tf * 4), o_hb = take((I + 1) * 8), o_en = take((size_t)d->n_entries * 4);
+  const size_t in_bytes = off;
+  const size_t o_sets = take(N * sizeof(SetDesc)), o_locks = take(N * 4), o_stamp = take(N * 4),
+               o_queue = take(3 * N * 4), o_counts = take(256), o_bar = take(256), o_err = take(256),
+               o_top = take(256);
+  size_t free_b = 0, total_b = 0;
+  CU(cudaMemGetInfo(&free_b, &total_b));
+  int blocks = plain_max_blocks(a->device);
+  const size_t per_thread = 3 * maxset * 8;
+  const size_t scratch_budget = std::min<size_t>(free_b / 4, (size_t)32 << 30);
+  while (blocks > 1 && (size_t)blocks * 128 * per_thread > scratch_budget) blocks /= 2;
+  const size_t o_scr = take((size_t)blocks * 128 * per_thread);
+  const size_t heap_bytes = std::max<size_t>((size_t)64 << 20,
+      std::min<size_t>((free_b > off ? (free_b - off) / 2 : 0), (size_t)dense_bound * 8 * 4 + ((size_t)16 << 20)));
+  const size_t o_heap = take(heap_bytes);
+  void* mem = nullptr;
+  cudaError_t e = cudaMalloc(&mem, off);
+  if (e != cudaSuccess) return set_err(GDROID_E_OOM, "plain state (%zu B): %s", off, cudaGetErrorString(e));
+  a->d_plain = mem;
+  char* B = (char*)mem;
+  std::vector<char> h(in_bytes, 0);
+  auto put = [&](size_t o, const void* src, size_t bytes) { if (bytes) std::memcpy(h.data() + o, src, bytes); };
+  put(o_rp, d->row_ptr, (N + 1) * 8); put(o_col, d->col, E * 4); put(o_ek, d->edge_kind, E);
+  put(o_nk, d->node_kind, N); put(o_nm, d->node_method, N * 4); put(o_ops, d->node_ops, N * 16);
+  put(o_ap, d->call_arg_ptr, (N + 1) * 8); put(o_args, d->call_args, n_args * 4);
+  put(o_lb, local_base.data(), (M + 1) * 8); put(o_np, d->method_n_params, M * 4); put(o_mm, d->method_module, M * 4);
+  put(o_ip, d->module_inst_ptr, (Dm + 1) * 8); put(o_is, d->module_insts, n_insts * 4);
+  put(o_sp, d->module_static_ptr, (Dm + 1) * 8); put(o_ss, d->module_statics, n_stat * 4);
+  put(o_it, d->inst_type, I * 4); put(o_tp, d->type_field_ptr, (T + 1) * 8); put(o_tf, d->type_fields, n_tf * 4);
+  put(o_hb, heap_base.data(), (I + 1) * 8); put(o_en, d->entries, (size_t)d->n_entries * 4);
+  CU(cudaMemcpy(mem, h.data(), in_bytes, cudaMemcpyHostToDevice));
+  PlainDev& P = a->P;
+  P.row_ptr = (const uint64_t*)(B + o_rp); P.col = (const uint32_t*)(B + o_col); P.ekind = (const uint8_t*)(B + o_ek);
+  P.nkind = (const uint8_t*)(B + o_nk); P.nmeth = (const uint32_t*)(B + o_nm); P.ops = (const int32_t*)(B + o_ops);
+  P.arg_ptr = (const uint64_t*)(B + o_ap); P.args = (const int32_t*)(B + o_args);
+  P.local_base = (const uint64_t*)(B + o_lb); P.n_params = (const uint32_t*)(B + o_np); P.mmod = (const uint32_t*)(B + o_mm);
+  P.inst_ptr = (const uint64_t*)(B + o_ip); P.insts = (const uint32_t*)(B + o_is);
+  P.stat_ptr = (const uint64_t*)(B + o_sp); P.statics = (const uint32_t*)(B + o_ss);
+  P.inst_type = (const int32_t*)(B + o_it); P.tf_ptr = (const uint64_t*)(B + o_tp); P.tfields = (const uint32_t*)(B + o_tf);
+  P.heap_base = (const uint64_t*)(B + o_hb); P.entries = (const uint32_t*)(B + o_en);
+  P.L_total = local_base[M]; P.G = d->n_statics;
+  P.n_nodes = (uint32_t)N; P.n_instances = (uint32_t)I; P.n_entries = d->n_entries;
+  P.sets = (SetDesc*)(B + o_sets); P.locks = (uint32_t*)(B + o_locks); P.stamp = (uint32_t*)(B + o_stamp);
+  P.queue = (uint32_t*)(B + o_queue); P.counts = (uint32_t*)(B + o_counts); P.bar = (uint32_t*)(B + o_bar);
+  P.err = (uint32_t*)(B + o_err); P.heap_top = (unsigned long long*)(B + o_top);
+  P.scratch = (uint64_t*)(B + o_scr); P.maxset = maxset;
+  P.heap = (uint64_t*)(B + o_heap); P.heap_cap = heap_bytes / 8;
+  P.stats = a->D.stats; P.node_digest = a->D.node_digest; P.app_digest = a->D.app_digest;
+  a->plain_blocks = blocks;
+  return GDROID_OK;
+}
+
+// One PLAIN build: zero the sets / worklist state, seed, fixed point, digests (same events
+// and stats as the MAT path; alg_bytes = live set bytes, dense_bytes = allocated set bytes
+// (Fig. 10 footprint), atomics = array (re)allocations).
+gdroid_status build_plain(gdroid_app* a, const gdroid_build_opts& o, gdroid_build_stats* stats) {
+  if (!a->d_plain) return set_err(GDROID_E_STATE, "PLAIN variant needs a handle loaded with gdroid_load_icfg_plain");
+  PlainDev& P = a->P;
+  P.max_rounds = o.max_rounds;
+  cudaStream_t s = a->stream;
+  const uint32_t N = P.n_nodes;
+  a->launches = 0;
+  CU(cudaEventRecord(a->ev[0], s));
+  CU(cudaMemsetAsync(P.sets, 0, (size_t)N * sizeof(SetDesc), s));
+  CU(cudaMemsetAsync(P.locks, 0, (size_t)N * 4, s));
+  CU(cudaMemsetAsync(P.stamp, 0, (size_t)N * 4, s));
+  CU(cudaMemsetAsync(P.counts, 0, 256, s));
+  CU(cudaMemsetAsync(P.bar, 0, 256, s));
+  CU(cudaMemsetAsync(P.err, 0, 256, s));
+  CU(cudaMemsetAsync(P.heap_top, 0, 256, s));
+  CU(cudaMemsetAsync(a->D.stats, 0, sizeof(DevStats), s));
+  CU(cudaMemsetAsync(a->D.app_digest, 0, 8, s));
+  CU(cudaEventRecord(a->ev[1], s));
+  CU(launch_plain(P, (uint32_t)a->plain_blocks, s));
+  a->launches += 2;
+  CU(cudaEventRecord(a->ev[2], s));
+  CU(launch_plain_digest(P, s));
+  a->launches++;
+  CU(cudaEventRecord(a->ev[3], s));
+  CU(cudaMemcpyAsync(a->h_stats, a->D.stats, sizeof(DevStats), cudaMemcpyDeviceToHost, s));
+  uint32_t err = 0;
+  CU(cudaMemcpyAsync(&err, P.err, 4, cudaMemcpyDeviceToHost, s));
+  CU(cudaStreamSynchronize(s));
+  a->pending = true;
+  a->last_plain = true;
+  gdroid_status st = finish_stats(a, stats);
+  a->last.fact_bytes = a->h_stats->dense_bytes;
+  if (stats) stats->fact_bytes = a->last.fact_bytes;
+  if (err) {
+    a->built = false;
+    return set_err(GDROID_E_OOM, "PLAIN set heap exhausted (%llu words)", (unsigned long long)P.heap_cap);
+  }
+  return st;
+}
+
 }  // namespace
 
 extern "C" {
+
+gdroid_status gdroid_load_icfg_plain(const gdroid_icfg_desc* desc, int device, void* cuda_stream, gdroid_app** out) {
+  gdroid_status st = gdroid_load_batch(desc, 1, device, cuda_stream, out);   // validates; MAT variants too
+  if (st != GDROID_OK) return st;
+  DeviceGuard guard(device);
+  CU(cudaStreamSynchronize((cudaStream_t)cuda_stream));
+  st = load_plain(*out, desc);
+  if (st != GDROID_OK) { free_app(*out); *out = nullptr; }
+  return st;
+}
+
 
 uint32_t gdroid_abi_version(void) { return GDROID_ABI_VERSION; }
 const char* gdroid_last_error(void) { return g_err.c_str(); }
@@ -970,7 +1123,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.n_chunks = NC;
   D.n_entries = (uint32_t)Lo.n_entries;
   uint32_t acc = 0;
-  for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += Lo.cls_count[c]; }
+  for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += Lo.cls_count[c]; a->cls_count[c] = Lo.cls_count[c]; }
   D.seg[NCLS] = acc;
   D.n_words = Lo.fact_words;
   D.wide = Lo.wide ? 1u : 0u;
@@ -1015,6 +1168,18 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   DeviceGuard guard(a->device);
   Dev& D = a->D;
   D.max_rounds = o.max_rounds;
+  if (o.variant == GDROID_V_PLAIN) return build_plain(a, o, stats);
+  if (o.variant > GDROID_V_GDROID) return set_err(GDROID_E_INVALID, "unknown variant %u", o.variant);
+  a->last_plain = false;
+  static const uint32_t vflags[4] = {F_GRP | F_CONT, 0u, F_GRP, F_GRP | F_MER};
+  D.flags = vflags[o.variant];
+  {                                                   // GRP off: one segment holds every item
+    uint32_t acc = 0;
+    for (int c = 0; c <= NCLS; ++c) {
+      D.seg[c] = (D.flags & F_GRP) ? acc : (c == 0 ? 0u : D.n_chunks);
+      if (c < NCLS) acc += a->cls_count[c];
+    }
+  }
   cudaStream_t s = a->stream;
   const uint32_t N = D.n_nodes;
   uint32_t blocks = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks) : (uint32_t)a->max_blocks;
@@ -1025,7 +1190,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));
   CU(cudaMemsetAsync(D.stats, 0, sizeof(DevStats), s));
-  CU(cudaMemsetAsync(D.bar, 0, 16, s));
+  CU(cudaMemsetAsync(D.bar, 0, 256, s));                 // barrier + round descriptor words
   CU(cudaMemsetAsync(D.app_digest, 0, (size_t)a->n_apps * 8, s));
   CU(launch_seed(D, s));
   a->launches++;
@@ -1086,7 +1251,8 @@ gdroid_status gdroid_read_all_facts(const gdroid_app* ca, uint32_t k, uint64_t* 
   const uint32_t n0 = a->app_base[k], n1 = a->app_base[k + 1], n = n1 - n0;
   gdroid_status st = ensure_scratch(a, (size_t)(n + 1) * 8);
   if (st) return st;
-  CU(launch_popc(a->D, n0, n1, a->d_scratch, a->stream));
+  CU(a->last_plain ? launch_plain_sizes(a->P, n0, n1, a->d_scratch, a->stream)
+                   : launch_popc(a->D, n0, n1, a->d_scratch, a->stream));
   std::vector<uint64_t> cnt(n);
   CU(cudaMemcpyAsync(cnt.data(), a->d_scratch, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));
@@ -1100,7 +1266,8 @@ gdroid_status gdroid_read_all_facts(const gdroid_app* ca, uint32_t k, uint64_t* 
   uint64_t* d_ptr = a->d_scratch;
   uint64_t* d_pairs = a->d_scratch + (n + 1);
   CU(cudaMemcpyAsync(d_ptr, ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, a->stream));
-  CU(launch_expand(a->D, n0, n1, d_ptr, d_pairs, a->stream));
+  CU(a->last_plain ? launch_plain_gather(a->P, n0, n1, d_ptr, d_pairs, a->stream)
+                   : launch_expand(a->D, n0, n1, d_ptr, d_pairs, a->stream));
   CU(cudaMemcpyAsync(pairs, d_pairs, (size_t)total * 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));
   return GDROID_OK;
@@ -1119,7 +1286,8 @@ gdroid_status gdroid_read_facts_in(const gdroid_app* ca, uint32_t k, uint32_t no
   gdroid_status st = ensure_scratch(a, 16);
   if (st) return st;
   const uint32_t g = n0 + node;
-  CU(launch_popc(a->D, g, g + 1, a->d_scratch, a->stream));
+  CU(a->last_plain ? launch_plain_sizes(a->P, g, g + 1, a->d_scratch, a->stream)
+                   : launch_popc(a->D, g, g + 1, a->d_scratch, a->stream));
   uint64_t cnt = 0;
   CU(cudaMemcpyAsync(&cnt, a->d_scratch, 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));
@@ -1130,7 +1298,8 @@ gdroid_status gdroid_read_facts_in(const gdroid_app* ca, uint32_t k, uint32_t no
   if (st) return st;
   uint64_t zero = 0;
   CU(cudaMemcpyAsync(a->d_scratch, &zero, 8, cudaMemcpyHostToDevice, a->stream));
-  CU(launch_expand(a->D, g, g + 1, a->d_scratch, a->d_scratch + 2, a->stream));
+  CU(a->last_plain ? launch_plain_gather(a->P, g, g + 1, a->d_scratch, a->d_scratch + 2, a->stream)
+                   : launch_expand(a->D, g, g + 1, a->d_scratch, a->d_scratch + 2, a->stream));
   CU(cudaMemcpyAsync(pairs, a->d_scratch + 2, (size_t)cnt * 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));
   return GDROID_OK;

@@ -50,15 +50,17 @@ def _check(app, k, g, ref):
         assert [str(int(p)) for p in got] == pairs, f"{ref['name']} node {n}"
 
 
-@pytest.mark.parametrize("name", ["small", "median", "worst"])
-def test_preset_full_size(name):
+@pytest.mark.parametrize("name,variant", [("small", "default"), ("median", "default"), ("worst", "default"),
+                                          ("small", "mat"), ("median", "mat_grp"), ("median", "gdroid"),
+                                          ("small", "plain")])
+def test_preset_full_size(name, variant):
     fx = _fixture()
     if name not in fx:
         pytest.skip(f"{name} not in fixture")
     ref = fx[name]
     g = G.preset(name)
-    app = gd.load(g)
-    app.build()
+    app = gd.load(g, plain=(variant == "plain"))
+    app.build(variant=variant)
     per, dig = app.node_digests()
     assert str(dig) == ref["app_digest"]
     assert str(_node_hash(per)) == ref["node_digest_hash"]

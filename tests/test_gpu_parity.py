@@ -151,3 +151,59 @@ def test_wide_and_narrow_mixed_batch():
     app.build()
     for k, g in enumerate(gs):
         _assert_same(app, k, g, oracle.build_idfg(g), g.name)
+
+
+@pytest.mark.parametrize("variant", ["mat", "mat_grp", "gdroid"])
+@pytest.mark.parametrize("blocks", [0, 3])
+def test_ablation_variants(variant, blocks):
+    """The ablation schedules (MAT / MAT+GRP / MAT+GRP+MER) reach the same
+    least fixed point: narrow and wide random tiny ICFGs in one handle; with 3 CTAs (24 warps)
+    most rounds exceed one wave, so MER's head/tail split defers tails."""
+    gs = [random_tiny(s, wide_pad=(90 if s % 3 == 0 else 0)) for s in range(9000, 9120)]
+    app = gd.load(gs)
+    st = app.build(variant=variant, blocks=blocks)
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        _assert_same(app, k, g, r, f"{variant}/{g.name}")
+        assert int(digs[k]) == r.app_digest
+    assert st["rounds"] > 0
+
+
+@pytest.mark.parametrize("which", ["tiny", "tiny_m2", "tiny2", "fig2"])
+def test_plain_variant_golden(which):
+    """PLAIN (set-based, thread per node; Alg. 2) on the hand-written programs."""
+    g = fig2()[0] if which == "fig2" else (tiny2()[0] if which == "tiny2" else tiny(m2_entry=(which == "tiny_m2"))[0])
+    app = gd.load(g, plain=True)
+    st = app.build(variant="plain")
+    r = oracle.build_idfg(g)
+    _assert_same(app, 0, g, r, f"plain/{which}")
+    per, dig = app.node_digests()
+    assert dig == r.app_digest and np.array_equal(per, r.node_digest)
+    assert st["node_visits"] > 0 and st["fact_bytes"] > 0
+    app.build()                                   # the same handle runs the MAT path too
+    _assert_same(app, 0, g, r, f"mat-after-plain/{which}")
+
+
+@pytest.mark.parametrize("chunk", range(2))
+def test_plain_variant_random(chunk):
+    """PLAIN on 80 random tiny ICFGs (narrow and wide pools; every node/edge kind, recursion,
+    projection) — one handle each, as the plain variant takes one app."""
+    for s in range(11000 + chunk * 40, 11040 + chunk * 40):
+        g = random_tiny(s, wide_pad=(80 if s % 4 == 0 else 0))
+        app = gd.load(g, plain=True)
+        app.build(variant="plain")
+        r = oracle.build_idfg(g)
+        _assert_same(app, 0, g, r, f"plain/{g.name}")
+        assert app.node_digests()[1] == r.app_digest
+        app.free()
+
+
+def test_plain_variant_errors():
+    g = tiny()[0]
+    app = gd.load(g)                              # not loaded for PLAIN
+    with pytest.raises(gd.GdroidError) as e:
+        app.build(variant="plain")
+    assert e.value.code == -5
+    with pytest.raises(ValueError):
+        gd.load([g, g], plain=True)
