@@ -51,6 +51,15 @@ static_assert(sizeof(NodeRec) == 64, "NodeRec must be 64 bytes");
 // flagged rows (a fact written after the reader's bitmap load is re-processed next round,
 // because its writer also queued the node).
 __host__ __device__ __forceinline__ uint32_t occ_offset(uint32_t B) { return (B + 3u) & ~3u; }
+// Narrow blocks (one word per row) carry a 64-bit group-occupancy mask in D.smask: bit i covers
+// words [i << s, (i + 1) << s) with s = mshift_of(B) (s = 2: one 32-byte sector for B <= 256).
+// Readers load only flagged groups; every writer that turns a zero word non-zero sets the bit
+// (same visibility argument as the wide row-occupancy bitmaps).
+__host__ __device__ __forceinline__ uint32_t mshift_of(uint32_t B) {
+  uint32_t l = 0;
+  while ((1u << l) < B) ++l;          // ceil(log2 B)
+  return l > 8 ? l - 6 : 2u;
+}
 __host__ __device__ __forceinline__ uint32_t occ_words(uint32_t rows) { return (rows + 63u) >> 6; }
 
 // Work items.  A node's out-edges are split into chunks of ebs(deg) edges (at most 32 chunks
@@ -133,6 +142,7 @@ struct Dev {
   const uint32_t* node_method;  // [N] (digest / readback only)
   const int32_t* frow;          // field-row tables: frow[r3 + c] = global row of (col c, f) | -1
   uint64_t* facts;
+  uint64_t* smask;              // [N] narrow blocks: bit i = word group i (mshift_of(B)) may be non-zero
   uint32_t* stamp;              // [N] last round a node was queued for (0 = never)
   uint32_t* cont;               // [N] last round a warp continued into the node (0 = never)
   uint32_t* queue;              // [3][n_chunks] rotating class-segmented worklists of

@@ -34,6 +34,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_CONT_LOAD
 #define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
 #endif
+#ifndef GD_SMASK
+#define GD_SMASK 1             // narrow blocks: read only word groups flagged in D.smask
+#endif
 #ifndef GD_PF
 #define GD_PF 0                // prefetch the next item's fact lines / edges into L2 (two-ahead NodeRec)
 #endif
@@ -192,7 +195,7 @@ __device__ __forceinline__ void stage_publish(const Dev& D, CtaStage& st, uint32
 // Words of row `kill` are dropped (C2R).  Returns the number of non-zero words in the low
 // 16 bits and the number of REDs issued in the high bits.
 __device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uint64_t (&y)[KW], uint32_t c0,
-                                             int lane, int kill, uint32_t logW) {
+                                             int lane, int kill, uint32_t logW, uint64_t& mbits, uint32_t msh) {
   uint64_t cur[KW];
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
@@ -209,9 +212,18 @@ __device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uin
     if (z & ~cur[k]) {
       red_or(Z + w, z);
       ++red;
+      if (GD_SMASK && cur[k] == 0) mbits |= 1ull << (w >> msh);   // zero word becomes non-zero
     }
   }
   return nz | (red << 16);
+}
+
+// Publish the warp's new group-occupancy bits of narrow block `dst` (one RED per warp).
+__device__ __forceinline__ void set_mask(const Dev& D, uint32_t dst, uint64_t mbits, int lane) {
+  if (!GD_SMASK) return;
+  if (!__any_sync(FULL, mbits != 0)) return;
+  const uint64_t m = warp_or64(mbits);
+  if (lane == 0) red_or(D.smask + dst, m);
 }
 
 // ---------------------------------------------------------------------------------- wide blocks
@@ -222,7 +234,8 @@ __device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uin
 constexpr int WROWS = 1024;    // row-list capacity per warp (rows of one block)
 
 __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_t logWt, uint32_t rt,
-                                               const uint64_t (&v)[MAXW], uint32_t& nz, uint32_t& red, bool& g) {
+                                               const uint64_t (&v)[MAXW], uint32_t& nz, uint32_t& red, bool& g,
+                                               uint64_t* mask_t) {
   const uint32_t Wt = 1u << logWt;
   uint64_t* row = Z + ((uint64_t)rt << logWt);
   uint64_t cur[MAXW];
@@ -233,14 +246,16 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
     any |= (j < (int)Wt && v[j] != 0);
   }
   if (!any) return;
+  bool wrote = false;
 #pragma unroll
   for (int j = 0; j < MAXW; ++j) {
     if (j >= (int)Wt || !v[j]) continue;
     ++nz;
     if (cur[j]) was_zero = false;
-    if (v[j] & ~cur[j]) { red_or(row + j, v[j]); ++red; g = true; }
+    if (v[j] & ~cur[j]) { red_or(row + j, v[j]); ++red; g = true; wrote = true; }
   }
   if (logWt >= 1 && was_zero) red_or(Z + occ_offset(Bt) + (rt >> 6), 1ull << (rt & 63));   // occupancy
+  if (GD_SMASK && logWt == 0 && was_zero && wrote) red_or(mask_t, 1ull << (rt >> mshift_of(Bt)));
 }
 
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
@@ -390,7 +405,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
         for (int q = 0; q < 3; ++q) {
           if (rt[q] < 0) continue;
           if (!proj) {
-            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], y, nz, red, g);
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], y, nz, red, g, D.smask + ep->dst);
           } else {
             uint64_t out[MAXW];
 #pragma unroll
@@ -409,7 +424,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
                   if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
               }
             }
-            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], out, nz, red, g);
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], out, nz, red, g, D.smask + ep->dst);
           }
         }
       }
@@ -431,6 +446,7 @@ template <bool WIDE>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
+  const uint64_t mk = GD_SMASK ? __ldcg(D.smask + n) : ~0ull;   // (issued with the NodeRec load)
   const NodeRec R = D.nodes[n];
   const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
@@ -454,11 +470,13 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
 
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
   //      the rows the transfer function reads
+  const uint32_t msh = mshift_of(B);
+  auto has = [&](uint32_t w) -> bool { return !GD_SMASK || ((mk >> (w >> msh)) & 1ull); };
   uint64_t y[KW];
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
     const uint32_t w = lane + 32 * k;
-    y[k] = (w < B) ? X[w] : 0ull;
+    y[k] = (w < B && has(w)) ? X[w] : 0ull;
   }
   const uint32_t kind = R.kind;
   int mode = 0, t = -1;                                     // 0 identity, 1 replace, 2 or-in, 3 FSTORE
@@ -527,7 +545,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
 #pragma unroll
           for (int k = 0; k < KW; ++k) {
             const uint32_t w = c0 + lane + 32 * k;
-            y[k] = (w < B) ? X[w] : 0ull;
+            y[k] = (w < B && has(w)) ? X[w] : 0ull;
           }
         }
 #pragma unroll
@@ -555,7 +573,9 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
           const uint32_t info = ep->info;
           const uint64_t off = ep->off;
           const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;     // C2R drops lhs(c)
-          const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW);
+          uint64_t mb = 0;
+          const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW, mb, msh);
+          set_mask(D, ep->dst, mb, lane);
           nz += r & 0xffffu;
           red += r >> 16;
           if (r >> 16) gmask |= 1u << i;
@@ -598,9 +618,12 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
             const uint32_t w = c0 + lane + 32 * k, r = w >> logW, j = w & (W - 1);
             int src = -1;
             if (w < Bt) src = (r < Lt) ? local_src(r) : (int)(L + (r - Lt));
-            z[k] = src >= 0 ? X[((uint64_t)src << logW) + j] : 0ull;   // CALL/EXIT: identity
+            const uint32_t ws = ((uint32_t)src << logW) + j;
+            z[k] = (src >= 0 && has(ws)) ? X[ws] : 0ull;                  // CALL/EXIT: identity
           }
-          const uint32_t r = or_chunk(Z, z, c0, lane, -1, logW);
+          uint64_t mb = 0;
+          const uint32_t r = or_chunk(Z, z, c0, lane, -1, logW, mb, mshift_of(Bt));
+          set_mask(D, ep->dst, mb, lane);
           nz += r & 0xffffu;
           red += r >> 16;
           if (r >> 16) g = true;
@@ -628,9 +651,10 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
           }
           __syncwarp();
           if (!WIDE || (W == 1 && logWt == 0)) {            // one word per row on both sides
-            uint64_t v[KW], cur[KW];
+            uint64_t v[KW], cur[KW], mb = 0;
+            const uint32_t mst = mshift_of(Bt);
 #pragma unroll
-            for (int k = 0; k < KW; ++k) v[k] = src[k] >= 0 ? X[src[k]] : 0ull;
+            for (int k = 0; k < KW; ++k) v[k] = (src[k] >= 0 && has((uint32_t)src[k])) ? X[src[k]] : 0ull;
 #pragma unroll
             for (int k = 0; k < KW; ++k) {
               uint64_t o = 0, b = v[k];
@@ -650,8 +674,10 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                 red_or(Z + r0 + lane + 32 * k, v[k]);
                 ++red;
                 g = true;
+                if (GD_SMASK && cur[k] == 0) mb |= 1ull << ((r0 + lane + 32 * k) >> mst);
               }
             }
+            set_mask(D, ep->dst, mb, lane);
           } else if constexpr (WIDE) {
 #pragma unroll
             for (int k = 0; k < KW; ++k) {
@@ -672,7 +698,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                     if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
                 }
               }
-              emit_row_words(Z, Bt, logWt, r, out, nz, red, g);   // sets occupancy if wide
+              emit_row_words(Z, Bt, logWt, r, out, nz, red, g, D.smask + ep->dst);   // occupancy
             }
           }
         }

@@ -1133,12 +1133,14 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     cudaError_t e = cudaMallocAsync(&a->d_facts, std::max<uint64_t>(Lo.fact_words, 4) * 8, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(Lo.fact_words * 8), cudaGetErrorString(e)));
     D.facts = a->d_facts;
+    size_t s_mask = align256((size_t)N * 8);
     size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
-    size_t st = s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
+    size_t st = s_mask + s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
     e = cudaMallocAsync(&a->d_state, st, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "device state (%zu B): %s", st, cudaGetErrorString(e)));
     char* S = (char*)a->d_state;
+    D.smask = (uint64_t*)S; S += s_mask;
     D.stamp = (uint32_t*)S;
     D.cont = D.stamp + N; S += s_stamp;
     D.queue = (uint32_t*)S; S += s_queue;
@@ -1188,6 +1190,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   // (a2) zero the fact matrices and the worklist state
   CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
   CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
+  CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));
   CU(cudaMemsetAsync(D.stats, 0, sizeof(DevStats), s));
   CU(cudaMemsetAsync(D.bar, 0, 256, s));                 // barrier + round descriptor words

@@ -13,7 +13,7 @@ for rep in 1 2; do
   cp /tmp/lib_base.so paper_conf_ipps_yuwobby20_b200/libgdroid.so; touch paper_conf_ipps_yuwobby20_b200/libgdroid.so
   for w in ${WORKLOADS:-small median corpus}; do echo "== base $w"; timeout 600 python bench.py --workload $w --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 0 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['ms_per_step'], d['rounds_per_step'])"; done
   for v in "$@"; do
-    GDROID_NVCC_FLAGS="$v" python -c "import paper_conf_ipps_yuwobby20_b200._build as b; b.build()"
+    GDROID_NVCC_FLAGS="-DGD_AB $v" python -c "import paper_conf_ipps_yuwobby20_b200._build as b; b.build()"
     for w in ${WORKLOADS:-small median corpus}; do echo "== [$v] $w"; timeout 600 python bench.py --workload $w --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 0 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(d['ms_per_step'], d['rounds_per_step'])"; done
   done
 done

@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 for v in "$@"; do
   flags="${v%%|*}"; envs=""; [[ "$v" == *"|"* ]] && envs="${v#*|}"
-  GDROID_NVCC_FLAGS="$flags" python -c "import paper_conf_ipps_yuwobby20_b200._build as b; b.build()" || exit 1
+  GDROID_NVCC_FLAGS="-DGD_AB $flags" python -c "import paper_conf_ipps_yuwobby20_b200._build as b; b.build()" || exit 1
   for w in ${WORKLOADS:-median corpus worst}; do
     echo "== [$flags] [$envs] $w"
     env $envs timeout 600 python bench.py --workload $w --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 1 2>&1 | tail -1 | \
