@@ -100,6 +100,10 @@ typedef struct {
   uint32_t variant;      /* gdroid_variant: ablation of the paper's optimisations (SURVEY
                             §8(f) 1).  Every variant computes the same
                             least fixed point; only the schedule / data structure differ.  */
+  uint32_t no_byte_model;/* 1: skip the on-device byte-model counters (alg_bytes, dense_bytes
+                            and atomics of the stats are then 0); rounds and visits are
+                            always counted.  A separate kernel instantiation without the
+                            counting code (fewer instructions per visit).                  */
 } gdroid_build_opts;
 
 /* Variants (Fig. 8-12), recast on B200:

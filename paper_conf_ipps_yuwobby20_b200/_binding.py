@@ -33,7 +33,7 @@ class IcfgDesc(C.Structure):
 
 class BuildOpts(C.Structure):
     _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
-                ("loop_mode", C.c_uint32), ("variant", C.c_uint32)]
+                ("loop_mode", C.c_uint32), ("variant", C.c_uint32), ("no_byte_model", C.c_uint32)]
 
 
 class BuildStats(C.Structure):
@@ -157,8 +157,9 @@ class App:
         self.stats: Optional[dict] = None
 
     def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
-              asynchronous: bool = False, variant=0) -> Optional[dict]:
-        o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant))
+              asynchronous: bool = False, variant=0, byte_model: bool = True) -> Optional[dict]:
+        o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant),
+                      0 if byte_model else 1)
         s = BuildStats()
         _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
         if asynchronous:

@@ -160,6 +160,7 @@ struct Dev {
   uint32_t max_rounds;
   uint32_t wide;                // 1 if some module has > 64 instances (row-occupancy path)
   uint32_t flags;               // F_* scheduling switches of the build (ablation variants)
+  uint32_t count;               // 1: evaluate the byte models (alg/dense bytes, atomics) on the device
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
   uint32_t trace_cap;           // rounds recorded (0 = off)
 };

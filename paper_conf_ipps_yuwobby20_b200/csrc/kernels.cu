@@ -35,7 +35,7 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
 #endif
 #ifndef GD_SMASK
-#define GD_SMASK 1             // narrow blocks: read only word groups flagged in D.smask
+#define GD_SMASK 0             // narrow blocks: read only word groups flagged in D.smask (measured slower)
 #endif
 #ifndef GD_PF
 #define GD_PF 0                // prefetch the next item's fact lines / edges into L2 (two-ahead NodeRec)
@@ -139,6 +139,21 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
   const int cls = push ? ((D.flags & F_GRP) ? (int)((info >> 2) & 7u) : 0) : -1;   // GRP segment
   const uint32_t nch = ((info >> 5) & 31u) + 1;
   unsigned pm = __ballot_sync(FULL, push);
+  if (__popc(pm) == 1) {                                     // common case: one destination
+    if (push) {
+      atomicAdd(&st.nodes, 1u);
+      const uint32_t base = atomicAdd(&st.cnt[cls], nch);
+      for (uint32_t q = 0; q < nch; ++q) {
+        const uint32_t idx = base + q, entry = (dst << 5) | q;
+        if (idx < (uint32_t)SCAP) st.buf[cls][idx] = entry;
+        else {
+          const uint32_t g = atomicAdd(&D.counts[nxt * CNT_STRIDE + cls], 1u);
+          D.queue[(size_t)nxt * D.n_chunks + D.seg[cls] + g] = entry;
+        }
+      }
+    }
+    return;
+  }
   if (pm && lane == 0) atomicAdd(&st.nodes, (uint32_t)__popc(pm));
   while (pm) {                                               // warp-aggregated append per class
     const int leader = __ffs(pm) - 1;
@@ -258,6 +273,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
   if (GD_SMASK && logWt == 0 && was_zero && wrote) red_or(mask_t, 1ull << (rt >> mshift_of(Bt)));
 }
 
+template <bool CNT>
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
                              uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
@@ -436,13 +452,15 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
     flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt, cont, cont_dense);
   }
-  acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
-  acc_add(acc.atom, red);
-  if (lane == 0) acc.dense += dense_l0 + alg_l0;
+  if constexpr (CNT) {                     // byte models (dead code, removed, when !CNT)
+    acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
+    acc_add(acc.atom, red);
+    if (lane == 0) acc.dense += dense_l0 + alg_l0;
+  }
 }
 
 // ---------------------------------------------------------------------------------- one item
-template <bool WIDE>
+template <bool WIDE, bool CNT>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
@@ -451,20 +469,23 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
   const bool first = ci == 0;
-  const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B;
+  const uint32_t L = R.L, B = R.B;
   uint32_t alg_l0 = (first ? (uint32_t)sizeof(NodeRec) : 0u) + (uint32_t)sizeof(Edge) * (e1 - e0) + 4u;
   if (e0 >= e1) {                                           // no successor: nothing to propagate
-    if (lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
+    if (CNT && lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
     return NO_CONT;
   }
   if constexpr (WIDE) {
-    if (logW >= 1) {                                        // wide block: row-sparse path
+    if (R.logW >= 1) {                                      // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
-      process_wide(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
+      process_wide<CNT>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
                    allow_cont ? &cont_v : nullptr, GD_CONT_DENSE && light);
       return cont_v;
     }
   }
+  // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
+  // instantiations: word index = row index.
+  constexpr uint32_t logW = 0u, W = 1u;
   const uint64_t* __restrict__ X = D.facts + R.off;
   uint32_t cont_v = NO_CONT;                                // node to continue into (warp-uniform)
 
@@ -480,54 +501,48 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   }
   const uint32_t kind = R.kind;
   int mode = 0, t = -1;                                     // 0 identity, 1 replace, 2 or-in, 3 FSTORE
-  uint32_t f = 0, hwords = 0;
-  uint64_t genv = 0;                                        // lane j < W: word j of the generated row
+  uint32_t f = 0, hwords = 0, fmask = 0;                   // fmask: FSTORE target words (bit k: word lane + 32k)
+  uint64_t genv = 0;                                        // word of the generated row
   if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
     mode = 1; t = R.r0;
-    if (kind != GK_PRIM && (R.r3 >> 6) == lane) genv = 1ull << (R.r3 & 63);
+    if (kind != GK_PRIM) genv = 1ull << (R.r3 & 63);       // narrow: column r3 < 64
   } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
     mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
-    if (lane < (int)W) genv = X[((uint64_t)R.r1 << logW) + lane];
+    genv = X[R.r1];                                         // row rhs (all lanes: broadcast)
   } else if (kind == GK_FLOAD || kind == GK_ALOAD) {       // v = w.f: OR of rows (o1,f), o1 ∈ w
     mode = 1; t = R.r0;
-    if (lane < (int)W) ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
-    int hr[(64 * MAXW) / 32];                               // heap rows of this lane's columns
+    const uint64_t wrow = X[R.r1];                          // row w (all lanes: broadcast)
+    int hr[2];                                              // heap rows of this lane's columns
 #pragma unroll
-    for (int q = 0; q < (64 * MAXW) / 32; ++q) {
+    for (int q = 0; q < 2; ++q) {
       const uint32_t c = lane + 32 * q;
       hr[q] = (c < R.n_cols) ? D.frow[R.r3 + c] : -1;
     }
-    __syncwarp();
-    uint64_t a[MAXW];
+    uint64_t a = 0;
 #pragma unroll
-    for (int j = 0; j < MAXW; ++j) a[j] = 0;
-#pragma unroll
-    for (int q = 0; q < (64 * MAXW) / 32; ++q) {
+    for (int q = 0; q < 2; ++q) {
       const uint32_t c = lane + 32 * q;
-      if (hr[q] < 0 || !((ws.rw[c >> 6] >> (c & 63)) & 1ull)) continue;   // NULL has no row
-      const uint64_t* H = X + ((uint64_t)(L + hr[q]) << logW);
-#pragma unroll
-      for (int j = 0; j < MAXW; ++j)
-        if (j < (int)W) a[j] |= H[j];
-      hwords += W;
+      if (hr[q] < 0 || !((wrow >> c) & 1ull)) continue;   // NULL has no row
+      a |= X[L + hr[q]];
+      hwords += 1;
     }
-#pragma unroll
-    for (int j = 0; j < MAXW; ++j)
-      if (j < (int)W) {
-        const uint64_t v = warp_or64(a[j]);
-        if (lane == j) genv = v;
-      }
+    genv = warp_or64(a);
   } else if (kind == GK_FSTORE || kind == GK_ASTORE) {     // v.f = w (weak)
     mode = 3; f = (uint32_t)R.r2;
-    if (lane < (int)W) {
-      ws.rv[lane] = X[((uint64_t)R.r0 << logW) + lane];
-      ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
+    const uint64_t vrow = X[R.r0];                          // row v (all lanes: broadcast)
+    genv = X[R.r1];                                         // row w, OR-ed into rows (o1, f)
+    uint64_t b = vrow;
+    while (b) {                                             // o1 in row v (NULL has no row)
+      const int c = __ffsll((long long)b) - 1;
+      b &= b - 1;
+      const int hr = D.frow[R.r3 + c];
+      if (hr < 0) continue;
+      const uint32_t w = L + (uint32_t)hr;
+      if (w < 32u * KW && (w & 31u) == (uint32_t)lane) fmask |= 1u << (w >> 5);
     }
-    __syncwarp();
   }
-  // every word w of this lane has column-word index j = w & (W-1) = lane & (W-1)
-  const uint64_t gsel = __shfl_sync(FULL, genv, lane & (W - 1));
-  const uint64_t rwsel = (mode == 3) ? ws.rw[lane & (W - 1)] : 0ull;
+  const uint64_t gsel = genv, rwsel = genv;                // identical on every lane
+  (void)f;
 
   uint32_t nzx = 0, nz = 0, red = 0;                        // per-lane counters of this item
   unsigned long long dense_l0 = first ? 8ull * B : 0ull;
@@ -552,16 +567,14 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
         for (int k = 0; k < KW; ++k) {
           const uint32_t w = c0 + lane + 32 * k;
           if (first && eb == e0) nzx += (y[k] != 0);
-          if (w < B && mode != 0) {
-            const int r = (int)(w >> logW);
-            if (mode == 1) { if (r == t) y[k] = gsel; }
-            else if (mode == 2) { if (r == t) y[k] |= gsel; }
-            else if ((uint32_t)r >= L + R.n_stat) {           // FSTORE: heap rows (o1, f)
-              const uint32_t g = (uint32_t)r - L;
-              if (D.grow_field[R.grow_off + g] == (int)f) {
-                const int c = D.grow_col[R.grow_off + g];     // o1 (never NULL)
-                if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) y[k] |= rwsel;
-              }
+          if (mode == 1) { if ((int)w == t) y[k] = gsel; }
+          else if (mode == 2) { if ((int)w == t) y[k] |= gsel; }
+          else if (mode == 3 && c0 == 0) { if ((fmask >> k) & 1u) y[k] |= rwsel; }   // FSTORE rows (o1, f)
+          else if (mode == 3) {                               // blocks of > 128 rows
+            const uint32_t g = w - L;
+            if (w < B && w >= L + R.n_stat && D.grow_field[R.grow_off + g] == (int)f) {
+              const int c = D.grow_col[R.grow_off + g];       // o1 (never NULL)
+              if ((X[R.r0] >> c) & 1ull) y[k] |= rwsel;
             }
           }
         }
@@ -712,9 +725,11 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt,
                  (GD_CONT_DENSE && allow_cont && light) ? &cont_v : nullptr, true);
   }
-  acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
-  acc_add(acc.atom, red);
-  if (lane == 0) acc.dense += dense_l0 + alg_l0;
+  if constexpr (CNT) {
+    acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
+    acc_add(acc.atom, red);
+    if (lane == 0) acc.dense += dense_l0 + alg_l0;
+  }
   return cont_v;
 }
 
@@ -749,7 +764,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 
 // Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
-template <bool WIDE>
+template <bool WIDE, bool CNT>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
@@ -786,11 +801,10 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     }
   }
   const uint32_t* Q = D.queue + (size_t)cur * D.n_chunks;
+  const uint32_t b1 = cnt[0], b2 = b1 + cnt[1], b3 = b2 + cnt[2], b4 = b3 + cnt[3];   // class boundaries
   auto entry_of = [&](uint32_t item) -> uint32_t {          // item -> class segment -> entry
-    uint32_t c = 0, base = 0;
-#pragma unroll
-    for (int k = 0; k < NCLS - 1; ++k)
-      if (c == (uint32_t)k && item >= base + cnt[k]) { base += cnt[k]; c = k + 1; }
+    const uint32_t c = (item >= b1) + (item >= b2) + (item >= b3) + (item >= b4);
+    const uint32_t base = c == 0 ? 0u : (c == 1 ? b1 : (c == 2 ? b2 : (c == 3 ? b3 : b4)));
     return Q[D.seg[c] + (item - base)];
   };
   // Continuation into narrow destinations (GD_CONT_DENSE) only while the round leaves warps
@@ -833,11 +847,11 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
     }
     if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
-      process_item<WIDE>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
+      process_item<WIDE, CNT>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
     } else {
       uint32_t n = entry >> 5, ci = entry & 31u;
       for (int depth = 0;; ++depth) {
-        const uint32_t c = process_item<WIDE>(D, st, n, ci, round, nxt, lane, ws, acc,
+        const uint32_t c = process_item<WIDE, CNT>(D, st, n, ci, round, nxt, lane, ws, acc,
                                               depth < GD_CONT_DEPTH, cont_ok);
         if (c == NO_CONT) break;
         __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
@@ -853,7 +867,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   return total;
 }
 
-template <bool WIDE>
+template <bool WIDE, bool CNT>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -865,7 +879,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   stage_init(st);
   __syncthreads();
   for (uint32_t round = 1;; ++round) {
-    const uint32_t total = run_round<WIDE>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+    const uint32_t total = run_round<WIDE, CNT>(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == 0) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
@@ -877,7 +891,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   flush_acc(D, acc);
 }
 
-template <bool WIDE>
+template <bool WIDE, bool CNT>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t round) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -888,7 +902,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
-  const uint32_t total = run_round<WIDE>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+  const uint32_t total = run_round<WIDE, CNT>(D, st, round, gw, nw, lane, ws_all[wib], acc);
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);
@@ -1003,8 +1017,15 @@ cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
 int fixpoint_max_blocks(int device, bool wide) {
   int sms = 0, occ = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  if (wide) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<true>, THREADS, 0);
-  else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<false>, THREADS, 0);
+  int occ2 = 0;
+  if (wide) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<true, true>, THREADS, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_fixpoint<true, false>, THREADS, 0);
+  } else {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<false, true>, THREADS, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_fixpoint<false, false>, THREADS, 0);
+  }
+  occ = occ2 < occ ? occ2 : occ;          // one grid size serves both instantiations
   return sms * (occ > 0 ? occ : 1);
 }
 
@@ -1013,13 +1034,19 @@ int fixpoint_max_blocks(int device, bool wide) {
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s) {
   Dev d = D;
   void* args[] = {&d};
-  const void* f = D.wide ? (const void*)k_fixpoint<true> : (const void*)k_fixpoint<false>;
+  const void* f = D.wide ? (D.count ? (const void*)k_fixpoint<true, true> : (const void*)k_fixpoint<true, false>)
+                         : (D.count ? (const void*)k_fixpoint<false, true> : (const void*)k_fixpoint<false, false>);
   return cudaLaunchCooperativeKernel(f, dim3(blocks), dim3(THREADS), args, 0, s);
 }
 
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s) {
-  if (D.wide) k_round<true><<<blocks, THREADS, 0, s>>>(D, round);
-  else k_round<false><<<blocks, THREADS, 0, s>>>(D, round);
+  if (D.wide) {
+    if (D.count) k_round<true, true><<<blocks, THREADS, 0, s>>>(D, round);
+    else k_round<true, false><<<blocks, THREADS, 0, s>>>(D, round);
+  } else {
+    if (D.count) k_round<false, true><<<blocks, THREADS, 0, s>>>(D, round);
+    else k_round<false, false><<<blocks, THREADS, 0, s>>>(D, round);
+  }
   return cudaGetLastError();
 }
 

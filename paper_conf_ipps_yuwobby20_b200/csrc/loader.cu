@@ -1175,6 +1175,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   a->last_plain = false;
   static const uint32_t vflags[4] = {F_GRP | F_CONT, 0u, F_GRP, F_GRP | F_MER};
   D.flags = vflags[o.variant];
+  D.count = o.no_byte_model ? 0u : 1u;
   {                                                   // GRP off: one segment holds every item
     uint32_t acc = 0;
     for (int c = 0; c <= NCLS; ++c) {

@@ -207,3 +207,20 @@ def test_plain_variant_errors():
     assert e.value.code == -5
     with pytest.raises(ValueError):
         gd.load([g, g], plain=True)
+
+
+@pytest.mark.parametrize("wide", [0, 90])
+def test_uncounted_instantiation_same_results(wide):
+    """no_byte_model=1 runs the kernel instantiation without the byte-model counters: same
+    fixed point (oracle), visits still counted, byte models reported as 0."""
+    gs = [random_tiny(s, wide_pad=wide) for s in range(12000, 12080)]
+    app = gd.load(gs)
+    st = app.build(byte_model=False)
+    assert st["alg_bytes"] == 0 and st["dense_bytes"] == 0 and st["node_visits"] > 0
+    for k, g in enumerate(gs):
+        _assert_same(app, k, g, oracle.build_idfg(g), g.name)
+    st1 = app.build(byte_model=True)
+    assert st1["alg_bytes"] > 0 and st1["dense_bytes"] >= st1["alg_bytes"]
+    app.build(byte_model=False, loop_mode=1)
+    for k in (0, 41, 79):
+        _assert_same(app, k, gs[k], oracle.build_idfg(gs[k]))
