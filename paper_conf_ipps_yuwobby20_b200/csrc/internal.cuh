@@ -158,7 +158,8 @@ struct Dev {
   uint32_t n_entries;
   uint32_t seg[NCLS + 1];       // class segment starts inside one queue
   uint32_t max_rounds;
-  uint32_t wide;                // 1 if some module has > 64 instances (row-occupancy path)
+  uint32_t wide;                // max log2(words per row) over the batch's modules: 0 = all narrow,
+                                // >= 1: some module has > 64 instances (row-occupancy path)
   uint32_t flags;               // F_* scheduling switches of the build (ablation variants)
   uint32_t count;               // 1: evaluate the byte models (alg/dense bytes, atomics) on the device
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
@@ -208,6 +209,6 @@ cudaError_t launch_digest(const Dev& D, cudaStream_t s);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,
                           uint64_t* pairs, cudaStream_t s);
-int fixpoint_max_blocks(int device, bool wide);
+int fixpoint_max_blocks(int device, uint32_t wide);
 
 }  // namespace gd

@@ -248,22 +248,23 @@ __device__ __forceinline__ void set_mask(const Dev& D, uint32_t dst, uint64_t mb
 // occupancy bit.  Same results as the dense path, bytes proportional to non-zero rows.
 constexpr int WROWS = 1024;    // row-list capacity per warp (rows of one block)
 
+template <int MW>
 __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_t logWt, uint32_t rt,
-                                               const uint64_t (&v)[MAXW], uint32_t& nz, uint32_t& red, bool& g,
+                                               const uint64_t (&v)[MW], uint32_t& nz, uint32_t& red, bool& g,
                                                uint64_t* mask_t) {
   const uint32_t Wt = 1u << logWt;
   uint64_t* row = Z + ((uint64_t)rt << logWt);
-  uint64_t cur[MAXW];
+  uint64_t cur[MW];
   bool any = false, was_zero = true;
 #pragma unroll
-  for (int j = 0; j < MAXW; ++j) {
+  for (int j = 0; j < MW; ++j) {
     cur[j] = (j < (int)Wt && v[j]) ? row[j] : ~0ull;
     any |= (j < (int)Wt && v[j] != 0);
   }
   if (!any) return;
   bool wrote = false;
 #pragma unroll
-  for (int j = 0; j < MAXW; ++j) {
+  for (int j = 0; j < MW; ++j) {
     if (j >= (int)Wt || !v[j]) continue;
     ++nz;
     if (cur[j]) was_zero = false;
@@ -273,7 +274,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
   if (GD_SMASK && logWt == 0 && was_zero && wrote) red_or(mask_t, 1ull << (rt >> mshift_of(Bt)));
 }
 
-template <bool CNT>
+template <bool CNT, int MW>
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
                              uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
@@ -296,21 +297,21 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
     mode = 1; t = R.r0;
     if (lane < (int)W) ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
     __syncwarp();
-    uint64_t a[MAXW];
+    uint64_t a[MW];
 #pragma unroll
-    for (int j = 0; j < MAXW; ++j) a[j] = 0;
+    for (int j = 0; j < MW; ++j) a[j] = 0;
     for (uint32_t c = lane; c < R.n_cols; c += 32) {
       if (!((ws.rw[c >> 6] >> (c & 63)) & 1ull)) continue;
       const int hr = D.frow[R.r3 + c];
       if (hr < 0) continue;                                  // NULL / field not declared
       const uint64_t* H = X + ((uint64_t)(L + hr) << logW);
 #pragma unroll
-      for (int j = 0; j < MAXW; ++j)
+      for (int j = 0; j < MW; ++j)
         if (j < (int)W) a[j] |= H[j];
       hwords += W;
     }
 #pragma unroll
-    for (int j = 0; j < MAXW; ++j)
+    for (int j = 0; j < MW; ++j)
       if (j < (int)W) {
         const uint64_t v = warp_or64(a[j]);
         if (lane == j) ws.gen[j] = v;
@@ -377,26 +378,26 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
       for (uint32_t p = lane; p < cnt; p += 32) {
         const uint32_t r = ws.rowlist[p];
         // Y row r = f(X) row r
-        uint64_t y[MAXW];
+        uint64_t y[MW];
 #pragma unroll
-        for (int j = 0; j < MAXW; ++j) y[j] = (j < (int)W) ? X[((uint64_t)r << logW) + j] : 0ull;
+        for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? X[((uint64_t)r << logW) + j] : 0ull;
         if (first && eb == e0 && i == 0) {
 #pragma unroll
-          for (int j = 0; j < MAXW; ++j) nzx += (j < (int)W && y[j] != 0);
+          for (int j = 0; j < MW; ++j) nzx += (j < (int)W && y[j] != 0);
         }
         if (mode == 1 && (int)r == t) {
 #pragma unroll
-          for (int j = 0; j < MAXW; ++j) y[j] = (j < (int)W) ? ws.gen[j] : 0ull;
+          for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? ws.gen[j] : 0ull;
         } else if (mode == 2 && (int)r == t) {
 #pragma unroll
-          for (int j = 0; j < MAXW; ++j) if (j < (int)W) y[j] |= ws.gen[j];
+          for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.gen[j];
         } else if (mode == 3 && r >= L + R.n_stat) {
           const uint32_t gg = r - L;
           if (D.grow_field[R.grow_off + gg] == R.r2) {
             const int c = D.grow_col[R.grow_off + gg];
             if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) {
 #pragma unroll
-              for (int j = 0; j < MAXW; ++j) if (j < (int)W) y[j] |= ws.rw[j];
+              for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.rw[j];
             }
           }
         }
@@ -423,20 +424,20 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
           if (!proj) {
             emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], y, nz, red, g, D.smask + ep->dst);
           } else {
-            uint64_t out[MAXW];
+            uint64_t out[MW];
 #pragma unroll
-            for (int s2 = 0; s2 < MAXW; ++s2) out[s2] = 0;
+            for (int s2 = 0; s2 < MW; ++s2) out[s2] = 0;
             for (uint32_t j = 0; j < W; ++j) {
               uint64_t b = 0;
 #pragma unroll
-              for (int jj = 0; jj < MAXW; ++jj) if ((uint32_t)jj == j) b = y[jj];
+              for (int jj = 0; jj < MW; ++jj) if ((uint32_t)jj == j) b = y[jj];
               while (b) {
                 const int bit = __ffsll((long long)b) - 1;
                 b &= b - 1;
                 const int cd = ws.cmap[j * 64 + bit];
                 if (cd < 0) continue;
 #pragma unroll
-                for (int s2 = 0; s2 < MAXW; ++s2)
+                for (int s2 = 0; s2 < MW; ++s2)
                   if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
               }
             }
@@ -460,7 +461,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
 }
 
 // ---------------------------------------------------------------------------------- one item
-template <bool WIDE, bool CNT>
+template <bool WIDE, bool CNT, int MW>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
@@ -478,7 +479,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   if constexpr (WIDE) {
     if (R.logW >= 1) {                                      // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
-      process_wide<CNT>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
+      process_wide<CNT, MW>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
                    allow_cont ? &cont_v : nullptr, GD_CONT_DENSE && light);
       return cont_v;
     }
@@ -696,9 +697,9 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
             for (int k = 0; k < KW; ++k) {
               if (src[k] < 0) continue;
               const uint32_t r = r0 + lane + 32 * k;
-              uint64_t out[MAXW];
+              uint64_t out[MW];
 #pragma unroll
-              for (int q = 0; q < MAXW; ++q) out[q] = 0;
+              for (int q = 0; q < MW; ++q) out[q] = 0;
               for (uint32_t j = 0; j < W; ++j) {
                 uint64_t b = X[((uint64_t)src[k] << logW) + j];
                 while (b) {
@@ -707,7 +708,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                   const int cd = ws.cmap[j * 64 + bit];
                   if (cd < 0) continue;
 #pragma unroll
-                  for (int q = 0; q < MAXW; ++q)
+                  for (int q = 0; q < MW; ++q)
                     if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
                 }
               }
@@ -764,7 +765,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 
 // Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
-template <bool WIDE, bool CNT>
+template <bool WIDE, bool CNT, int MW>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
@@ -847,11 +848,11 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
     }
     if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
-      process_item<WIDE, CNT>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
+      process_item<WIDE, CNT, MW>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
     } else {
       uint32_t n = entry >> 5, ci = entry & 31u;
       for (int depth = 0;; ++depth) {
-        const uint32_t c = process_item<WIDE, CNT>(D, st, n, ci, round, nxt, lane, ws, acc,
+        const uint32_t c = process_item<WIDE, CNT, MW>(D, st, n, ci, round, nxt, lane, ws, acc,
                                               depth < GD_CONT_DEPTH, cont_ok);
         if (c == NO_CONT) break;
         __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
@@ -867,7 +868,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   return total;
 }
 
-template <bool WIDE, bool CNT>
+template <bool WIDE, bool CNT, int MW>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -879,7 +880,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   stage_init(st);
   __syncthreads();
   for (uint32_t round = 1;; ++round) {
-    const uint32_t total = run_round<WIDE, CNT>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+    const uint32_t total = run_round<WIDE, CNT, MW>(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == 0) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
@@ -891,7 +892,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
   flush_acc(D, acc);
 }
 
-template <bool WIDE, bool CNT>
+template <bool WIDE, bool CNT, int MW>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t round) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
@@ -902,7 +903,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
-  const uint32_t total = run_round<WIDE, CNT>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+  const uint32_t total = run_round<WIDE, CNT, MW>(D, st, round, gw, nw, lane, ws_all[wib], acc);
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);
@@ -1014,39 +1015,48 @@ cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-int fixpoint_max_blocks(int device, bool wide) {
-  int sms = 0, occ = 0;
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  int occ2 = 0;
-  if (wide) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<true, true>, THREADS, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_fixpoint<true, false>, THREADS, 0);
-  } else {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_fixpoint<false, true>, THREADS, 0);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, k_fixpoint<false, false>, THREADS, 0);
+// Instantiations: narrow batches (WIDE = false) and wide batches by the widest row of the
+// batch (MW = 2, 4, 8 words: register arrays sized to it), each with and without the
+// byte-model counters (CNT).
+template <bool CNT>
+static const void* fixpoint_fn(uint32_t wide) {
+  switch (wide) {
+    case 0: return (const void*)k_fixpoint<false, CNT, 1>;
+    case 1: return (const void*)k_fixpoint<true, CNT, 2>;
+    case 2: return (const void*)k_fixpoint<true, CNT, 4>;
+    default: return (const void*)k_fixpoint<true, CNT, 8>;
   }
+}
+
+int fixpoint_max_blocks(int device, uint32_t wide) {
+  int sms = 0, occ = 0, occ2 = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fixpoint_fn<true>(wide), THREADS, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, fixpoint_fn<false>(wide), THREADS, 0);
   occ = occ2 < occ ? occ2 : occ;          // one grid size serves both instantiations
   return sms * (occ > 0 ? occ : 1);
 }
 
-// The wide (row-sparse) path is compiled into a separate instantiation so batches without wide
-// modules keep the dense path's register allocation.
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s) {
   Dev d = D;
   void* args[] = {&d};
-  const void* f = D.wide ? (D.count ? (const void*)k_fixpoint<true, true> : (const void*)k_fixpoint<true, false>)
-                         : (D.count ? (const void*)k_fixpoint<false, true> : (const void*)k_fixpoint<false, false>);
+  const void* f = D.count ? fixpoint_fn<true>(D.wide) : fixpoint_fn<false>(D.wide);
   return cudaLaunchCooperativeKernel(f, dim3(blocks), dim3(THREADS), args, 0, s);
 }
 
-cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s) {
-  if (D.wide) {
-    if (D.count) k_round<true, true><<<blocks, THREADS, 0, s>>>(D, round);
-    else k_round<true, false><<<blocks, THREADS, 0, s>>>(D, round);
-  } else {
-    if (D.count) k_round<false, true><<<blocks, THREADS, 0, s>>>(D, round);
-    else k_round<false, false><<<blocks, THREADS, 0, s>>>(D, round);
+template <bool CNT>
+static void round_launch(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s) {
+  switch (D.wide) {
+    case 0: k_round<false, CNT, 1><<<blocks, THREADS, 0, s>>>(D, round); break;
+    case 1: k_round<true, CNT, 2><<<blocks, THREADS, 0, s>>>(D, round); break;
+    case 2: k_round<true, CNT, 4><<<blocks, THREADS, 0, s>>>(D, round); break;
+    default: k_round<true, CNT, 8><<<blocks, THREADS, 0, s>>>(D, round); break;
   }
+}
+
+cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s) {
+  if (D.count) round_launch<true>(D, round, blocks, s);
+  else round_launch<false>(D, round, blocks, s);
   return cudaGetLastError();
 }
 

@@ -650,7 +650,7 @@ struct Layout {
   std::vector<uint32_t> app_base;
   uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
-  bool wide = false;
+  uint32_t wide = 0;            // max logW over the modules
 };
 
 // Process-wide pinned staging buffer and per-app host images, reused by every load: in this
@@ -701,7 +701,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
                     b[k].frow + h.frow.size(), b[k].args + h.args.size(), b[k].fact + h.fact_words,
                     b[k].ent + h.entries.size()};
     for (int c = 0; c < NCLS; ++c) Lo.cls_count[c] += h.cls_count[c];
-    for (const ModRec& md : h.mods) Lo.wide |= md.logW >= 1;
+    for (const ModRec& md : h.mods) Lo.wide = std::max<uint32_t>(Lo.wide, md.logW);
   }
   const Base& T = b[n_apps];
   if (T.node >= (1ull << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
@@ -1126,7 +1126,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   for (int c = 0; c < NCLS; ++c) { D.seg[c] = acc; acc += Lo.cls_count[c]; a->cls_count[c] = Lo.cls_count[c]; }
   D.seg[NCLS] = acc;
   D.n_words = Lo.fact_words;
-  D.wide = Lo.wide ? 1u : 0u;
+  D.wide = Lo.wide;
 
   // ---- fact store + mutable state
   {
@@ -1153,7 +1153,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     for (auto& ev : a->ev)
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
-  a->max_blocks = fixpoint_max_blocks(device, D.wide != 0);
+  a->max_blocks = fixpoint_max_blocks(device, D.wide);
   *out = a;
   return GDROID_OK;
 }
