@@ -28,7 +28,8 @@ struct __align__(16) NodeRec {
   uint8_t kind;      // gdroid_node_kind
   uint8_t cls;       // Cls
   uint8_t logW;      // log2 words per row
-  uint8_t pad;
+  uint8_t n_inl;     // edges of chunk 0 held inline in InlEdge[4 * n ..] (all INTRA/C2R, narrow
+                     // block of <= 128 words), 0 = read them from the edge array
   int32_t r0;        // lhs row (PRIM/CONST/NEW/COPY/SLOAD/RETV/FLOAD/ALOAD), static row (SSTORE),
                      // base row (FSTORE/ASTORE), lhs row of the call (CALL/RETSITE) or -1
   int32_t r1;        // rhs row (COPY/SLOAD/SSTORE/RETV), w row (FLOAD/ALOAD/FSTORE/ASTORE),
@@ -76,6 +77,17 @@ __host__ __device__ __forceinline__ uint32_t chunk_edges(uint32_t deg, uint32_t 
 __host__ __device__ __forceinline__ uint32_t n_chunks_of(uint32_t deg, uint32_t cls) {
   return deg == 0 ? 1u : (deg + chunk_edges(deg, cls) - 1) / chunk_edges(deg, cls);
 }
+
+// Chunk 0's INTRA/C2R out-edges of a narrow node, held beside its NodeRec (4 x 16 B = one
+// 64-byte record per node, loaded in the same memory hop as the NodeRec): an intra-method edge
+// keeps the source's block layout, so only the destination id, info and fact offset are needed.
+struct __align__(16) InlEdge {
+  uint32_t dst;
+  uint32_t info;       // as Edge::info
+  uint64_t off;        // fact-block word offset of dst
+};
+static_assert(sizeof(InlEdge) == 16, "InlEdge must be 16 bytes");
+constexpr uint32_t INL_MAX_B = 128;   // inline path: narrow source blocks of at most 128 words
 
 struct __align__(16) MethRec {
   uint32_t n_locals, n_params, module, local_base;   // local_base: app-local slot gid of local 0
@@ -126,6 +138,7 @@ struct Dev {
   const ModRec* mods;
   const uint32_t* row_ptr;
   const Edge* edges;
+  const InlEdge* inl;           // [4 N] chunk-0 INTRA/C2R edges (NodeRec::n_inl of them valid)
   const uint32_t* arg_ptr;
   const int32_t* args;
   const uint32_t* col_gid;

@@ -37,8 +37,11 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_SMASK
 #define GD_SMASK 0             // narrow blocks: read only word groups flagged in D.smask (measured slower)
 #endif
-#ifndef GD_PF
-#define GD_PF 0                // prefetch the next item's fact lines / edges into L2 (two-ahead NodeRec)
+#ifndef GD_INL
+#define GD_INL 1               // chunk-0 INTRA/C2R edges read from the inline record (one hop less)
+#endif
+#ifndef GD_PRE
+#define GD_PRE 1               // inline path: load IN(dst) of the first two edges with IN(src)
 #endif
 #ifndef GD_CONT_DENSE
 #define GD_CONT_DENSE 0        // continue into narrow (one word per row) destinations too (light rounds)
@@ -113,10 +116,13 @@ __device__ __forceinline__ void stage_init(CtaStage& st) {
 // a second warp from continuing into the same node in the same round (it queues it instead).
 __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
                                              uint32_t dst, uint32_t info, bool grew, uint32_t round,
-                                             uint32_t nxt, uint32_t* cont = nullptr, bool cont_dense = false) {
+                                             uint32_t nxt, uint32_t* cont = nullptr, bool cont_dense = false,
+                                             uint32_t pre_stamp = NO_CONT) {
   bool push = false;
   bool want = false;
-  if (active) want = grew || (D.stamp[dst] == 0);           // grew, or first reach (A5)
+  // grew, or first reach (A5).  pre_stamp: stamp[dst] loaded early by the caller (a stale value
+  // is safe: stamps only grow, and the atomicMax below decides the push)
+  if (active) want = grew || ((pre_stamp != NO_CONT ? pre_stamp : D.stamp[dst]) == 0);
   if (cont && *cont == NO_CONT && (D.flags & F_CONT)) {
     const unsigned cand = __ballot_sync(FULL, want && (cont_dense || (info & INFO_WIDE)) && ((info >> 5) & 31u) == 0);
     if (cand) {
@@ -460,6 +466,146 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
   }
 }
 
+// ---------------------------------------------------------------------------------- inline items
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+  const uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src), hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src);
+  return ((uint64_t)hi << 32) | lo;
+}
+// Word r of a block held as y[k] = word lane + 32k.  uword_of: r warp-uniform (one shuffle);
+// word_of: r per lane (every lane takes part).
+__device__ __forceinline__ uint64_t uword_of(const uint64_t (&y)[KW], uint32_t r) {
+  uint64_t s = y[0];
+#pragma unroll
+  for (int k = 1; k < KW; ++k) if ((r >> 5) == (uint32_t)k) s = y[k];
+  return shfl64(s, (int)(r & 31u));
+}
+__device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r) {
+  uint64_t s = 0;
+#pragma unroll
+  for (int k = 0; k < KW; ++k) {
+    const uint64_t v = shfl64(y[k], (int)(r & 31u));
+    if ((r >> 5) == (uint32_t)k) s = v;
+  }
+  return s;
+}
+
+// Chunk 0 of a narrow node (block of <= 128 words) whose edges are all INTRA/C2R and held in
+// the node's inline record (NodeRec::n_inl).  Same transfer and union as process_item's narrow
+// path, with every read that the chain allows issued in the first memory hop: IN(src), the
+// destinations' round stamps and (FLOAD/FSTORE) the field-row table; the rows the transfer
+// function reads are taken from the IN(src) registers by shuffles instead of reloads.
+template <bool CNT>
+__device__ __forceinline__ void process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
+                                               uint32_t round, uint32_t nxt, int lane, Acc& acc) {
+  const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
+  const uint64_t* __restrict__ X = D.facts + R.off;
+  uint64_t y[KW], p0[KW], p1[KW];
+  const uint64_t off0 = shfl64(me.off, 0), off1 = shfl64(me.off, 1);
+#pragma unroll
+  for (int k = 0; k < KW; ++k) {
+    const uint32_t w = lane + 32 * k;
+    y[k] = w < B ? X[w] : 0ull;
+    if (GD_PRE) {                                           // IN(dst) of edges 0 and 1, same hop
+      p0[k] = w < B ? D.facts[off0 + w] : 0ull;
+      p1[k] = (ne > 1 && w < B) ? D.facts[off1 + w] : 0ull;
+    }
+  }
+  const uint32_t my_stamp = lane < (int)ne ? D.stamp[me.dst] : 1u;
+  const bool dbl = kind == GK_FLOAD || kind == GK_ALOAD || kind == GK_FSTORE || kind == GK_ASTORE;
+  int hr[2] = {-1, -1};                                     // heap rows of this lane's columns
+  if (dbl) {
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const uint32_t c = lane + 32 * q;
+      hr[q] = (c < R.n_cols) ? D.frow[R.r3 + c] : -1;
+    }
+  }
+  // ---- transfer (DESIGN.md §3 C2), on the registers
+  int mode = 0, t = -1;                                     // 0 identity, 1 replace, 2 or-in, 3 FSTORE
+  uint64_t genv = 0;
+  uint32_t fmask = 0, hwords = 0;
+  if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
+    mode = 1; t = R.r0;
+    if (kind != GK_PRIM) genv = 1ull << (R.r3 & 63);
+  } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
+    mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
+    genv = uword_of(y, (uint32_t)R.r1);                     // row rhs
+  } else if (kind == GK_FLOAD || kind == GK_ALOAD) {       // v = w.f: OR of rows (o1,f), o1 ∈ w
+    mode = 1; t = R.r0;
+    const uint64_t wrow = uword_of(y, (uint32_t)R.r1);
+    uint64_t a = 0;
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const uint32_t c = lane + 32 * q;
+      const bool take = hr[q] >= 0 && ((wrow >> c) & 1ull);  // NULL has no row
+      const uint64_t v = word_of(y, take ? L + (uint32_t)hr[q] : 0u);
+      if (take) { a |= v; hwords += 1; }
+    }
+    genv = warp_or64(a);
+  } else if (kind == GK_FSTORE || kind == GK_ASTORE) {     // v.f = w (weak)
+    mode = 3;
+    const uint64_t vrow = uword_of(y, (uint32_t)R.r0);
+    genv = uword_of(y, (uint32_t)R.r1);                     // row w, OR-ed into rows (o1, f)
+#pragma unroll
+    for (int k = 0; k < KW; ++k) {
+      uint32_t m = 0;
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        const uint32_t c = lane + 32 * q;
+        if (hr[q] >= 0 && ((vrow >> c) & 1ull)) {
+          const uint32_t w = L + (uint32_t)hr[q];
+          if ((w >> 5) == (uint32_t)k) m |= 1u << (w & 31u);
+        }
+      }
+      m = __reduce_or_sync(FULL, m);
+      if ((m >> lane) & 1u) fmask |= 1u << k;
+    }
+  }
+  uint32_t nzx = 0, nz = 0, red = 0;
+#pragma unroll
+  for (int k = 0; k < KW; ++k) {
+    const uint32_t w = lane + 32 * k;
+    if (CNT) nzx += (y[k] != 0);
+    if (mode == 1) { if ((int)w == t) y[k] = genv; }
+    else if (mode == 2) { if ((int)w == t) y[k] |= genv; }
+    else if (mode == 3) { if ((fmask >> k) & 1u) y[k] |= genv; }
+  }
+  // ---- unions into IN(dst) (a5)
+  unsigned gmask = 0;
+  for (uint32_t i = 0; i < ne; ++i) {
+    const uint64_t off = shfl64(me.off, (int)i);
+    const uint32_t info = __shfl_sync(FULL, me.info, (int)i);
+    const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;  // C2R drops lhs(c)
+    uint64_t* Z = D.facts + off;
+    uint64_t cur[KW];
+#pragma unroll
+    for (int k = 0; k < KW; ++k) {
+      const uint32_t w = lane + 32 * k;
+      const bool keep = y[k] && (int)w != kill;
+      if (GD_PRE && i == 0) cur[k] = keep ? p0[k] : ~0ull;
+      else if (GD_PRE && i == 1) cur[k] = keep ? p1[k] : ~0ull;
+      else cur[k] = keep ? Z[w] : ~0ull;
+    }
+    bool g = false;
+#pragma unroll
+    for (int k = 0; k < KW; ++k) {
+      const uint32_t w = lane + 32 * k;
+      const uint64_t z = (int)w == kill ? 0ull : y[k];
+      nz += (z != 0);
+      if (z & ~cur[k]) { red_or(Z + w, z); ++red; g = true; }
+    }
+    if (__any_sync(FULL, g)) gmask |= 1u << i;
+  }
+  flush_pushes(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt, nullptr, false,
+               my_stamp);
+  if constexpr (CNT) {
+    const uint32_t alg_l0 = (uint32_t)sizeof(NodeRec) + (uint32_t)sizeof(InlEdge) * ne + 4u;
+    acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
+    acc_add(acc.atom, red);
+    if (lane == 0) acc.dense += 8ull * B + 16ull * B * ne + alg_l0;
+  }
+}
+
 // ---------------------------------------------------------------------------------- one item
 template <bool WIDE, bool CNT, int MW>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
@@ -467,6 +613,8 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                                  bool light = false) {
   const uint64_t mk = GD_SMASK ? __ldcg(D.smask + n) : ~0ull;   // (issued with the NodeRec load)
   const NodeRec R = D.nodes[n];
+  InlEdge me{0u, 0u, 0ull};                                 // inline chunk-0 edge of this lane (same hop)
+  if (GD_INL && !WIDE && lane < 4) me = D.inl[4 * n + lane];
   const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
   const bool first = ci == 0;
@@ -483,6 +631,10 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                    allow_cont ? &cont_v : nullptr, GD_CONT_DENSE && light);
       return cont_v;
     }
+  }
+  if (GD_INL && !WIDE && !GD_SMASK && first && R.n_inl) {   // (wide batches: measured slower)
+    process_inline<CNT>(D, st, R, me, round, nxt, lane, acc);
+    return NO_CONT;
   }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
@@ -769,9 +921,9 @@ template <bool WIDE, bool CNT, int MW>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
-  if (D.bar[2]) return 0;                 // an earlier round found the worklist empty
   uint32_t cnt[NCLS];
   uint32_t total = 0;
+  if (D.bar[2]) return 0;                 // an earlier round found the worklist empty
 #pragma unroll
   for (int c = 0; c < NCLS; ++c) { cnt[c] = D.counts[cur * CNT_STRIDE + c]; total += cnt[c]; }
   if (total == 0) {
@@ -816,8 +968,6 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   const uint32_t head = ((D.flags & F_MER) && total > nw) ? (total / nw) * nw : total;
   uint32_t item = gw;
   uint32_t entry = item < total ? entry_of(item) : 0u;
-  if (GD_PF && item + nw < total && lane < 4)                           // first look-ahead NodeRec
-    asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (entry_of(item + nw) >> 5)) + 16 * lane));
   while (item < total) {
     if (item >= head) {                                                // tail: defer to round+1
       const uint32_t n = entry >> 5;
@@ -833,19 +983,9 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     }
     const uint32_t nitem = item + nw;
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
-    if (GD_PF) {
-      // two ahead: NodeRec of item + 2nw into L1; the next item's fact lines and edge records
-      // into L2 (its NodeRec was prefetched one item ago)
-      const uint32_t n2 = nitem + nw;
-      if (n2 < total && lane < 4)
-        asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (entry_of(n2) >> 5)) + 16 * lane));
-      if (nitem < total && lane < 9) {
-        const NodeRec* RN = D.nodes + (nentry >> 5);
-        const char* a = lane < 8 ? (const char*)(D.facts + RN->off) + 128 * lane : (const char*)(D.edges + RN->e0);
-        if (lane == 8 || (uint32_t)(16 * lane) < RN->B) asm volatile("prefetch.global.L2 [%0];" :: "l"(a));
-      }
-    } else if (nitem < total && lane < 4) {                            // NodeRec into L1
-      asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + (nentry >> 5)) + 16 * lane));
+    if (nitem < total && lane < 2) {                                   // NodeRec, inline edges into L1
+      const uint32_t nn = nentry >> 5;
+      asm volatile("prefetch.global.L1 [%0];" :: "l"(lane == 0 ? (const char*)(D.nodes + nn) : (const char*)(D.inl + 4 * nn)));
     }
     if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
       process_item<WIDE, CNT, MW>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);

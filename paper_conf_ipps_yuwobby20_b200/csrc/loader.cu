@@ -85,6 +85,7 @@ struct HostImage {
   std::vector<ModRec> mods;
   std::vector<uint32_t> row_ptr{0};
   std::vector<Edge> edges;
+  std::vector<InlEdge> inl;                    // [4 N] chunk-0 INTRA/C2R edges (NodeRec::n_inl)
   std::vector<uint32_t> arg_ptr{0};
   std::vector<int32_t> args;
   std::vector<uint32_t> col_gid, col_hbase;
@@ -384,7 +385,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
   };
-  H.nodes.resize(nb + N); H.node_method.resize(nb + N);
+  H.nodes.resize(nb + N); H.node_method.resize(nb + N); H.inl.resize(4 * (nb + N));
   H.row_ptr.resize(nb + N + 1); H.arg_ptr.resize(nb + N + 1); H.args.resize(n_args);
   FirstErr fe;
   std::mutex cls_mu;
@@ -621,6 +622,22 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       out_edges[e] = E2;
     }
     if (kind == GK_CALL && n_c2r != 1) return set_err(GDROID_E_INVALID, "app %u: node %llu: a CALL needs exactly one C2R edge (V5)", k, (unsigned long long)n);
+    // chunk 0 inline beside the NodeRec when it holds only INTRA/C2R edges of a narrow block
+    NodeRec& RN = H.nodes[nb + n];
+    const uint32_t deg = (uint32_t)(d->row_ptr[n + 1] - d->row_ptr[n]);
+    const uint32_t n0 = std::min(deg, chunk_edges(deg, RN.cls));
+    bool inl = deg > 0 && n0 <= 4 && RN.logW == 0 && RN.B <= INL_MAX_B;
+    for (uint32_t j = 0; j < n0 && inl; ++j) {
+      const uint32_t ek = out_edges[d->row_ptr[n] + j].info & 3u;
+      inl = ek == GE_INTRA || ek == GE_C2R;
+    }
+    if (inl) {
+      for (uint32_t j = 0; j < n0; ++j) {
+        const Edge& E2 = out_edges[d->row_ptr[n] + j];
+        H.inl[4 * (nb + n) + j] = InlEdge{E2.dst, E2.info, E2.off};
+      }
+      RN.n_inl = (uint8_t)n0;
+    }
     return GDROID_OK;
   };
   parallel_ranges(N, 1 << 14, [&](uint64_t lo, uint64_t hi) {
@@ -641,7 +658,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
 
 enum PartId { P_NODES, P_METHS, P_MODS, P_ROWPTR, P_EDGES, P_ARGPTR, P_ARGS, P_COLGID, P_COLTYPE,
               P_COLHB, P_GROWGID, P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE, P_ENTRIES,
-              P_NODEMETH, P_FROW, NPART };
+              P_NODEMETH, P_FROW, P_INL, NPART };
 
 // Device-table layout of a batch inside the staging buffer.
 struct Layout {
@@ -664,7 +681,7 @@ struct LoadCache {
 LoadCache g_cache;
 
 void reset_image(HostImage& h) {
-  h.nodes.clear(); h.meths.clear(); h.mods.clear(); h.edges.clear(); h.args.clear();
+  h.nodes.clear(); h.inl.clear(); h.meths.clear(); h.mods.clear(); h.edges.clear(); h.args.clear();
   h.col_gid.clear(); h.col_hbase.clear(); h.col_type.clear(); h.grow_gid.clear(); h.grow_col.clear();
   h.grow_field.clear(); h.tf.clear(); h.xmap.clear(); h.frow.clear(); h.app_node_base.clear();
   h.entries.clear(); h.node_method.clear();
@@ -718,7 +735,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
       T.edge * sizeof(Edge), (T.node + 1) * 4, std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4,
       T.col * 4, T.grow * 4, T.grow * 4, T.grow * 4, (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4,
       std::max<uint64_t>(T.xmap, 1) * 4, (n_apps + 1) * 4, std::max<uint64_t>(T.ent, 1) * 4, T.node * 4,
-      std::max<uint64_t>(T.frow, 1) * 4};
+      std::max<uint64_t>(T.frow, 1) * 4, T.node * 4 * sizeof(InlEdge)};
   Lo.total = 0;
   for (int p = 0; p < NPART; ++p) { Lo.off[p] = Lo.total; Lo.total += align256(bytes[p]); }
   if (g_cache.cap < Lo.total) {
@@ -751,6 +768,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   uint32_t* g_entries = (uint32_t*)P(P_ENTRIES);
   uint32_t* g_nodemeth = (uint32_t*)P(P_NODEMETH);
   int32_t* g_frow = (int32_t*)P(P_FROW);
+  InlEdge* g_inl = (InlEdge*)P(P_INL);
   g_rowptr[0] = 0; g_argptr[0] = 0; g_tfptr[0] = 0;
   g_args[0] = -1; g_tf[0] = 0; g_xmap[0] = -1; g_entries[0] = 0; g_frow[0] = -1;   // non-empty
   for (uint32_t k = 0; k <= n_apps; ++k) g_appbase[k] = (uint32_t)b[k].node;
@@ -775,6 +793,11 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
         R.col_off += (uint32_t)B.col; R.grow_off += (uint32_t)B.grow; R.module += (uint32_t)B.mod;
         if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)B.frow;
         g_nodes[B.node + i] = R;
+        for (uint32_t j = 0; j < 4; ++j) {
+          InlEdge X = h.inl[4 * i + j];
+          if (j < R.n_inl) { X.dst += (uint32_t)B.node; X.off += B.fact; }
+          g_inl[4 * (B.node + i) + j] = X;
+        }
         g_nodemeth[B.node + i] = h.node_method[i] + (uint32_t)B.meth;
         g_rowptr[B.node + i + 1] = h.row_ptr[i + 1] + (uint32_t)B.edge;
         g_argptr[B.node + i + 1] = h.arg_ptr[i + 1] + (uint32_t)B.args;
@@ -1119,6 +1142,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.entries = (const uint32_t*)(T + Lo.off[P_ENTRIES]);
   D.node_method = (const uint32_t*)(T + Lo.off[P_NODEMETH]);
   D.frow = (const int32_t*)(T + Lo.off[P_FROW]);
+  D.inl = (const InlEdge*)(T + Lo.off[P_INL]);
   D.n_nodes = N;
   D.n_chunks = NC;
   D.n_entries = (uint32_t)Lo.n_entries;
