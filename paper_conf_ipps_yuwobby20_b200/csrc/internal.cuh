@@ -216,6 +216,8 @@ cudaError_t launch_plain_gather(const PlainDev& P, uint32_t n0, uint32_t n1, con
 
 // kernels.cu launch wrappers (return cudaError_t of the launch)
 cudaError_t launch_seed(const Dev& D, cudaStream_t s);
+cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,
+                         const uint8_t* ekind, const uint32_t* exoff, cudaStream_t s);
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_digest(const Dev& D, cudaStream_t s);

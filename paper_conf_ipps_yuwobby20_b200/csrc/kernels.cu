@@ -1050,6 +1050,41 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   flush_acc(D, acc);
 }
 
+// (a1) Edge records (destination layout copied in) and the inline chunk-0 records, one thread
+// per source node: col is app-local, so the destination id is app_node_base[app] + col[e].
+// CALL aux = the callee's n_params (its ENTRY NodeRec holds it in r1); RET aux = lhs(c) of the
+// return site (its r0).  Chunk 0 goes inline when it holds only INTRA/C2R edges of a narrow
+// block of <= INL_MAX_B words.
+__global__ void k_edges(Dev D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* __restrict__ ecol,
+                        const uint8_t* __restrict__ ekind, const uint32_t* __restrict__ exoff) {
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < D.n_nodes; n += stride) {
+    const NodeRec R = nodes[n];
+    const uint32_t base = D.app_node_base[R.app];
+    const uint32_t deg = R.e1 - R.e0, n0 = min(deg, chunk_edges(deg, R.cls));
+    bool inl_ok = deg > 0 && n0 <= 4 && R.logW == 0 && R.B <= INL_MAX_B;
+    InlEdge rec[4];
+    for (uint32_t e = R.e0; e < R.e1; ++e) {
+      const uint32_t s = base + ecol[e], ek = ekind[e];
+      const NodeRec& RS = nodes[s];
+      const uint32_t cls = RS.cls, logW = RS.logW;
+      const uint32_t nch = n_chunks_of(RS.e1 - RS.e0, cls);
+      Edge E2;
+      E2.dst = s;
+      E2.info = ek | (cls << 2) | ((nch - 1) << 5) | (logW >= 1 ? INFO_WIDE : 0u);
+      E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = (uint8_t)logW; E2.pad = 0;
+      E2.aux = ek == GE_CALL ? RS.r1 : (ek == GE_RET ? RS.r0 : -1);
+      E2.xoff = exoff[e];
+      edges[e] = E2;
+      const uint32_t j = e - R.e0;
+      if (j < 4) rec[j] = InlEdge{E2.dst, E2.info, E2.off};
+      if (j < n0) inl_ok = inl_ok && (ek == GE_INTRA || ek == GE_C2R);
+    }
+    for (uint32_t j = 0; j < 4; ++j) inl[4 * n + j] = (inl_ok && j < n0) ? rec[j] : InlEdge{0u, 0u, 0ull};
+    nodes[n].n_inl = inl_ok ? (uint8_t)n0 : (uint8_t)0;   // (other threads read other fields only)
+  }
+}
+
 // (a2) seed round 1 with the component entries (Alg. 1 l.9)
 __global__ void k_seed(Dev D) {
   __shared__ CtaStage st;
@@ -1149,6 +1184,14 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
 }
 
 }  // namespace
+
+cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,
+                         const uint8_t* ekind, const uint32_t* exoff, cudaStream_t s) {
+  uint32_t blocks = (D.n_nodes + 255) / 256;
+  blocks = blocks == 0 ? 1u : (blocks > 148 * 8 ? 148 * 8 : blocks);
+  k_edges<<<blocks, 256, 0, s>>>(D, edges, inl, nodes, ecol, ekind, exoff);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
   k_seed<<<1, 32, 0, s>>>(D);

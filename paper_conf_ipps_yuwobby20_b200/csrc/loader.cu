@@ -84,8 +84,11 @@ struct HostImage {
   std::vector<MethRec> meths;
   std::vector<ModRec> mods;
   std::vector<uint32_t> row_ptr{0};
-  std::vector<Edge> edges;
-  std::vector<InlEdge> inl;                    // [4 N] chunk-0 INTRA/C2R edges (NodeRec::n_inl)
+  // edges: the device builds the Edge / InlEdge records (k_edges) from the descriptor's col and
+  // edge_kind plus the projection-table offset of each CALL/RET edge computed here
+  const gdroid_icfg_desc* desc = nullptr;
+  uint64_t n_edges = 0;
+  std::vector<uint32_t> xo;                    // [E] app-local xmap offset | NO_XMAP
   std::vector<uint32_t> arg_ptr{0};
   std::vector<int32_t> args;
   std::vector<uint32_t> col_gid, col_hbase;
@@ -100,6 +103,9 @@ struct HostImage {
   std::vector<uint32_t> node_method;
   uint64_t fact_words = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
+  // per-load temporaries, kept so their pages are touched once per process (first-touch faults
+  // cost more than the table build itself in this environment)
+  std::vector<uint64_t> t_heap_base, t_local_base, t_foff;
 };
 
 // Per-module host-side lookup info of the app being loaded.
@@ -110,24 +116,36 @@ struct ModInfo {
 };
 
 // Persistent worker pool for the host-side table build (spawning threads per parallel loop
-// costs more than the loops themselves on small apps).
+// costs more than the loops themselves on small apps).  Nested loops are allowed: a
+// parallel_for called from inside a task publishes its own job and its caller works on it (and
+// on any other open job) until it completes, so apps and node ranges inside apps share the
+// pool.
 class Pool {
  public:
+  struct Job {
+    const std::function<void(uint32_t)>* f = nullptr;
+    uint32_t n = 0;
+    std::atomic<uint32_t> next{0}, done{0}, refs{0};
+  };
   static Pool& get() {
     static Pool p;
     return p;
   }
   uint32_t size() const { return (uint32_t)workers_.size() + 1; }
-  // Run job(k) for k in [0, n); the caller participates.  Not re-entrant.
-  void run(uint32_t n, const std::function<void(uint32_t)>& job) {
-    std::unique_lock<std::mutex> lk(mu_);
-    job_ = &job; n_ = n; next_.store(0); pending_ = (uint32_t)workers_.size(); ++gen_;
-    lk.unlock();
+  void run(uint32_t n, const std::function<void(uint32_t)>& f) {
+    Job j;
+    j.f = &f; j.n = n;
+    {
+      std::lock_guard<std::mutex> lk(mu_);
+      jobs_.push_back(&j);
+    }
     cv_.notify_all();
-    for (uint32_t k; (k = next_.fetch_add(1)) < n;) job(k);
-    lk.lock();
-    done_cv_.wait(lk, [&] { return pending_ == 0; });
-    job_ = nullptr;
+    for (uint32_t k; (k = j.next.fetch_add(1)) < n;) { f(k); j.done.fetch_add(1); }
+    while (j.done.load() < n || j.refs.load() != 0)
+      if (!help_one()) std::this_thread::yield();
+    std::lock_guard<std::mutex> lk(mu_);
+    for (size_t i = 0; i < jobs_.size(); ++i)
+      if (jobs_[i] == &j) { jobs_.erase(jobs_.begin() + i); break; }
   }
 
  private:
@@ -136,42 +154,51 @@ class Pool {
     for (uint32_t t = 1; t < T; ++t) workers_.emplace_back([this] { loop(); });
   }
   ~Pool() {
-    { std::lock_guard<std::mutex> lk(mu_); stop_ = true; ++gen_; }
+    { std::lock_guard<std::mutex> lk(mu_); stop_ = true; }
     cv_.notify_all();
     for (auto& w : workers_) w.join();
   }
+  // Claim and run one index of an open job; false if there is none.  refs keeps the job (on its
+  // caller's stack) alive while a helper holds it.
+  bool help_one() {
+    Job* j = nullptr;
+    {
+      std::lock_guard<std::mutex> lk(mu_);
+      for (size_t i = 0; i < jobs_.size(); ++i)
+        if (jobs_[i]->next.load() < jobs_[i]->n) { j = jobs_[i]; break; }
+      if (!j) return false;
+      j->refs.fetch_add(1);
+    }
+    const uint32_t k = j->next.fetch_add(1);
+    if (k < j->n) { (*j->f)(k); j->done.fetch_add(1); }
+    j->refs.fetch_sub(1);
+    return true;
+  }
   void loop() {
-    uint64_t seen = 0;
     for (;;) {
+      if (help_one()) continue;
       std::unique_lock<std::mutex> lk(mu_);
-      cv_.wait(lk, [&] { return stop_ || gen_ != seen; });
       if (stop_) return;
-      seen = gen_;
-      const std::function<void(uint32_t)>* job = job_;
-      const uint32_t n = n_;
-      lk.unlock();
-      for (uint32_t k; (k = next_.fetch_add(1)) < n;) (*job)(k);
-      lk.lock();
-      if (--pending_ == 0) done_cv_.notify_one();
+      cv_.wait_for(lk, std::chrono::milliseconds(2), [&] {
+        if (stop_) return true;
+        for (Job* j : jobs_) if (j->next.load() < j->n) return true;
+        return false;
+      });
+      if (stop_) return;
     }
   }
   std::vector<std::thread> workers_;
   std::mutex mu_;
-  std::condition_variable cv_, done_cv_;
-  const std::function<void(uint32_t)>* job_ = nullptr;
-  uint32_t n_ = 0, pending_ = 0;
-  uint64_t gen_ = 0;
+  std::condition_variable cv_;
+  std::vector<Job*> jobs_;
   bool stop_ = false;
-  std::atomic<uint32_t> next_{0};
 };
-std::mutex g_pool_mu;   // one parallel loop at a time (loads are serialised by g_cache.mu too)
 
-// Run f(k) for k in [0, n) on the worker pool.
+// Run f(k) for k in [0, n) on the worker pool (callable from inside a task).
 template <class F>
 void parallel_for(uint32_t n, F f) {
   if (n <= 1) { if (n) f(0); return; }
   std::function<void(uint32_t)> job = [&](uint32_t k) { f(k); };
-  std::lock_guard<std::mutex> lk(g_pool_mu);
   Pool::get().run(n, job);
 }
 
@@ -206,25 +233,33 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   const uint64_t N = d->n_nodes, E = d->n_edges, M = d->n_methods, Dm = d->n_modules;
   const uint64_t I = d->n_instances, G = d->n_statics, T = d->n_types;
   if (N == 0 || M == 0 || Dm == 0 || I == 0) return set_err(GDROID_E_INVALID, "app %u: empty ICFG", k);
-  if ((uint64_t)H.nodes.size() + N >= (1ull << 32) || (uint64_t)H.edges.size() + E >= (1ull << 32))
+  if ((uint64_t)H.nodes.size() + N >= (1ull << 32) || E >= (1ull << 32))
     return set_err(GDROID_E_LIMIT, "app %u: batch exceeds 2^32 nodes or edges", k);
   H.nodes.reserve(H.nodes.size() + N); H.node_method.reserve(H.node_method.size() + N);
-  H.edges.reserve(H.edges.size() + E); H.row_ptr.reserve(H.row_ptr.size() + N);
+  H.row_ptr.reserve(H.row_ptr.size() + N);
   H.arg_ptr.reserve(H.arg_ptr.size() + N); H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
   const uint32_t nb = (uint32_t)H.nodes.size(), mb = (uint32_t)H.meths.size();
   const uint32_t db = (uint32_t)H.mods.size(), tb = (uint32_t)(H.tf_ptr.size() - 1);
   // ---- CSR (structure)
   if (d->row_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: row_ptr[0] != 0", k);
-  for (uint64_t n = 0; n < N; ++n)
-    if (d->row_ptr[n + 1] < d->row_ptr[n]) return set_err(GDROID_E_INVALID, "app %u: row_ptr not monotone at node %llu", k, (unsigned long long)n);
-  if (d->row_ptr[N] != E) return set_err(GDROID_E_INVALID, "app %u: row_ptr[n_nodes] != n_edges", k);
-  for (uint64_t e = 0; e < E; ++e) {
-    if (d->col[e] >= N) return set_err(GDROID_E_INVALID, "app %u: edge %llu target out of range", k, (unsigned long long)e);
-    if (d->edge_kind[e] > GE_C2R) return set_err(GDROID_E_INVALID, "app %u: edge %llu bad kind", k, (unsigned long long)e);
-  }
-  for (uint64_t n = 0; n < N; ++n) {
-    if (d->node_kind[n] > GK_ASTORE) return set_err(GDROID_E_INVALID, "app %u: node %llu bad kind", k, (unsigned long long)n);
-    if (d->node_method[n] >= M) return set_err(GDROID_E_INVALID, "app %u: node %llu method out of range", k, (unsigned long long)n);
+  {
+    FirstErr fc;                                             // parallel over ranges; lowest index wins
+    parallel_ranges(N, 1 << 16, [&](uint64_t lo, uint64_t hi) {
+      for (uint64_t n = lo; n < hi; ++n) {
+        if (d->row_ptr[n + 1] < d->row_ptr[n]) { fc.offer(n, set_err(GDROID_E_INVALID, "app %u: row_ptr not monotone at node %llu", k, (unsigned long long)n)); return; }
+        if (d->node_kind[n] > GK_ASTORE) { fc.offer(n, set_err(GDROID_E_INVALID, "app %u: node %llu bad kind", k, (unsigned long long)n)); return; }
+        if (d->node_method[n] >= M) { fc.offer(n, set_err(GDROID_E_INVALID, "app %u: node %llu method out of range", k, (unsigned long long)n)); return; }
+      }
+    });
+    if (fc.st != GDROID_OK) return fc.result();
+    if (d->row_ptr[N] != E) return set_err(GDROID_E_INVALID, "app %u: row_ptr[n_nodes] != n_edges", k);
+    parallel_ranges(E, 1 << 17, [&](uint64_t lo, uint64_t hi) {
+      for (uint64_t e = lo; e < hi; ++e) {
+        if (d->col[e] >= N) { fc.offer(N + e, set_err(GDROID_E_INVALID, "app %u: edge %llu target out of range", k, (unsigned long long)e)); return; }
+        if (d->edge_kind[e] > GE_C2R) { fc.offer(N + e, set_err(GDROID_E_INVALID, "app %u: edge %llu bad kind", k, (unsigned long long)e)); return; }
+      }
+    });
+    if (fc.st != GDROID_OK) return fc.result();
   }
   PHASE("csr checks");
   // ---- types
@@ -239,7 +274,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     for (uint64_t q = d->type_field_ptr[t]; q < d->type_field_ptr[t + 1]; ++q) H.tf.push_back(d->type_fields[q]);
   }
   if (d->inst_type[0] != -1) return set_err(GDROID_E_INVALID, "app %u: instance 0 must be NULL (type -1)", k);
-  std::vector<uint64_t> heap_base(I + 1, 0);
+  std::vector<uint64_t>& heap_base = H.t_heap_base;
+  heap_base.assign(I + 1, 0);
   for (uint64_t o = 0; o < I; ++o) {
     const int32_t t = d->inst_type[o];
     if (t < -1 || t >= (int64_t)T) return set_err(GDROID_E_INVALID, "app %u: instance %llu type out of range", k, (unsigned long long)o);
@@ -247,7 +283,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   }
   PHASE("types");
   // ---- methods / slot numbering
-  std::vector<uint64_t> local_base(M + 1, 0);
+  std::vector<uint64_t>& local_base = H.t_local_base;
+  local_base.assign(M + 1, 0);
   for (uint64_t m = 0; m < M; ++m) {
     if (d->method_module[m] >= Dm) return set_err(GDROID_E_INVALID, "app %u: method %llu module out of range", k, (unsigned long long)m);
     if (d->method_n_locals[m] < d->method_n_params[m] + 1) return set_err(GDROID_E_INVALID, "app %u: method %llu n_locals < n_params + 1", k, (unsigned long long)m);
@@ -316,7 +353,9 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   // per range: call_arg_ptr monotone, fact-block sizes, (module, field) keys of heap accesses
   constexpr uint64_t RG = 1 << 15;
   const uint64_t n_rg = (N + RG - 1) / RG;
-  std::vector<uint64_t> foff(N + 1, 0), rg_sum(n_rg + 1, 0);
+  std::vector<uint64_t>& foff = H.t_foff;
+  foff.assign(N + 1, 0);
+  std::vector<uint64_t> rg_sum(n_rg + 1, 0);
   std::vector<std::vector<uint64_t>> rg_keys(n_rg);
   FirstErr fe0;
   auto fkey = [&](uint64_t n) -> uint64_t {                 // UINT64_MAX: no field-row table
@@ -385,7 +424,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
   };
-  H.nodes.resize(nb + N); H.node_method.resize(nb + N); H.inl.resize(4 * (nb + N));
+  H.nodes.resize(nb + N); H.node_method.resize(nb + N);
   H.row_ptr.resize(nb + N + 1); H.arg_ptr.resize(nb + N + 1); H.args.resize(n_args);
   FirstErr fe;
   std::mutex cls_mu;
@@ -569,8 +608,9 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   });
   PHASE("projection tables");
   // ---- edges (V5, V6), parallel over source-node ranges
-  H.edges.resize(H.edges.size() + E);
-  Edge* out_edges = H.edges.data() + (H.edges.size() - E);
+  H.desc = d;
+  H.n_edges = E;
+  H.xo.resize(E);
   auto edge_pass = [&](uint64_t n) -> gdroid_status {
     const uint8_t kind = d->node_kind[n];
     const uint64_t m = d->node_method[n];
@@ -611,33 +651,9 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           xoff = (uint32_t)(xbase + pair_off[i]);
         }
       }
-      const NodeRec& RS = H.nodes[nb + s];
-      const uint32_t nch = n_chunks_of((uint32_t)(d->row_ptr[s + 1] - d->row_ptr[s]), RS.cls);
-      Edge E2{};
-      E2.dst = nb + s;
-      E2.info = (uint32_t)ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5) | (RS.logW >= 1 ? INFO_WIDE : 0u);
-      E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = RS.logW;
-      E2.aux = (ek == GE_CALL) ? (int32_t)d->method_n_params[d->node_method[s]] : (ek == GE_RET ? RS.r0 : -1);
-      E2.xoff = xoff;
-      out_edges[e] = E2;
+      H.xo[e] = xoff;
     }
     if (kind == GK_CALL && n_c2r != 1) return set_err(GDROID_E_INVALID, "app %u: node %llu: a CALL needs exactly one C2R edge (V5)", k, (unsigned long long)n);
-    // chunk 0 inline beside the NodeRec when it holds only INTRA/C2R edges of a narrow block
-    NodeRec& RN = H.nodes[nb + n];
-    const uint32_t deg = (uint32_t)(d->row_ptr[n + 1] - d->row_ptr[n]);
-    const uint32_t n0 = std::min(deg, chunk_edges(deg, RN.cls));
-    bool inl = deg > 0 && n0 <= 4 && RN.logW == 0 && RN.B <= INL_MAX_B;
-    for (uint32_t j = 0; j < n0 && inl; ++j) {
-      const uint32_t ek = out_edges[d->row_ptr[n] + j].info & 3u;
-      inl = ek == GE_INTRA || ek == GE_C2R;
-    }
-    if (inl) {
-      for (uint32_t j = 0; j < n0; ++j) {
-        const Edge& E2 = out_edges[d->row_ptr[n] + j];
-        H.inl[4 * (nb + n) + j] = InlEdge{E2.dst, E2.info, E2.off};
-      }
-      RN.n_inl = (uint8_t)n0;
-    }
     return GDROID_OK;
   };
   parallel_ranges(N, 1 << 14, [&](uint64_t lo, uint64_t hi) {
@@ -656,14 +672,17 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
 }
 
 
-enum PartId { P_NODES, P_METHS, P_MODS, P_ROWPTR, P_EDGES, P_ARGPTR, P_ARGS, P_COLGID, P_COLTYPE,
-              P_COLHB, P_GROWGID, P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE, P_ENTRIES,
-              P_NODEMETH, P_FROW, P_INL, NPART };
+// Parts up to P_UPLOAD are staged on the host and uploaded; the edge records after it are
+// built on the device by k_edges from P_ECOL / P_EKIND / P_EXOFF.
+enum PartId { P_NODES, P_METHS, P_MODS, P_ROWPTR, P_ECOL, P_EKIND, P_EXOFF, P_ARGPTR, P_ARGS, P_COLGID,
+              P_COLTYPE, P_COLHB, P_GROWGID, P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE,
+              P_ENTRIES, P_NODEMETH, P_FROW, P_UPLOAD, P_EDGES = P_UPLOAD, P_INL, NPART };
 
 // Device-table layout of a batch inside the staging buffer.
 struct Layout {
   size_t off[NPART] = {};
-  size_t total = 0;
+  size_t total = 0;              // device bytes of the tables
+  size_t upload = 0;             // staged (host-built) prefix of them
   std::vector<uint32_t> app_base;
   uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
@@ -681,7 +700,7 @@ struct LoadCache {
 LoadCache g_cache;
 
 void reset_image(HostImage& h) {
-  h.nodes.clear(); h.inl.clear(); h.meths.clear(); h.mods.clear(); h.edges.clear(); h.args.clear();
+  h.nodes.clear(); h.meths.clear(); h.mods.clear(); h.xo.clear(); h.n_edges = 0; h.desc = nullptr; h.args.clear();
   h.col_gid.clear(); h.col_hbase.clear(); h.col_type.clear(); h.grow_gid.clear(); h.grow_col.clear();
   h.grow_field.clear(); h.tf.clear(); h.xmap.clear(); h.frow.clear(); h.app_node_base.clear();
   h.entries.clear(); h.node_method.clear();
@@ -699,11 +718,11 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   std::vector<HostImage>& img = g_cache.img;
   std::vector<gdroid_status> st(n_apps, GDROID_OK);
   std::vector<std::string> err(n_apps);
-  for (uint32_t k = 0; k < n_apps; ++k) {                  // each app is built in parallel inside
+  parallel_for(n_apps, [&](uint32_t k) {                   // apps in parallel, and node ranges inside
     reset_image(img[k]);
     st[k] = add_app(img[k], &descs[k], k);
     if (st[k] != GDROID_OK) err[k] = g_err;
-  }
+  });
   for (uint32_t k = 0; k < n_apps; ++k)
     if (st[k] != GDROID_OK) { g_err = err[k]; return st[k]; }
   PHASE("apps (parallel)");
@@ -712,7 +731,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   b[0] = Base{};
   for (uint32_t k = 0; k < n_apps; ++k) {
     const HostImage& h = img[k];
-    b[k + 1] = Base{b[k].node + h.nodes.size(), b[k].edge + h.edges.size(), b[k].meth + h.meths.size(),
+    b[k + 1] = Base{b[k].node + h.nodes.size(), b[k].edge + h.n_edges, b[k].meth + h.meths.size(),
                     b[k].mod + h.mods.size(), b[k].col + h.col_gid.size(), b[k].grow + h.grow_gid.size(),
                     b[k].type + (h.tf_ptr.size() - 1), b[k].tf + h.tf.size(), b[k].xmap + h.xmap.size(),
                     b[k].frow + h.frow.size(), b[k].args + h.args.size(), b[k].fact + h.fact_words,
@@ -732,19 +751,25 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
   const size_t bytes[NPART] = {
       T.node * sizeof(NodeRec), T.meth * sizeof(MethRec), T.mod * sizeof(ModRec), (T.node + 1) * 4,
-      T.edge * sizeof(Edge), (T.node + 1) * 4, std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4,
+      std::max<uint64_t>(T.edge, 1) * 4, std::max<uint64_t>(T.edge, 1), std::max<uint64_t>(T.edge, 1) * 4,
+      (T.node + 1) * 4, std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4,
       T.col * 4, T.grow * 4, T.grow * 4, T.grow * 4, (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4,
       std::max<uint64_t>(T.xmap, 1) * 4, (n_apps + 1) * 4, std::max<uint64_t>(T.ent, 1) * 4, T.node * 4,
-      std::max<uint64_t>(T.frow, 1) * 4, T.node * 4 * sizeof(InlEdge)};
+      std::max<uint64_t>(T.frow, 1) * 4, std::max<uint64_t>(T.edge, 1) * sizeof(Edge),
+      T.node * 4 * sizeof(InlEdge)};
   Lo.total = 0;
-  for (int p = 0; p < NPART; ++p) { Lo.off[p] = Lo.total; Lo.total += align256(bytes[p]); }
-  if (g_cache.cap < Lo.total) {
+  for (int p = 0; p < NPART; ++p) {
+    if (p == P_UPLOAD) Lo.upload = Lo.total;
+    Lo.off[p] = Lo.total;
+    Lo.total += align256(bytes[p]);
+  }
+  if (g_cache.cap < Lo.upload) {
     if (g_cache.stage) cudaFreeHost(g_cache.stage);
     g_cache.stage = nullptr;
     g_cache.cap = 0;
-    cudaError_t e = cudaMallocHost(&g_cache.stage, Lo.total + (Lo.total >> 2));
-    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "pinned staging (%zu B): %s", Lo.total, cudaGetErrorString(e));
-    g_cache.cap = Lo.total + (Lo.total >> 2);
+    cudaError_t e = cudaMallocHost(&g_cache.stage, Lo.upload + (Lo.upload >> 2));
+    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "pinned staging (%zu B): %s", Lo.upload, cudaGetErrorString(e));
+    g_cache.cap = Lo.upload + (Lo.upload >> 2);
   }
   char* S = (char*)g_cache.stage;
   auto P = [&](int p) { return S + Lo.off[p]; };
@@ -752,7 +777,9 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   MethRec* g_meths = (MethRec*)P(P_METHS);
   ModRec* g_mods = (ModRec*)P(P_MODS);
   uint32_t* g_rowptr = (uint32_t*)P(P_ROWPTR);
-  Edge* g_edges = (Edge*)P(P_EDGES);
+  uint32_t* g_ecol = (uint32_t*)P(P_ECOL);
+  uint8_t* g_ekind = (uint8_t*)P(P_EKIND);
+  uint32_t* g_exoff = (uint32_t*)P(P_EXOFF);
   uint32_t* g_argptr = (uint32_t*)P(P_ARGPTR);
   int32_t* g_args = (int32_t*)P(P_ARGS);
   uint32_t* g_colgid = (uint32_t*)P(P_COLGID);
@@ -768,7 +795,6 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   uint32_t* g_entries = (uint32_t*)P(P_ENTRIES);
   uint32_t* g_nodemeth = (uint32_t*)P(P_NODEMETH);
   int32_t* g_frow = (int32_t*)P(P_FROW);
-  InlEdge* g_inl = (InlEdge*)P(P_INL);
   g_rowptr[0] = 0; g_argptr[0] = 0; g_tfptr[0] = 0;
   g_args[0] = -1; g_tf[0] = 0; g_xmap[0] = -1; g_entries[0] = 0; g_frow[0] = -1;   // non-empty
   for (uint32_t k = 0; k <= n_apps; ++k) g_appbase[k] = (uint32_t)b[k].node;
@@ -779,7 +805,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   for (uint32_t k = 0; k < n_apps; ++k) {
     const HostImage& h = img[k];
     for (size_t lo = 0; lo < h.nodes.size(); lo += SLICE) units.push_back({k, 0, lo, std::min(h.nodes.size(), lo + SLICE)});
-    for (size_t lo = 0; lo < h.edges.size(); lo += SLICE) units.push_back({k, 1, lo, std::min(h.edges.size(), lo + SLICE)});
+    for (size_t lo = 0; lo < h.n_edges; lo += SLICE) units.push_back({k, 1, lo, std::min<size_t>(h.n_edges, lo + SLICE)});
     units.push_back({k, 2, 0, 0});
   }
   parallel_for((uint32_t)units.size(), [&](uint32_t u) {
@@ -793,11 +819,6 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
         R.col_off += (uint32_t)B.col; R.grow_off += (uint32_t)B.grow; R.module += (uint32_t)B.mod;
         if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)B.frow;
         g_nodes[B.node + i] = R;
-        for (uint32_t j = 0; j < 4; ++j) {
-          InlEdge X = h.inl[4 * i + j];
-          if (j < R.n_inl) { X.dst += (uint32_t)B.node; X.off += B.fact; }
-          g_inl[4 * (B.node + i) + j] = X;
-        }
         g_nodemeth[B.node + i] = h.node_method[i] + (uint32_t)B.meth;
         g_rowptr[B.node + i + 1] = h.row_ptr[i + 1] + (uint32_t)B.edge;
         g_argptr[B.node + i + 1] = h.arg_ptr[i + 1] + (uint32_t)B.args;
@@ -806,11 +827,11 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
     }
     if (U.kind == 1) {
       for (size_t i = U.lo; i < U.hi; ++i) {
-        Edge E = h.edges[i];
-        E.dst += (uint32_t)B.node; E.off += B.fact;
-        if (E.xoff != NO_XMAP) E.xoff += (uint32_t)B.xmap;
-        g_edges[B.edge + i] = E;
+        const uint32_t x = h.xo[i];
+        g_exoff[B.edge + i] = x == NO_XMAP ? NO_XMAP : x + (uint32_t)B.xmap;
       }
+      std::memcpy(g_ecol + B.edge + U.lo, h.desc->col + U.lo, (U.hi - U.lo) * 4);   // app-local ids
+      std::memcpy(g_ekind + B.edge + U.lo, h.desc->edge_kind + U.lo, U.hi - U.lo);
       return;
     }
     for (size_t i = 0; i < h.meths.size(); ++i) { MethRec M = h.meths[i]; M.module += (uint32_t)B.mod; g_meths[B.meth + i] = M; }
@@ -1112,7 +1133,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     t0 = std::chrono::steady_clock::now();
     cudaError_t e = cudaMallocAsync(&a->d_tables, Lo.total, a->stream);
     if (e != cudaSuccess) return fail(set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", Lo.total, cudaGetErrorString(e)));
-    e = cudaMemcpyAsync(a->d_tables, g_cache.stage, Lo.total, cudaMemcpyHostToDevice, a->stream);
+    e = cudaMemcpyAsync(a->d_tables, g_cache.stage, Lo.upload, cudaMemcpyHostToDevice, a->stream);
     cudaError_t e2 = cudaStreamSynchronize(a->stream);
     if (e != cudaSuccess || e2 != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "H2D upload: %s", cudaGetErrorString(e != cudaSuccess ? e : e2)));
   }
@@ -1151,6 +1172,15 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.seg[NCLS] = acc;
   D.n_words = Lo.fact_words;
   D.wide = Lo.wide;
+  {
+    // (a1) edge records and inline chunk-0 edges, derived on the device from col / edge_kind /
+    // projection offsets and the uploaded NodeRecs (stream-ordered after the upload)
+    cudaError_t e = launch_edges(D, (Edge*)(T + Lo.off[P_EDGES]), (InlEdge*)(T + Lo.off[P_INL]),
+                                 (NodeRec*)(T + Lo.off[P_NODES]), (const uint32_t*)(T + Lo.off[P_ECOL]),
+                                 (const uint8_t*)(T + Lo.off[P_EKIND]), (const uint32_t*)(T + Lo.off[P_EXOFF]),
+                                 a->stream);
+    if (e != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "k_edges: %s", cudaGetErrorString(e)));
+  }
 
   // ---- fact store + mutable state
   {
