@@ -89,6 +89,13 @@ struct __align__(16) InlEdge {
 static_assert(sizeof(InlEdge) == 16, "InlEdge must be 16 bytes");
 constexpr uint32_t INL_MAX_B = 128;   // inline path: narrow source blocks of at most 128 words
 
+// Per-app table bases of a batch: the loader stages each app's node tables with app-local
+// indices, k_rebase adds these.
+struct __align__(16) AppBase {
+  uint64_t fact;
+  uint32_t edge, meth, mod, col, grow, frow, args, pad;
+};
+
 struct __align__(16) MethRec {
   uint32_t n_locals, n_params, module, local_base;   // local_base: app-local slot gid of local 0
 };
@@ -216,6 +223,8 @@ cudaError_t launch_plain_gather(const PlainDev& P, uint32_t n0, uint32_t n1, con
 
 // kernels.cu launch wrappers (return cudaError_t of the launch)
 cudaError_t launch_seed(const Dev& D, cudaStream_t s);
+cudaError_t launch_rebase(const Dev& D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* rowptr, uint32_t* argptr,
+                          const AppBase* bases, cudaStream_t s);
 cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,
                          const uint8_t* ekind, const uint32_t* exoff, cudaStream_t s);
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s);

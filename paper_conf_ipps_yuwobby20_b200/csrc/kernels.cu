@@ -1050,6 +1050,23 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   flush_acc(D, acc);
 }
 
+// (a1) Rebase the staged app-local node tables by their app's bases (NodeRec::app).
+__global__ void k_rebase(Dev D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* rowptr, uint32_t* argptr,
+                         const AppBase* __restrict__ bases) {
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < D.n_nodes; n += stride) {
+    NodeRec R = nodes[n];
+    const AppBase b = bases[R.app];
+    R.off += b.fact; R.e0 += b.edge; R.e1 += b.edge;
+    R.col_off += b.col; R.grow_off += b.grow; R.module += b.mod;
+    if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)b.frow;
+    nodes[n] = R;
+    nodemeth[n] += b.meth;
+    rowptr[n + 1] += b.edge;
+    argptr[n + 1] += b.args;
+  }
+}
+
 // (a1) Edge records (destination layout copied in) and the inline chunk-0 records, one thread
 // per source node: col is app-local, so the destination id is app_node_base[app] + col[e].
 // CALL aux = the callee's n_params (its ENTRY NodeRec holds it in r1); RET aux = lhs(c) of the
@@ -1184,6 +1201,14 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
 }
 
 }  // namespace
+
+cudaError_t launch_rebase(const Dev& D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* rowptr, uint32_t* argptr,
+                          const AppBase* bases, cudaStream_t s) {
+  uint32_t blocks = (D.n_nodes + 255) / 256;
+  blocks = blocks == 0 ? 1u : (blocks > 148 * 8 ? 148 * 8 : blocks);
+  k_rebase<<<blocks, 256, 0, s>>>(D, nodes, nodemeth, rowptr, argptr, bases);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,
                          const uint8_t* ekind, const uint32_t* exoff, cudaStream_t s) {

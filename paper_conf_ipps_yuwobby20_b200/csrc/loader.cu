@@ -80,16 +80,20 @@ uint32_t cls_of(uint8_t k) {
 
 // Host images of every device table of a batch.
 struct HostImage {
-  std::vector<NodeRec> nodes;
+  // per-node tables are written straight into the pinned staging buffer (region A) with
+  // app-local indices; k_rebase adds the app's bases on the device
+  NodeRec* o_nodes = nullptr;
+  uint32_t* o_nodemeth = nullptr;
+  uint32_t* o_rowptr = nullptr;                // [n + 1] of this app's node n
+  uint32_t* o_argptr = nullptr;
+  uint64_t n_nodes = 0;
   std::vector<MethRec> meths;
   std::vector<ModRec> mods;
-  std::vector<uint32_t> row_ptr{0};
   // edges: the device builds the Edge / InlEdge records (k_edges) from the descriptor's col and
   // edge_kind plus the projection-table offset of each CALL/RET edge computed here
   const gdroid_icfg_desc* desc = nullptr;
   uint64_t n_edges = 0;
   std::vector<uint32_t> xo;                    // [E] app-local xmap offset | NO_XMAP
-  std::vector<uint32_t> arg_ptr{0};
   std::vector<int32_t> args;
   std::vector<uint32_t> col_gid, col_hbase;
   std::vector<int32_t> col_type;
@@ -100,7 +104,6 @@ struct HostImage {
   std::vector<int32_t> frow;                   // per (module, field): column -> global heap row | -1
   std::vector<uint32_t> app_node_base;
   std::vector<uint32_t> entries;
-  std::vector<uint32_t> node_method;
   uint64_t fact_words = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
   // per-load temporaries, kept so their pages are touched once per process (first-touch faults
@@ -233,12 +236,10 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   const uint64_t N = d->n_nodes, E = d->n_edges, M = d->n_methods, Dm = d->n_modules;
   const uint64_t I = d->n_instances, G = d->n_statics, T = d->n_types;
   if (N == 0 || M == 0 || Dm == 0 || I == 0) return set_err(GDROID_E_INVALID, "app %u: empty ICFG", k);
-  if ((uint64_t)H.nodes.size() + N >= (1ull << 32) || E >= (1ull << 32))
+  if (N >= (1ull << 32) || E >= (1ull << 32))
     return set_err(GDROID_E_LIMIT, "app %u: batch exceeds 2^32 nodes or edges", k);
-  H.nodes.reserve(H.nodes.size() + N); H.node_method.reserve(H.node_method.size() + N);
-  H.row_ptr.reserve(H.row_ptr.size() + N);
-  H.arg_ptr.reserve(H.arg_ptr.size() + N); H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
-  const uint32_t nb = (uint32_t)H.nodes.size(), mb = (uint32_t)H.meths.size();
+  H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
+  const uint32_t nb = 0, mb = (uint32_t)H.meths.size();   // app-local node / method indices
   const uint32_t db = (uint32_t)H.mods.size(), tb = (uint32_t)(H.tf_ptr.size() - 1);
   // ---- CSR (structure)
   if (d->row_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: row_ptr[0] != 0", k);
@@ -424,8 +425,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (gid < (int64_t)local_base[m] || gid >= (int64_t)local_base[m + 1]) return -1;
     return gid - (int64_t)local_base[m];
   };
-  H.nodes.resize(nb + N); H.node_method.resize(nb + N);
-  H.row_ptr.resize(nb + N + 1); H.arg_ptr.resize(nb + N + 1); H.args.resize(n_args);
+  H.n_nodes = N;
+  H.args.resize(n_args);
   FirstErr fe;
   std::mutex cls_mu;
   auto node_pass = [&](uint64_t n, uint32_t* cls_cnt) -> gdroid_status {
@@ -521,10 +522,10 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     R.e0 = (uint32_t)d->row_ptr[n]; R.e1 = (uint32_t)d->row_ptr[n + 1];
     R.col_off = md.col_off; R.grow_off = md.grow_off; R.n_cols = (uint16_t)md.n_cols;
     R.logW = (uint8_t)md.logW; R.module = db + (uint32_t)dd;
-    H.nodes[nb + n] = R;
-    H.node_method[nb + n] = mb + (uint32_t)m;
-    H.row_ptr[nb + n + 1] = (uint32_t)d->row_ptr[n + 1];
-    H.arg_ptr[nb + n + 1] = (uint32_t)a1;
+    H.o_nodes[n] = R;
+    H.o_nodemeth[n] = mb + (uint32_t)m;
+    H.o_rowptr[n + 1] = (uint32_t)d->row_ptr[n + 1];
+    H.o_argptr[n + 1] = (uint32_t)a1;
     cls_cnt[R.cls] += n_chunks_of(R.e1 - R.e0, R.cls);     // work items per GRP class
     return GDROID_OK;
   };
@@ -674,9 +675,11 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
 
 // Parts up to P_UPLOAD are staged on the host and uploaded; the edge records after it are
 // built on the device by k_edges from P_ECOL / P_EKIND / P_EXOFF.
-enum PartId { P_NODES, P_METHS, P_MODS, P_ROWPTR, P_ECOL, P_EKIND, P_EXOFF, P_ARGPTR, P_ARGS, P_COLGID,
-              P_COLTYPE, P_COLHB, P_GROWGID, P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE,
-              P_ENTRIES, P_NODEMETH, P_FROW, P_UPLOAD, P_EDGES = P_UPLOAD, P_INL, NPART };
+enum PartId { P_NODES, P_NODEMETH, P_ROWPTR, P_ARGPTR,               // region A: per node
+              P_METHS, P_MODS, P_ECOL, P_EKIND, P_EXOFF, P_ARGS, P_COLGID, P_COLTYPE, P_COLHB, P_GROWGID,
+              P_GROWCOL, P_GROWFLD, P_TFPTR, P_TF, P_XMAP, P_APPBASE, P_ENTRIES, P_FROW, P_BASES,
+              P_UPLOAD, P_EDGES = P_UPLOAD, P_INL, NPART };
+constexpr int P_REGION_B = P_METHS;
 
 // Device-table layout of a batch inside the staging buffer.
 struct Layout {
@@ -693,18 +696,21 @@ struct Layout {
 // environment first-touch page faults (~1 GB/s) dominate host-side table building otherwise.
 struct LoadCache {
   std::mutex mu;
-  void* stage = nullptr;
+  void* stage = nullptr;         // region B (all tables but the per-node ones)
   size_t cap = 0;
+  void* stage_a = nullptr;       // region A (per-node tables, written by the node pass)
+  size_t cap_a = 0;
+  bool pinned = false, pinned_a = false;
   std::vector<HostImage> img;
 };
 LoadCache g_cache;
 
 void reset_image(HostImage& h) {
-  h.nodes.clear(); h.meths.clear(); h.mods.clear(); h.xo.clear(); h.n_edges = 0; h.desc = nullptr; h.args.clear();
+  h.n_nodes = 0; h.meths.clear(); h.mods.clear(); h.xo.clear(); h.n_edges = 0; h.desc = nullptr; h.args.clear();
   h.col_gid.clear(); h.col_hbase.clear(); h.col_type.clear(); h.grow_gid.clear(); h.grow_col.clear();
   h.grow_field.clear(); h.tf.clear(); h.xmap.clear(); h.frow.clear(); h.app_node_base.clear();
-  h.entries.clear(); h.node_method.clear();
-  h.row_ptr.assign(1, 0); h.arg_ptr.assign(1, 0); h.tf_ptr.assign(1, 0);
+  h.entries.clear();
+  h.tf_ptr.assign(1, 0);
   h.fact_words = 0;
   for (auto& c : h.cls_count) c = 0;
 }
@@ -713,13 +719,57 @@ size_t align256(size_t x);
 
 // Build every app's image (in parallel, app-local indices) and write the rebased batch tables
 // straight into the pinned staging buffer.  Caller holds g_cache.mu.
-gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout& Lo) {
+// Pinned staging buffer of at least `need` bytes.  Without a usable device (CPU-only hosts run
+// the validation tests) it falls back to pageable memory; the upload then fails with the CUDA
+// error after validation has reported any input error.
+gdroid_status ensure_pinned(void*& buf, size_t& cap, bool& pinned, size_t need, const char* what) {
+  if (cap >= need) return GDROID_OK;
+  if (buf) { if (pinned) cudaFreeHost(buf); else std::free(buf); }
+  buf = nullptr;
+  cap = 0;
+  const size_t want = need + (need >> 2);
+  pinned = cudaMallocHost(&buf, want) == cudaSuccess;
+  if (!pinned) {
+    cudaGetLastError();
+    buf = std::malloc(want);
+    if (!buf) return set_err(GDROID_E_OOM, "staging %s (%zu B)", what, need);
+  }
+  cap = want;
+  return GDROID_OK;
+}
+
+// Region A of the device tables (per-node parts) for a batch of N nodes.
+size_t region_a_layout(uint64_t N, Layout& Lo) {
+  const size_t bytes[P_REGION_B] = {N * sizeof(NodeRec), N * 4, (N + 1) * 4, (N + 1) * 4};
+  size_t t = 0;
+  for (int p = 0; p < P_REGION_B; ++p) { Lo.off[p] = t; t += align256(bytes[p]); }
+  return t;
+}
+
+// upload_a(Lo): called once region A is complete and the full layout is known (before region B
+// is written), so its H2D overlaps the rest of the host work.
+gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout& Lo,
+                          const std::function<gdroid_status(const Layout&)>& upload_a) {
   if (g_cache.img.size() < n_apps) g_cache.img.resize(n_apps);
   std::vector<HostImage>& img = g_cache.img;
   std::vector<gdroid_status> st(n_apps, GDROID_OK);
   std::vector<std::string> err(n_apps);
+  std::vector<uint64_t> nbase(n_apps + 1, 0);
+  for (uint32_t k = 0; k < n_apps; ++k) nbase[k + 1] = nbase[k] + descs[k].n_nodes;
+  if (nbase[n_apps] >= (1ull << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
+  const size_t a_bytes = region_a_layout(nbase[n_apps], Lo);
+  gdroid_status sa = ensure_pinned(g_cache.stage_a, g_cache.cap_a, g_cache.pinned_a, a_bytes, "A");
+  if (sa != GDROID_OK) return sa;
+  char* SA = (char*)g_cache.stage_a;
+  NodeRec* a_nodes = (NodeRec*)(SA + Lo.off[P_NODES]);
+  uint32_t* a_nodemeth = (uint32_t*)(SA + Lo.off[P_NODEMETH]);
+  uint32_t* a_rowptr = (uint32_t*)(SA + Lo.off[P_ROWPTR]);
+  uint32_t* a_argptr = (uint32_t*)(SA + Lo.off[P_ARGPTR]);
+  a_rowptr[0] = 0; a_argptr[0] = 0;
   parallel_for(n_apps, [&](uint32_t k) {                   // apps in parallel, and node ranges inside
     reset_image(img[k]);
+    img[k].o_nodes = a_nodes + nbase[k]; img[k].o_nodemeth = a_nodemeth + nbase[k];
+    img[k].o_rowptr = a_rowptr + nbase[k]; img[k].o_argptr = a_argptr + nbase[k];
     st[k] = add_app(img[k], &descs[k], k);
     if (st[k] != GDROID_OK) err[k] = g_err;
   });
@@ -731,7 +781,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   b[0] = Base{};
   for (uint32_t k = 0; k < n_apps; ++k) {
     const HostImage& h = img[k];
-    b[k + 1] = Base{b[k].node + h.nodes.size(), b[k].edge + h.n_edges, b[k].meth + h.meths.size(),
+    b[k + 1] = Base{b[k].node + h.n_nodes, b[k].edge + h.n_edges, b[k].meth + h.meths.size(),
                     b[k].mod + h.mods.size(), b[k].col + h.col_gid.size(), b[k].grow + h.grow_gid.size(),
                     b[k].type + (h.tf_ptr.size() - 1), b[k].tf + h.tf.size(), b[k].xmap + h.xmap.size(),
                     b[k].frow + h.frow.size(), b[k].args + h.args.size(), b[k].fact + h.fact_words,
@@ -750,37 +800,30 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   Lo.app_base.resize(n_apps + 1);
   for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
   const size_t bytes[NPART] = {
-      T.node * sizeof(NodeRec), T.meth * sizeof(MethRec), T.mod * sizeof(ModRec), (T.node + 1) * 4,
+      0, 0, 0, 0,                                            // region A (laid out above)
+      T.meth * sizeof(MethRec), T.mod * sizeof(ModRec),
       std::max<uint64_t>(T.edge, 1) * 4, std::max<uint64_t>(T.edge, 1), std::max<uint64_t>(T.edge, 1) * 4,
-      (T.node + 1) * 4, std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4,
-      T.col * 4, T.grow * 4, T.grow * 4, T.grow * 4, (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4,
-      std::max<uint64_t>(T.xmap, 1) * 4, (n_apps + 1) * 4, std::max<uint64_t>(T.ent, 1) * 4, T.node * 4,
-      std::max<uint64_t>(T.frow, 1) * 4, std::max<uint64_t>(T.edge, 1) * sizeof(Edge),
-      T.node * 4 * sizeof(InlEdge)};
-  Lo.total = 0;
-  for (int p = 0; p < NPART; ++p) {
+      std::max<uint64_t>(T.args, 1) * 4, T.col * 4, T.col * 4, T.col * 4, T.grow * 4, T.grow * 4, T.grow * 4,
+      (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4, std::max<uint64_t>(T.xmap, 1) * 4, (n_apps + 1) * 4,
+      std::max<uint64_t>(T.ent, 1) * 4, std::max<uint64_t>(T.frow, 1) * 4, n_apps * sizeof(AppBase),
+      std::max<uint64_t>(T.edge, 1) * sizeof(Edge), T.node * 4 * sizeof(InlEdge)};
+  Lo.total = a_bytes;
+  for (int p = P_REGION_B; p < NPART; ++p) {
     if (p == P_UPLOAD) Lo.upload = Lo.total;
     Lo.off[p] = Lo.total;
     Lo.total += align256(bytes[p]);
   }
-  if (g_cache.cap < Lo.upload) {
-    if (g_cache.stage) cudaFreeHost(g_cache.stage);
-    g_cache.stage = nullptr;
-    g_cache.cap = 0;
-    cudaError_t e = cudaMallocHost(&g_cache.stage, Lo.upload + (Lo.upload >> 2));
-    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "pinned staging (%zu B): %s", Lo.upload, cudaGetErrorString(e));
-    g_cache.cap = Lo.upload + (Lo.upload >> 2);
-  }
-  char* S = (char*)g_cache.stage;
+  sa = upload_a(Lo);
+  if (sa != GDROID_OK) return sa;
+  sa = ensure_pinned(g_cache.stage, g_cache.cap, g_cache.pinned, Lo.upload - a_bytes, "B");
+  if (sa != GDROID_OK) return sa;
+  char* S = (char*)g_cache.stage - a_bytes;                  // region B starts at device offset a_bytes
   auto P = [&](int p) { return S + Lo.off[p]; };
-  NodeRec* g_nodes = (NodeRec*)P(P_NODES);
   MethRec* g_meths = (MethRec*)P(P_METHS);
   ModRec* g_mods = (ModRec*)P(P_MODS);
-  uint32_t* g_rowptr = (uint32_t*)P(P_ROWPTR);
   uint32_t* g_ecol = (uint32_t*)P(P_ECOL);
   uint8_t* g_ekind = (uint8_t*)P(P_EKIND);
   uint32_t* g_exoff = (uint32_t*)P(P_EXOFF);
-  uint32_t* g_argptr = (uint32_t*)P(P_ARGPTR);
   int32_t* g_args = (int32_t*)P(P_ARGS);
   uint32_t* g_colgid = (uint32_t*)P(P_COLGID);
   int32_t* g_coltype = (int32_t*)P(P_COLTYPE);
@@ -793,9 +836,12 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   int32_t* g_xmap = (int32_t*)P(P_XMAP);
   uint32_t* g_appbase = (uint32_t*)P(P_APPBASE);
   uint32_t* g_entries = (uint32_t*)P(P_ENTRIES);
-  uint32_t* g_nodemeth = (uint32_t*)P(P_NODEMETH);
   int32_t* g_frow = (int32_t*)P(P_FROW);
-  g_rowptr[0] = 0; g_argptr[0] = 0; g_tfptr[0] = 0;
+  AppBase* g_bases = (AppBase*)P(P_BASES);
+  for (uint32_t k = 0; k < n_apps; ++k)
+    g_bases[k] = AppBase{b[k].fact, (uint32_t)b[k].edge, (uint32_t)b[k].meth, (uint32_t)b[k].mod, (uint32_t)b[k].col,
+                         (uint32_t)b[k].grow, (uint32_t)b[k].frow, (uint32_t)b[k].args, 0u};
+  g_tfptr[0] = 0;
   g_args[0] = -1; g_tf[0] = 0; g_xmap[0] = -1; g_entries[0] = 0; g_frow[0] = -1;   // non-empty
   for (uint32_t k = 0; k <= n_apps; ++k) g_appbase[k] = (uint32_t)b[k].node;
   // work units: (app, slice of its nodes / edges) so one big app does not serialise the copy
@@ -804,7 +850,6 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   std::vector<Unit> units;
   for (uint32_t k = 0; k < n_apps; ++k) {
     const HostImage& h = img[k];
-    for (size_t lo = 0; lo < h.nodes.size(); lo += SLICE) units.push_back({k, 0, lo, std::min(h.nodes.size(), lo + SLICE)});
     for (size_t lo = 0; lo < h.n_edges; lo += SLICE) units.push_back({k, 1, lo, std::min<size_t>(h.n_edges, lo + SLICE)});
     units.push_back({k, 2, 0, 0});
   }
@@ -812,19 +857,6 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
     const Unit U = units[u];
     const HostImage& h = img[U.k];
     const Base& B = b[U.k];
-    if (U.kind == 0) {
-      for (size_t i = U.lo; i < U.hi; ++i) {
-        NodeRec R = h.nodes[i];
-        R.off += B.fact; R.e0 += (uint32_t)B.edge; R.e1 += (uint32_t)B.edge;
-        R.col_off += (uint32_t)B.col; R.grow_off += (uint32_t)B.grow; R.module += (uint32_t)B.mod;
-        if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)B.frow;
-        g_nodes[B.node + i] = R;
-        g_nodemeth[B.node + i] = h.node_method[i] + (uint32_t)B.meth;
-        g_rowptr[B.node + i + 1] = h.row_ptr[i + 1] + (uint32_t)B.edge;
-        g_argptr[B.node + i + 1] = h.arg_ptr[i + 1] + (uint32_t)B.args;
-      }
-      return;
-    }
     if (U.kind == 1) {
       for (size_t i = U.lo; i < U.hi; ++i) {
         const uint32_t x = h.xo[i];
@@ -1128,12 +1160,19 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   auto t0 = std::chrono::steady_clock::now();
   {
     std::lock_guard<std::mutex> lock(g_cache.mu);
-    gdroid_status st = build_image(descs, n_apps, Lo);
-    if (st != GDROID_OK) return fail(st);
+    gdroid_status st = build_image(descs, n_apps, Lo, [&](const Layout& L) -> gdroid_status {
+      cudaError_t e = cudaMallocAsync(&a->d_tables, L.total, a->stream);
+      if (e != cudaSuccess) return set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", L.total, cudaGetErrorString(e));
+      e = cudaMemcpyAsync(a->d_tables, g_cache.stage_a, L.off[P_REGION_B], cudaMemcpyHostToDevice, a->stream);
+      return e == cudaSuccess ? GDROID_OK : set_err(GDROID_E_CUDA, "H2D upload (A): %s", cudaGetErrorString(e));
+    });
+    if (st != GDROID_OK) {
+      if (a->d_tables) cudaStreamSynchronize(a->stream);
+      return fail(st);
+    }
     t0 = std::chrono::steady_clock::now();
-    cudaError_t e = cudaMallocAsync(&a->d_tables, Lo.total, a->stream);
-    if (e != cudaSuccess) return fail(set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", Lo.total, cudaGetErrorString(e)));
-    e = cudaMemcpyAsync(a->d_tables, g_cache.stage, Lo.upload, cudaMemcpyHostToDevice, a->stream);
+    cudaError_t e = cudaMemcpyAsync((char*)a->d_tables + Lo.off[P_REGION_B], g_cache.stage, Lo.upload - Lo.off[P_REGION_B],
+                                    cudaMemcpyHostToDevice, a->stream);
     cudaError_t e2 = cudaStreamSynchronize(a->stream);
     if (e != cudaSuccess || e2 != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "H2D upload: %s", cudaGetErrorString(e != cudaSuccess ? e : e2)));
   }
@@ -1173,9 +1212,14 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.n_words = Lo.fact_words;
   D.wide = Lo.wide;
   {
-    // (a1) edge records and inline chunk-0 edges, derived on the device from col / edge_kind /
-    // projection offsets and the uploaded NodeRecs (stream-ordered after the upload)
-    cudaError_t e = launch_edges(D, (Edge*)(T + Lo.off[P_EDGES]), (InlEdge*)(T + Lo.off[P_INL]),
+    // (a1) per-app bases added to the staged app-local node tables, then the edge records and
+    // inline chunk-0 edges derived from col / edge_kind / projection offsets and the NodeRecs
+    // (stream-ordered after the upload)
+    cudaError_t e = launch_rebase(D, (NodeRec*)(T + Lo.off[P_NODES]), (uint32_t*)(T + Lo.off[P_NODEMETH]),
+                                  (uint32_t*)(T + Lo.off[P_ROWPTR]), (uint32_t*)(T + Lo.off[P_ARGPTR]),
+                                  (const AppBase*)(T + Lo.off[P_BASES]), a->stream);
+    if (e != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "k_rebase: %s", cudaGetErrorString(e)));
+    e = launch_edges(D, (Edge*)(T + Lo.off[P_EDGES]), (InlEdge*)(T + Lo.off[P_INL]),
                                  (NodeRec*)(T + Lo.off[P_NODES]), (const uint32_t*)(T + Lo.off[P_ECOL]),
                                  (const uint8_t*)(T + Lo.off[P_EKIND]), (const uint32_t*)(T + Lo.off[P_EXOFF]),
                                  a->stream);
