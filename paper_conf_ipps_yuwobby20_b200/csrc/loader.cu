@@ -766,6 +766,9 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   uint32_t* a_rowptr = (uint32_t*)(SA + Lo.off[P_ROWPTR]);
   uint32_t* a_argptr = (uint32_t*)(SA + Lo.off[P_ARGPTR]);
   a_rowptr[0] = 0; a_argptr[0] = 0;
+  PHASE("staging A");
+  PhaseTimer* pt_saved = g_pt;
+  if (n_apps > 1) g_pt = nullptr;                           // per-app phases only for single apps
   parallel_for(n_apps, [&](uint32_t k) {                   // apps in parallel, and node ranges inside
     reset_image(img[k]);
     img[k].o_nodes = a_nodes + nbase[k]; img[k].o_nodemeth = a_nodemeth + nbase[k];
@@ -773,6 +776,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
     st[k] = add_app(img[k], &descs[k], k);
     if (st[k] != GDROID_OK) err[k] = g_err;
   });
+  g_pt = pt_saved;
   for (uint32_t k = 0; k < n_apps; ++k)
     if (st[k] != GDROID_OK) { g_err = err[k]; return st[k]; }
   PHASE("apps (parallel)");
@@ -1252,6 +1256,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
   a->max_blocks = fixpoint_max_blocks(device, D.wide);
+  PHASE("device state + k_rebase/k_edges");
   *out = a;
   return GDROID_OK;
 }
