@@ -211,6 +211,9 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # ranks on one host share its cores: the library's loader pool gets an equal share
+    per_host = int(os.environ.get("LOCAL_WORLD_SIZE", "1"))
+    os.environ.setdefault("GDROID_HOST_THREADS", str(max(1, len(os.sched_getaffinity(0)) // max(1, per_host))))
     assert torch.cuda.is_available(), "bench needs a GPU"
     torch.cuda.set_device(local)
     if world > 1:

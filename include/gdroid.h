@@ -140,7 +140,11 @@ gdroid_status gdroid_load_icfg(const gdroid_icfg_desc* desc, int device, void* c
                                gdroid_app** out);
 /* Load n_apps independent apps into ONE handle; they share every device round
  * (IDFG-instance batching).  Node ids, slot gids and digests stay
- * per app. */
+ * per app.  Host side: the apps are validated and laid out in parallel on a worker
+ * pool of min(hardware threads, $GDROID_HOST_THREADS) threads; the call returns once
+ * the tables are on the device (stream-ordered kernels k_rebase / k_edges finish the
+ * layout before any later work on cuda_stream).  The descriptor arrays are only read
+ * during the call. */
 gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, int device,
                                 void* cuda_stream, gdroid_app** out);
 /* Load ONE app for every variant including GDROID_V_PLAIN: the MAT handle of

@@ -153,7 +153,12 @@ class Pool {
 
  private:
   Pool() {
-    const uint32_t T = std::max(1u, std::thread::hardware_concurrency());
+    // GDROID_HOST_THREADS caps the pool (several ranks per host share its cores)
+    uint32_t T = std::max(1u, std::thread::hardware_concurrency());
+    if (const char* e = getenv("GDROID_HOST_THREADS")) {
+      const long v = strtol(e, nullptr, 10);
+      if (v > 0) T = std::min<uint32_t>(T, (uint32_t)v);
+    }
     for (uint32_t t = 1; t < T; ++t) workers_.emplace_back([this] { loop(); });
   }
   ~Pool() {
