@@ -13,6 +13,7 @@ constexpr int NCLS = 5;            // GRP classes + 2 interpr
 enum Cls : uint8_t { C_ONETIME = 0, C_SINGLE = 1, C_DOUBLE = 2, C_CALL = 3, C_EXIT = 4 };
 constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]; slot CNT_NODES = nodes queued
 constexpr int CNT_NODES = 5;
+constexpr uint32_t HIOCC_NODES = 1u << 20;   // batches this large are item-throughput bound
 #ifndef GD_THREADS
 #define GD_THREADS 256
 #endif
@@ -180,6 +181,7 @@ struct Dev {
   uint32_t max_rounds;
   uint32_t wide;                // max log2(words per row) over the batch's modules: 0 = all narrow,
                                 // >= 1: some module has > 64 instances (row-occupancy path)
+  uint32_t hiocc;               // 1: narrow batch of >= HIOCC_NODES nodes, 4-CTA/SM instantiation
   uint32_t flags;               // F_* scheduling switches of the build (ablation variants)
   uint32_t count;               // 1: evaluate the byte models (alg/dense bytes, atomics) on the device
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}
@@ -233,6 +235,6 @@ cudaError_t launch_digest(const Dev& D, cudaStream_t s);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,
                           uint64_t* pairs, cudaStream_t s);
-int fixpoint_max_blocks(int device, uint32_t wide);
+int fixpoint_max_blocks(int device, uint32_t wide, uint32_t hiocc);
 
 }  // namespace gd

@@ -24,6 +24,9 @@ namespace {
 #ifndef GD_MINB
 #define GD_MINB 3              // resident CTAs per SM the fixed-point kernels are compiled for
 #endif
+#ifndef GD_MINB_HI
+#define GD_MINB_HI 4           // ... for large narrow batches (Dev::hiocc)
+#endif
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int KW = 4;          // words per lane per chunk of a fact block (loads issued together)
@@ -42,6 +45,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #endif
 #ifndef GD_PRE
 #define GD_PRE 1               // inline path: load IN(dst) of the first two edges with IN(src)
+#endif
+#ifndef GD_PRE2
+#define GD_PRE2 1              // ... and of the second edge
 #endif
 #ifndef GD_CONT_DENSE
 #define GD_CONT_DENSE 0        // continue into narrow (one word per row) destinations too (light rounds)
@@ -507,7 +513,7 @@ __device__ __forceinline__ void process_inline(const Dev& D, CtaStage& st, const
     y[k] = w < B ? X[w] : 0ull;
     if (GD_PRE) {                                           // IN(dst) of edges 0 and 1, same hop
       p0[k] = w < B ? D.facts[off0 + w] : 0ull;
-      p1[k] = (ne > 1 && w < B) ? D.facts[off1 + w] : 0ull;
+      if (GD_PRE2) p1[k] = (ne > 1 && w < B) ? D.facts[off1 + w] : 0ull;
     }
   }
   const uint32_t my_stamp = lane < (int)ne ? D.stamp[me.dst] : 1u;
@@ -583,7 +589,7 @@ __device__ __forceinline__ void process_inline(const Dev& D, CtaStage& st, const
       const uint32_t w = lane + 32 * k;
       const bool keep = y[k] && (int)w != kill;
       if (GD_PRE && i == 0) cur[k] = keep ? p0[k] : ~0ull;
-      else if (GD_PRE && i == 1) cur[k] = keep ? p1[k] : ~0ull;
+      else if (GD_PRE && GD_PRE2 && i == 1) cur[k] = keep ? p1[k] : ~0ull;
       else cur[k] = keep ? Z[w] : ~0ull;
     }
     bool g = false;
@@ -1008,8 +1014,8 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   return total;
 }
 
-template <bool WIDE, bool CNT, int MW>
-__global__ void __launch_bounds__(THREADS, GD_MINB) k_fixpoint(Dev D) {
+template <bool WIDE, bool CNT, int MW, int MINB>
+__global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   __shared__ WarpScratch ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
   __shared__ CtaStage st;
@@ -1225,22 +1231,25 @@ cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
 
 // Instantiations: narrow batches (WIDE = false) and wide batches by the widest row of the
 // batch (MW = 2, 4, 8 words: register arrays sized to it), each with and without the
-// byte-model counters (CNT).
+// byte-model counters (CNT).  Large narrow batches (Dev::hiocc) use a 4-CTA/SM build (64
+// registers): their big rounds are item-throughput bound and gain from the extra warps, while
+// small batches are round-latency bound and lose to its spills.
 template <bool CNT>
-static const void* fixpoint_fn(uint32_t wide) {
+static const void* fixpoint_fn(uint32_t wide, uint32_t hiocc) {
   switch (wide) {
-    case 0: return (const void*)k_fixpoint<false, CNT, 1>;
-    case 1: return (const void*)k_fixpoint<true, CNT, 2>;
-    case 2: return (const void*)k_fixpoint<true, CNT, 4>;
-    default: return (const void*)k_fixpoint<true, CNT, 8>;
+    case 0: return hiocc ? (const void*)k_fixpoint<false, CNT, 1, GD_MINB_HI>
+                         : (const void*)k_fixpoint<false, CNT, 1, GD_MINB>;
+    case 1: return (const void*)k_fixpoint<true, CNT, 2, GD_MINB>;
+    case 2: return (const void*)k_fixpoint<true, CNT, 4, GD_MINB>;
+    default: return (const void*)k_fixpoint<true, CNT, 8, GD_MINB>;
   }
 }
 
-int fixpoint_max_blocks(int device, uint32_t wide) {
+int fixpoint_max_blocks(int device, uint32_t wide, uint32_t hiocc) {
   int sms = 0, occ = 0, occ2 = 0;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fixpoint_fn<true>(wide), THREADS, 0);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, fixpoint_fn<false>(wide), THREADS, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fixpoint_fn<true>(wide, hiocc), THREADS, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, fixpoint_fn<false>(wide, hiocc), THREADS, 0);
   occ = occ2 < occ ? occ2 : occ;          // one grid size serves both instantiations
   return sms * (occ > 0 ? occ : 1);
 }
@@ -1248,7 +1257,7 @@ int fixpoint_max_blocks(int device, uint32_t wide) {
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s) {
   Dev d = D;
   void* args[] = {&d};
-  const void* f = D.count ? fixpoint_fn<true>(D.wide) : fixpoint_fn<false>(D.wide);
+  const void* f = D.count ? fixpoint_fn<true>(D.wide, D.hiocc) : fixpoint_fn<false>(D.wide, D.hiocc);
   return cudaLaunchCooperativeKernel(f, dim3(blocks), dim3(THREADS), args, 0, s);
 }
 

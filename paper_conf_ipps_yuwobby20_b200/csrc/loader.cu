@@ -1260,7 +1260,8 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     for (auto& ev : a->ev)
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
-  a->max_blocks = fixpoint_max_blocks(device, D.wide);
+  D.hiocc = (D.wide == 0 && N >= HIOCC_NODES) ? 1u : 0u;
+  a->max_blocks = fixpoint_max_blocks(device, D.wide, D.hiocc);
   PHASE("device state + k_rebase/k_edges");
   *out = a;
   return GDROID_OK;
