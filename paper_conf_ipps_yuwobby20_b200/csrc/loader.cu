@@ -15,6 +15,8 @@
 #include <condition_variable>
 #include <functional>
 #include <map>
+#include <memory>
+#include <new>
 #include <mutex>
 #include <thread>
 #include <unordered_map>
@@ -78,6 +80,15 @@ uint32_t cls_of(uint8_t k) {
   }
 }
 
+// Allocator whose resize() leaves new elements uninitialised (large tables are filled in parallel).
+template <class T>
+struct NoInit : std::allocator<T> {
+  template <class U> struct rebind { using other = NoInit<U>; };
+  template <class U, class... A> void construct(U* p, A&&... a) {
+    if constexpr (sizeof...(A) == 0) ::new ((void*)p) U; else ::new ((void*)p) U(std::forward<A>(a)...);
+  }
+};
+
 // Host images of every device table of a batch.
 struct HostImage {
   // per-node tables are written straight into the pinned staging buffer (region A) with
@@ -93,14 +104,14 @@ struct HostImage {
   // edge_kind plus the projection-table offset of each CALL/RET edge computed here
   const gdroid_icfg_desc* desc = nullptr;
   uint64_t n_edges = 0;
-  std::vector<uint32_t> xo;                    // [E] app-local xmap offset | NO_XMAP
+  std::vector<uint32_t, NoInit<uint32_t>> xo; // [E] app-local xmap offset | NO_XMAP (all written)
   std::vector<int32_t> args;
   std::vector<uint32_t> col_gid, col_hbase;
   std::vector<int32_t> col_type;
   std::vector<uint32_t> grow_gid;
   std::vector<int32_t> grow_col, grow_field;
   std::vector<uint32_t> tf_ptr{0}, tf;
-  std::vector<int32_t> xmap;                   // projection tables: colmap then rowmap
+  std::vector<int32_t, NoInit<int32_t>> xmap;  // projection tables: colmap then rowmap (filled in parallel)
   std::vector<int32_t> frow;                   // per (module, field): column -> global heap row | -1
   std::vector<uint32_t> app_node_base;
   std::vector<uint32_t> entries;
@@ -108,7 +119,10 @@ struct HostImage {
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
   // per-load temporaries, kept so their pages are touched once per process (first-touch faults
   // cost more than the table build itself in this environment)
-  std::vector<uint64_t> t_heap_base, t_local_base, t_foff;
+  std::vector<uint64_t> t_heap_base, t_local_base, t_msize;
+  std::vector<uint64_t, NoInit<uint64_t>> t_foff;             // every entry written by the size pass
+  std::vector<uint8_t> t_kmark, t_pmark;
+  std::vector<uint32_t> t_kidx, t_pidx;
 };
 
 // Per-module host-side lookup info of the app being loaded.
@@ -234,6 +248,24 @@ struct FirstErr {
   }
 };
 
+// Call f(i) for every non-zero byte of a (sparse) mark table, in index order.
+template <class F>
+void scan_marks(const std::vector<uint8_t>& mark, F f) {
+  const uint64_t n = mark.size();
+  uint64_t i = 0;
+  for (; i + 8 <= n; i += 8) {
+    uint64_t w;
+    std::memcpy(&w, mark.data() + i, 8);
+    while (w) {
+      const int b = __builtin_ctzll(w) >> 3;
+      f(i + b);
+      w &= ~(0xffull << (8 * b));
+    }
+  }
+  for (; i < n; ++i)
+    if (mark[i]) f(i);
+}
+
 gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   if (!d) return set_err(GDROID_E_INVALID, "app %u: NULL descriptor", k);
   if (d->abi_version != GDROID_ABI_VERSION)
@@ -302,54 +334,83 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   const uint64_t Lt = local_base[M];
   if (Lt + G + heap_base[I] >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: more than 2^32 slots", k);
   PHASE("methods");
-  // ---- modules: pools, rows, columns
+  // ---- modules: pools, rows, columns (validated and sized in parallel, prefix, filled in parallel)
   std::vector<ModInfo> mi(Dm);
-  for (uint64_t dd = 0; dd < Dm; ++dd) {
-    const uint64_t a = d->module_inst_ptr[dd], b = d->module_inst_ptr[dd + 1];
-    const uint64_t sa = d->module_static_ptr[dd], sb = d->module_static_ptr[dd + 1];
-    if (b < a || sb < sa) return set_err(GDROID_E_INVALID, "app %u: module %llu pool CSR not monotone", k, (unsigned long long)dd);
-    if (b == a || d->module_insts[a] != 0) return set_err(GDROID_E_POOL, "app %u: module %llu pool lacks NULL", k, (unsigned long long)dd);
-    for (uint64_t q = a; q < b; ++q) {
-      if (d->module_insts[q] >= I) return set_err(GDROID_E_INVALID, "app %u: module %llu instance out of range", k, (unsigned long long)dd);
-      if (q > a && d->module_insts[q] <= d->module_insts[q - 1]) return set_err(GDROID_E_INVALID, "app %u: module %llu pool not strictly ascending", k, (unsigned long long)dd);
-    }
-    for (uint64_t q = sa; q < sb; ++q) {
-      if (d->module_statics[q] >= G) return set_err(GDROID_E_INVALID, "app %u: module %llu static out of range", k, (unsigned long long)dd);
-      if (q > sa && d->module_statics[q] <= d->module_statics[q - 1]) return set_err(GDROID_E_INVALID, "app %u: module %llu statics not strictly ascending", k, (unsigned long long)dd);
-    }
-    const uint64_t ncol = b - a;
-    if (ncol > 64ull * MAXW) return set_err(GDROID_E_LIMIT, "app %u: module %llu pool has %llu > %d instances", k, (unsigned long long)dd, (unsigned long long)ncol, 64 * MAXW);
-    uint32_t W = 1, logW = 0;
-    while (64ull * W < ncol) { W <<= 1; ++logW; }
-    ModRec md{};
-    md.n_cols = (uint32_t)ncol; md.W = W; md.logW = logW;
-    md.n_stat = (uint32_t)(sb - sa);
-    md.col_off = (uint32_t)H.col_gid.size();
-    md.grow_off = (uint32_t)H.grow_gid.size();
-    for (uint64_t q = sa; q < sb; ++q) {                       // static rows
-      H.grow_gid.push_back((uint32_t)(Lt + d->module_statics[q]));
-      H.grow_col.push_back(-1); H.grow_field.push_back(-1);
-    }
-    uint32_t hrow = md.n_stat;
-    for (uint64_t c = 0; c < ncol; ++c) {                      // columns + heap rows
-      const uint32_t o = d->module_insts[a + c];
-      const int32_t t = d->inst_type[o];
-      H.col_gid.push_back(o);
-      H.col_type.push_back(t < 0 ? -1 : (int32_t)(tb + t));
-      H.col_hbase.push_back(hrow);
-      if (t >= 0) {
-        for (uint64_t q = d->type_field_ptr[t]; q < d->type_field_ptr[t + 1]; ++q) {
-          H.grow_gid.push_back((uint32_t)(Lt + G + heap_base[o] + (q - d->type_field_ptr[t])));
-          H.grow_col.push_back((int32_t)c);
-          H.grow_field.push_back((int32_t)d->type_fields[q]);
-          ++hrow;
+  std::vector<uint64_t>& msz = H.t_msize;                     // per module: cols, heap rows
+  msz.assign(2 * Dm + 2, 0);
+  {
+    FirstErr fm;
+    parallel_ranges(Dm, 64, [&](uint64_t lo, uint64_t hi) {
+      for (uint64_t dd = lo; dd < hi; ++dd) {
+        const uint64_t a = d->module_inst_ptr[dd], b = d->module_inst_ptr[dd + 1];
+        const uint64_t sa = d->module_static_ptr[dd], sb = d->module_static_ptr[dd + 1];
+        if (b < a || sb < sa) { fm.offer(dd, set_err(GDROID_E_INVALID, "app %u: module %llu pool CSR not monotone", k, (unsigned long long)dd)); return; }
+        if (b == a || d->module_insts[a] != 0) { fm.offer(dd, set_err(GDROID_E_POOL, "app %u: module %llu pool lacks NULL", k, (unsigned long long)dd)); return; }
+        uint64_t nheap = 0;
+        for (uint64_t q = a; q < b; ++q) {
+          if (d->module_insts[q] >= I) { fm.offer(dd, set_err(GDROID_E_INVALID, "app %u: module %llu instance out of range", k, (unsigned long long)dd)); return; }
+          if (q > a && d->module_insts[q] <= d->module_insts[q - 1]) { fm.offer(dd, set_err(GDROID_E_INVALID, "app %u: module %llu pool not strictly ascending", k, (unsigned long long)dd)); return; }
+          const int32_t t = d->inst_type[d->module_insts[q]];
+          if (t >= 0) nheap += d->type_field_ptr[t + 1] - d->type_field_ptr[t];
+        }
+        for (uint64_t q = sa; q < sb; ++q) {
+          if (d->module_statics[q] >= G) { fm.offer(dd, set_err(GDROID_E_INVALID, "app %u: module %llu static out of range", k, (unsigned long long)dd)); return; }
+          if (q > sa && d->module_statics[q] <= d->module_statics[q - 1]) { fm.offer(dd, set_err(GDROID_E_INVALID, "app %u: module %llu statics not strictly ascending", k, (unsigned long long)dd)); return; }
+        }
+        if (b - a > 64ull * MAXW) { fm.offer(dd, set_err(GDROID_E_LIMIT, "app %u: module %llu pool has %llu > %d instances", k, (unsigned long long)dd, (unsigned long long)(b - a), 64 * MAXW)); return; }
+        msz[2 * dd + 2] = b - a;                                // prefixed below
+        msz[2 * dd + 3] = (sb - sa) + nheap;
+      }
+    });
+    if (fm.st != GDROID_OK) return fm.result();
+  }
+  for (uint64_t dd = 0; dd < Dm; ++dd) {                        // prefix: column / global-row offsets
+    msz[2 * dd + 2] += msz[2 * dd];
+    msz[2 * dd + 3] += msz[2 * dd + 1];
+  }
+  const size_t col0 = H.col_gid.size(), grow0 = H.grow_gid.size();
+  H.col_gid.resize(col0 + msz[2 * Dm]); H.col_type.resize(col0 + msz[2 * Dm]); H.col_hbase.resize(col0 + msz[2 * Dm]);
+  H.grow_gid.resize(grow0 + msz[2 * Dm + 1]); H.grow_col.resize(grow0 + msz[2 * Dm + 1]);
+  H.grow_field.resize(grow0 + msz[2 * Dm + 1]);
+  H.mods.resize(db + Dm);
+  parallel_ranges(Dm, 64, [&](uint64_t lo, uint64_t hi) {
+    for (uint64_t dd = lo; dd < hi; ++dd) {
+      const uint64_t a = d->module_inst_ptr[dd], b = d->module_inst_ptr[dd + 1];
+      const uint64_t sa = d->module_static_ptr[dd], sb = d->module_static_ptr[dd + 1];
+      const uint64_t ncol = b - a;
+      uint32_t W = 1, logW = 0;
+      while (64ull * W < ncol) { W <<= 1; ++logW; }
+      ModRec md{};
+      md.n_cols = (uint32_t)ncol; md.W = W; md.logW = logW;
+      md.n_stat = (uint32_t)(sb - sa);
+      md.col_off = (uint32_t)(col0 + msz[2 * dd]);
+      md.grow_off = (uint32_t)(grow0 + msz[2 * dd + 1]);
+      uint32_t g = md.grow_off;
+      for (uint64_t q = sa; q < sb; ++q, ++g) {                // static rows
+        H.grow_gid[g] = (uint32_t)(Lt + d->module_statics[q]);
+        H.grow_col[g] = -1; H.grow_field[g] = -1;
+      }
+      uint32_t hrow = md.n_stat;
+      for (uint64_t c = 0; c < ncol; ++c) {                    // columns + heap rows
+        const uint32_t o = d->module_insts[a + c];
+        const int32_t t = d->inst_type[o];
+        H.col_gid[md.col_off + c] = o;
+        H.col_type[md.col_off + c] = t < 0 ? -1 : (int32_t)(tb + t);
+        H.col_hbase[md.col_off + c] = hrow;
+        if (t >= 0) {
+          for (uint64_t q = d->type_field_ptr[t]; q < d->type_field_ptr[t + 1]; ++q, ++g) {
+            H.grow_gid[g] = (uint32_t)(Lt + G + heap_base[o] + (q - d->type_field_ptr[t]));
+            H.grow_col[g] = (int32_t)c;
+            H.grow_field[g] = (int32_t)d->type_fields[q];
+            ++hrow;
+          }
         }
       }
+      md.n_glob = hrow;
+      H.mods[db + dd] = md;
+      mi[dd] = ModInfo{d->module_insts + a, ncol, d->module_statics + sa, sb - sa, db + (uint32_t)dd};
     }
-    md.n_glob = hrow;
-    H.mods.push_back(md);
-    mi[dd] = ModInfo{d->module_insts + a, ncol, d->module_statics + sa, sb - sa, db + (uint32_t)dd};
-  }
+  });
   for (uint64_t m = 0; m < M; ++m)
     H.meths.push_back(MethRec{d->method_n_locals[m], d->method_n_params[m], db + d->method_module[m], (uint32_t)local_base[m]});
   PHASE("modules");
@@ -359,10 +420,17 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   // per range: call_arg_ptr monotone, fact-block sizes, (module, field) keys of heap accesses
   constexpr uint64_t RG = 1 << 15;
   const uint64_t n_rg = (N + RG - 1) / RG;
-  std::vector<uint64_t>& foff = H.t_foff;
-  foff.assign(N + 1, 0);
+  auto& foff = H.t_foff;
+  foff.resize(N + 1);
+  foff[0] = 0;
   std::vector<uint64_t> rg_sum(n_rg + 1, 0);
   std::vector<std::vector<uint64_t>> rg_keys(n_rg);
+  // (module, field) keys of heap accesses: a dense mark table when Dm x n_fields is small,
+  // else per-range sorted key lists merged below
+  const uint64_t NF = d->n_fields;
+  const bool kdense = (uint64_t)Dm * NF <= (1ull << 22);
+  std::vector<uint8_t>& kmark = H.t_kmark;
+  if (kdense) kmark.assign(Dm * NF, 0);
   FirstErr fe0;
   auto fkey = [&](uint64_t n) -> uint64_t {                 // UINT64_MAX: no field-row table
     const uint8_t kind = d->node_kind[n];
@@ -388,11 +456,16 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       acc += w;
       foff[n + 1] = acc;                                       // range-local inclusive prefix
       const uint64_t key = fkey(n);
-      if (key != UINT64_MAX) keys.push_back(key);
+      if (key != UINT64_MAX) {
+        if (kdense) __atomic_store_n(&kmark[(key >> 32) * NF + (uint32_t)key], (uint8_t)1, __ATOMIC_RELAXED);
+        else keys.push_back(key);
+      }
     }
     rg_sum[lo / RG + 1] = acc;
-    std::sort(keys.begin(), keys.end());
-    keys.erase(std::unique(keys.begin(), keys.end()), keys.end());
+    if (!kdense) {
+      std::sort(keys.begin(), keys.end());
+      keys.erase(std::unique(keys.begin(), keys.end()), keys.end());
+    }
   });
   if (fe0.st != GDROID_OK) return fe0.result();
   const uint64_t n_args = d->call_arg_ptr[N];
@@ -401,29 +474,42 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     const uint64_t base = rg_sum[lo / RG];
     for (uint64_t n = lo; n < hi; ++n) foff[n + 1] += base;
   });
+  PHASE("node sizes + field keys");
   // field-row tables of FLOAD/FSTORE/ALOAD/ASTORE: one per (module, field) pair used
-  std::vector<uint64_t> fkeys;
-  for (auto& v : rg_keys) fkeys.insert(fkeys.end(), v.begin(), v.end());
-  std::sort(fkeys.begin(), fkeys.end());
-  fkeys.erase(std::unique(fkeys.begin(), fkeys.end()), fkeys.end());
-  std::vector<uint32_t> fkey_off(fkeys.size());
-  for (size_t i = 0; i < fkeys.size(); ++i) {
-    const uint64_t dd = fkeys[i] >> 32;
-    const uint32_t f = (uint32_t)fkeys[i];
-    const ModRec& md = H.mods[db + dd];
-    fkey_off[i] = (uint32_t)H.frow.size();
-    for (uint32_t c = 0; c < md.n_cols; ++c) {
-      const int32_t ty = H.col_type[md.col_off + c];
-      int32_t row = -1;
-      if (c != 0 && ty >= 0)
-        for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
-          if (H.tf[q] == f) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
-      H.frow.push_back(row);
-    }
+  std::vector<uint64_t> fkeys;                                  // sorted (module << 32 | field)
+  std::vector<uint32_t>& kidx = H.t_kidx;                       // dense: key -> index in fkeys
+  if (kdense) {
+    kidx.resize(Dm * NF);
+    scan_marks(kmark, [&](uint64_t i) { kidx[i] = (uint32_t)fkeys.size(); fkeys.push_back(((i / NF) << 32) | (i % NF)); });
+  } else {
+    for (auto& v : rg_keys) fkeys.insert(fkeys.end(), v.begin(), v.end());
+    std::sort(fkeys.begin(), fkeys.end());
+    fkeys.erase(std::unique(fkeys.begin(), fkeys.end()), fkeys.end());
   }
+  std::vector<uint32_t> fkey_off(fkeys.size() + 1);
+  const size_t frow0 = H.frow.size();
+  fkey_off[0] = (uint32_t)frow0;
+  for (size_t i = 0; i < fkeys.size(); ++i) fkey_off[i + 1] = fkey_off[i] + H.mods[db + (fkeys[i] >> 32)].n_cols;
+  H.frow.resize(fkey_off[fkeys.size()]);
+  parallel_ranges(fkeys.size(), 256, [&](uint64_t lo, uint64_t hi) {
+    for (uint64_t i = lo; i < hi; ++i) {
+      const uint64_t dd = fkeys[i] >> 32;
+      const uint32_t f = (uint32_t)fkeys[i];
+      const ModRec& md = H.mods[db + dd];
+      for (uint32_t c = 0; c < md.n_cols; ++c) {
+        const int32_t ty = H.col_type[md.col_off + c];
+        int32_t row = -1;
+        if (c != 0 && ty >= 0)
+          for (uint32_t q = H.tf_ptr[ty]; q < H.tf_ptr[ty + 1]; ++q)
+            if (H.tf[q] == f) row = (int32_t)(H.col_hbase[md.col_off + c] + (q - H.tf_ptr[ty]));
+        H.frow[fkey_off[i] + c] = row;
+      }
+    }
+  });
   auto frow_of = [&](uint64_t n) -> int32_t {
     const uint64_t key = fkey(n);
     if (key == UINT64_MAX) return -1;
+    if (kdense) return (int32_t)fkey_off[kidx[(key >> 32) * NF + (uint32_t)key]];
     return (int32_t)fkey_off[std::lower_bound(fkeys.begin(), fkeys.end(), key) - fkeys.begin()];
   };
   auto local_idx = [&](int64_t gid, uint64_t m) -> int64_t {
@@ -534,6 +620,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     cls_cnt[R.cls] += n_chunks_of(R.e1 - R.e0, R.cls);     // work items per GRP class
     return GDROID_OK;
   };
+  PHASE("field-row tables");
   parallel_ranges(N, 1 << 14, [&](uint64_t lo, uint64_t hi) {
     uint32_t cc[NCLS] = {0, 0, 0, 0, 0};
     for (uint64_t n = lo; n < hi; ++n) {
@@ -547,7 +634,13 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   H.fact_words += foff[N];
   PHASE("nodes");
   // ---- projection tables: one per (source module, target module) pair with a CALL/RET edge
+  // (source module, target module) pairs: a dense mark table when Dm^2 is small, else sorted
+  // per-range lists merged
   std::vector<uint64_t> pairs;
+  const bool pdense = (uint64_t)Dm * Dm <= (1ull << 22);
+  std::vector<uint8_t>& pmark = H.t_pmark;
+  std::vector<uint32_t>& pidx = H.t_pidx;
+  if (pdense) pmark.assign(Dm * Dm, 0);
   {
     std::mutex pm;
     parallel_ranges(N, 1 << 15, [&](uint64_t lo, uint64_t hi) {
@@ -560,16 +653,24 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
           const uint8_t ek = d->edge_kind[e];
           if (ek != GE_CALL && ek != GE_RET) continue;
           const uint32_t dm = d->method_module[d->node_method[d->col[e]]];
-          if (dm != sm) loc.push_back(((uint64_t)sm << 32) | dm);
+          if (dm == sm) continue;
+          if (pdense) __atomic_store_n(&pmark[(uint64_t)sm * Dm + dm], (uint8_t)1, __ATOMIC_RELAXED);
+          else loc.push_back(((uint64_t)sm << 32) | dm);
         }
       }
+      if (pdense) return;
       std::sort(loc.begin(), loc.end());
       loc.erase(std::unique(loc.begin(), loc.end()), loc.end());
       std::lock_guard<std::mutex> l(pm);
       pairs.insert(pairs.end(), loc.begin(), loc.end());
     });
-    std::sort(pairs.begin(), pairs.end());
-    pairs.erase(std::unique(pairs.begin(), pairs.end()), pairs.end());
+    if (pdense) {
+      pidx.resize(Dm * Dm);
+      scan_marks(pmark, [&](uint64_t i) { pidx[i] = (uint32_t)pairs.size(); pairs.push_back(((i / Dm) << 32) | (i % Dm)); });
+    } else {
+      std::sort(pairs.begin(), pairs.end());
+      pairs.erase(std::unique(pairs.begin(), pairs.end()), pairs.end());
+    }
   }
   std::vector<uint32_t> pair_off(pairs.size() + 1, 0);
   for (size_t i = 0; i < pairs.size(); ++i) {
@@ -577,7 +678,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     pair_off[i + 1] = pair_off[i] + ms.n_cols + mt.n_glob + ms.n_glob;   // colmap, rowmap, rowinv
   }
   const size_t xbase = H.xmap.size();
-  H.xmap.resize(xbase + pair_off[pairs.size()], -1);
+  H.xmap.resize(xbase + pair_off[pairs.size()]);              // uninitialised: each pair fills its own
   parallel_ranges(pairs.size(), 64, [&](uint64_t lo, uint64_t hi) {
     std::vector<int32_t> t2s;
     for (uint64_t i = lo; i < hi; ++i) {
@@ -587,6 +688,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
       const ModRec &ms = H.mods[db + sm], &mt = H.mods[db + dm];
       const ModInfo &Ps = mi[sm], &Pt = mi[dm];
       int32_t* cmap = H.xmap.data() + xbase + pair_off[i];   // src column -> dst column
+      std::fill(cmap, H.xmap.data() + xbase + pair_off[i + 1], -1);
       int32_t* rmap = cmap + ms.n_cols;                       // dst global row -> src global row
       t2s.assign(Pt.n_insts, -1);
       for (uint64_t a = 0, b2 = 0; a < Ps.n_insts && b2 < Pt.n_insts;) {
@@ -653,7 +755,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
         const uint32_t sm = d->method_module[m], dm = d->method_module[d->node_method[s]];
         if (sm != dm) {
           const uint64_t key = ((uint64_t)sm << 32) | dm;
-          const size_t i = std::lower_bound(pairs.begin(), pairs.end(), key) - pairs.begin();
+          const size_t i = pdense ? pidx[(uint64_t)sm * Dm + dm]
+                                  : std::lower_bound(pairs.begin(), pairs.end(), key) - pairs.begin();
           xoff = (uint32_t)(xbase + pair_off[i]);
         }
       }
