@@ -44,7 +44,7 @@ struct __align__(16) NodeRec {
   uint32_t grow_off; // module global-row tables
   uint16_t n_cols;   // |Q| of the module
   uint16_t app;      // index of the app inside a batch
-  uint32_t module;   // global module index
+  uint32_t local_base; // app-local slot gid of the method's local 0 (digest / readback)
 };
 static_assert(sizeof(NodeRec) == 64, "NodeRec must be 64 bytes");
 

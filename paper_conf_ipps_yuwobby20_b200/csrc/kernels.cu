@@ -1064,7 +1064,7 @@ __global__ void k_rebase(Dev D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* ro
     NodeRec R = nodes[n];
     const AppBase b = bases[R.app];
     R.off += b.fact; R.e0 += b.edge; R.e1 += b.edge;
-    R.col_off += b.col; R.grow_off += b.grow; R.module += b.mod;
+    R.col_off += b.col; R.grow_off += b.grow;
     if (R.kind >= GK_FLOAD && R.kind <= GK_ASTORE && R.r3 >= 0) R.r3 += (int32_t)b.frow;
     nodes[n] = R;
     nodemeth[n] += b.meth;
@@ -1128,13 +1128,17 @@ __global__ void k_seed(Dev D) {
   stage_publish(D, st, 1u);
 }
 
-// (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8)
+// (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp's nodes are
+// nw apart, so consecutive ones almost always belong to the same app: the app sum is carried in
+// a register and added once per app change (not one same-address atomic per node).
 __global__ void __launch_bounds__(256) k_digest(Dev D) {
   const int lane = threadIdx.x & 31;
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+  unsigned long long app_sum = 0;
+  uint32_t app_cur = 0xffffffffu;
   for (uint32_t n = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < D.n_nodes; n += nw) {
     const NodeRec R = D.nodes[n];
-    const uint32_t local_base = D.meths[D.node_method[n]].local_base;
+    const uint32_t local_base = R.local_base;
     const uint32_t logW = R.logW, L = R.L, B = R.B;
     const uint64_t* X = D.facts + R.off;
     const uint64_t hn = mix64((uint64_t)(n - D.app_node_base[R.app]));
@@ -1154,9 +1158,15 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
     s = warp_sum64(s);
     if (lane == 0) {
       D.node_digest[n] = s;
-      atomicAdd(&D.app_digest[R.app], s);
+      if (R.app != app_cur) {
+        if (app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
+        app_cur = R.app;
+        app_sum = 0;
+      }
+      app_sum += s;
     }
   }
+  if (lane == 0 && app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
 }
 
 __global__ void k_popc(Dev D, uint32_t n0, uint32_t n1, uint64_t* out) {
@@ -1178,7 +1188,7 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
   for (uint32_t n = n0 + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < n1; n += nw) {
     const NodeRec R = D.nodes[n];
-    const uint32_t local_base = D.meths[D.node_method[n]].local_base;
+    const uint32_t local_base = R.local_base;
     const uint32_t logW = R.logW, L = R.L, B = R.B;
     uint64_t base = ptr[n - n0];
     for (uint32_t w0 = 0; w0 < B; w0 += 32) {

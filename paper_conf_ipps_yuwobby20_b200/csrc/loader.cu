@@ -612,7 +612,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     R.B = (uint32_t)words; R.L = L; R.n_stat = md.n_stat;
     R.e0 = (uint32_t)d->row_ptr[n]; R.e1 = (uint32_t)d->row_ptr[n + 1];
     R.col_off = md.col_off; R.grow_off = md.grow_off; R.n_cols = (uint16_t)md.n_cols;
-    R.logW = (uint8_t)md.logW; R.module = db + (uint32_t)dd;
+    R.logW = (uint8_t)md.logW; R.local_base = (uint32_t)local_base[m];
     H.o_nodes[n] = R;
     H.o_nodemeth[n] = mb + (uint32_t)m;
     H.o_rowptr[n + 1] = (uint32_t)d->row_ptr[n + 1];

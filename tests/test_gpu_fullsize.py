@@ -99,3 +99,41 @@ def test_corpus_run_shard_pipeline():
     assert sorted(seen) == ids and len(res) >= 2
     for i in ids:
         assert seen[i] == fx[f"corpus{i}"]["app_digest"]
+
+
+# ---- the 1000-app corpus (BASELINE.json configs[4]) against tests/golden/corpus_digests.json
+# (written by scripts/make_corpus_digests.py, which calls only oracle/).  The clipped tail of 15
+# worst-shaped apps (|Q| = 256, ~800 s of oracle each) is covered by the `worst` preset entry.
+CFIX = os.path.join(HERE, "golden", "corpus_digests.json")
+
+
+def _corpus_check(ids):
+    if not os.path.exists(CFIX):
+        pytest.skip("no stored corpus digests")
+    fx = json.load(open(CFIX))
+    assert fx["gen_version"] == G.GEN_VERSION
+    ids = [i for i in ids if str(i) in fx["apps"]]
+    assert ids
+    for b0 in range(0, len(ids), 8):
+        batch = ids[b0:b0 + 8]
+        gs = [G.corpus_app(i) for i in batch]
+        app = gd.load(gs)
+        app.build()
+        digs = app.app_digests()
+        for k, (i, g) in enumerate(zip(batch, gs)):
+            ref = fx["apps"][str(i)]
+            assert g.n_nodes == ref["n_nodes"]
+            assert str(int(digs[k])) == ref["app_digest"], f"corpus{i}"
+        app.free()
+    return len(ids)
+
+
+def test_corpus_digest_sample():
+    """Every 20th app of the corpus (50 apps, 20K-2M nodes), in 8-app batches as bench.py runs them."""
+    assert _corpus_check(list(range(0, 1000, 20))) >= 45
+
+
+@pytest.mark.skipif(not os.environ.get("GDROID_FULL_CORPUS"), reason="set GDROID_FULL_CORPUS=1 (about 5 min)")
+def test_corpus_digest_all():
+    """All 985 narrow apps of the 1000-app corpus."""
+    assert _corpus_check(list(range(1000))) == 985
