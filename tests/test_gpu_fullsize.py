@@ -133,7 +133,7 @@ def test_corpus_digest_sample():
     assert _corpus_check(list(range(0, 1000, 20))) >= 45
 
 
-@pytest.mark.skipif(not os.environ.get("GDROID_FULL_CORPUS"), reason="set GDROID_FULL_CORPUS=1 (about 5 min)")
+@pytest.mark.skipif(bool(os.environ.get("GDROID_QUICK")), reason="GDROID_QUICK set (about 75 s on a B200)")
 def test_corpus_digest_all():
-    """All 985 narrow apps of the 1000-app corpus."""
+    """All 985 narrow apps of the 1000-app corpus (profiles/r01_full_corpus_parity.log)."""
     assert _corpus_check(list(range(1000))) == 985
