@@ -428,7 +428,8 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   // (module, field) keys of heap accesses: a dense mark table when Dm x n_fields is small,
   // else per-range sorted key lists merged below
   const uint64_t NF = d->n_fields;
-  const bool kdense = (uint64_t)Dm * NF <= (1ull << 22);
+  const bool force_sparse = getenv("GDROID_LOADER_SPARSE") != nullptr;   // tests: sorted-key paths
+  const bool kdense = !force_sparse && (uint64_t)Dm * NF <= (1ull << 22);
   std::vector<uint8_t>& kmark = H.t_kmark;
   if (kdense) kmark.assign(Dm * NF, 0);
   FirstErr fe0;
@@ -637,7 +638,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   // (source module, target module) pairs: a dense mark table when Dm^2 is small, else sorted
   // per-range lists merged
   std::vector<uint64_t> pairs;
-  const bool pdense = (uint64_t)Dm * Dm <= (1ull << 22);
+  const bool pdense = !force_sparse && (uint64_t)Dm * Dm <= (1ull << 22);
   std::vector<uint8_t>& pmark = H.t_pmark;
   std::vector<uint32_t>& pidx = H.t_pidx;
   if (pdense) pmark.assign(Dm * Dm, 0);

@@ -224,3 +224,17 @@ def test_uncounted_instantiation_same_results(wide):
     app.build(byte_model=False, loop_mode=1)
     for k in (0, 41, 79):
         _assert_same(app, k, gs[k], oracle.build_idfg(gs[k]))
+
+
+def test_loader_sorted_key_paths(monkeypatch):
+    """The loader's fallback for apps with too many modules / fields for the dense (module, field)
+    and (module, module) mark tables (GDROID_LOADER_SPARSE forces it): same tables, same facts."""
+    monkeypatch.setenv("GDROID_LOADER_SPARSE", "1")
+    gs = [random_tiny(s) for s in range(900, 960)] + [tiny2()[0]]
+    app = gd.load(gs)
+    app.build()
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        _assert_same(app, k, g, r, g.name)
+        assert int(digs[k]) == r.app_digest
