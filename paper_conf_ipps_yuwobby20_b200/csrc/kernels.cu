@@ -50,7 +50,7 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #define GD_PRE2 1              // ... and of the second edge
 #endif
 #ifndef GD_CONT_DENSE
-#define GD_CONT_DENSE 0        // continue into narrow (one word per row) destinations too (light rounds)
+#define GD_CONT_DENSE 1        // continue into narrow (one word per row) destinations too (light rounds)
 #endif
 constexpr uint32_t NO_CONT = 0xffffffffu;
 
@@ -500,9 +500,10 @@ __device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r)
 // path, with every read that the chain allows issued in the first memory hop: IN(src), the
 // destinations' round stamps and (FLOAD/FSTORE) the field-row table; the rows the transfer
 // function reads are taken from the IN(src) registers by shuffles instead of reloads.
-template <bool CNT>
-__device__ __forceinline__ void process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
-                                               uint32_t round, uint32_t nxt, int lane, Acc& acc) {
+template <bool CNT, bool CD>
+__device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
+                                                   uint32_t round, uint32_t nxt, int lane, Acc& acc,
+                                                   bool cont_ok) {
   const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
   const uint64_t* __restrict__ X = D.facts + R.off;
   uint64_t y[KW], p0[KW], p1[KW];
@@ -602,18 +603,20 @@ __device__ __forceinline__ void process_inline(const Dev& D, CtaStage& st, const
     }
     if (__any_sync(FULL, g)) gmask |= 1u << i;
   }
-  flush_pushes(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt, nullptr, false,
-               my_stamp);
+  uint32_t cont_v = NO_CONT;                               // GD_CONT_DENSE: depth-first successor
+  flush_pushes(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt,
+               (CD && cont_ok) ? &cont_v : nullptr, true, my_stamp);
   if constexpr (CNT) {
     const uint32_t alg_l0 = (uint32_t)sizeof(NodeRec) + (uint32_t)sizeof(InlEdge) * ne + 4u;
     acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
     acc_add(acc.atom, red);
     if (lane == 0) acc.dense += 8ull * B + 16ull * B * ne + alg_l0;
   }
+  return cont_v;
 }
 
 // ---------------------------------------------------------------------------------- one item
-template <bool WIDE, bool CNT, int MW>
+template <bool WIDE, bool CNT, int MW, bool CD>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
@@ -634,13 +637,12 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     if (R.logW >= 1) {                                      // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
       process_wide<CNT, MW>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
-                   allow_cont ? &cont_v : nullptr, GD_CONT_DENSE && light);
+                   allow_cont ? &cont_v : nullptr, CD && light);
       return cont_v;
     }
   }
   if (GD_INL && !WIDE && !GD_SMASK && first && R.n_inl) {   // (wide batches: measured slower)
-    process_inline<CNT>(D, st, R, me, round, nxt, lane, acc);
-    return NO_CONT;
+    return process_inline<CNT, CD>(D, st, R, me, round, nxt, lane, acc, allow_cont && light);
   }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
@@ -882,7 +884,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     const unsigned gall = __reduce_or_sync(FULL, gmask);
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
     flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt,
-                 (GD_CONT_DENSE && allow_cont && light) ? &cont_v : nullptr, true);
+                 (CD && allow_cont && light) ? &cont_v : nullptr, true);
   }
   if constexpr (CNT) {
     acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
@@ -923,7 +925,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 
 // Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
-template <bool WIDE, bool CNT, int MW>
+template <bool WIDE, bool CNT, int MW, bool CD>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
@@ -968,6 +970,9 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   };
   // Continuation into narrow destinations (GD_CONT_DENSE) only while the round leaves warps
   // idle (total items below GD_CONT_LOAD/4 x warps); wide destinations always continue.
+  // Narrow continuation (CD) is compiled into the 3-CTA/SM narrow instantiation only: small
+  // and median apps spend most rounds light (small 2.30 -> 1.92 ms, 332 -> 80 rounds; median
+  // 6.59 -> 6.31 ms), while the corpus shard (+7 %) and wide batches (+1 %) lost with it.
   const bool cont_ok = (uint64_t)total * 4u < (uint64_t)nw * GD_CONT_LOAD;
   // MER (Fig. 7): process the head list — whole waves of nw items — and
   // merge the tail into the next worklist (the round stamp removes repetitions).
@@ -993,12 +998,12 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       const uint32_t nn = nentry >> 5;
       asm volatile("prefetch.global.L1 [%0];" :: "l"(lane == 0 ? (const char*)(D.nodes + nn) : (const char*)(D.inl + 4 * nn)));
     }
-    if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !GD_CONT_DENSE)) {
-      process_item<WIDE, CNT, MW>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
+    if constexpr (GD_CONT_DEPTH == 0 || (!WIDE && !CD)) {
+      process_item<WIDE, CNT, MW, CD>(D, st, entry >> 5, entry & 31u, round, nxt, lane, ws, acc, false);
     } else {
       uint32_t n = entry >> 5, ci = entry & 31u;
       for (int depth = 0;; ++depth) {
-        const uint32_t c = process_item<WIDE, CNT, MW>(D, st, n, ci, round, nxt, lane, ws, acc,
+        const uint32_t c = process_item<WIDE, CNT, MW, CD>(D, st, n, ci, round, nxt, lane, ws, acc,
                                               depth < GD_CONT_DEPTH, cont_ok);
         if (c == NO_CONT) break;
         __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
@@ -1026,7 +1031,8 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   stage_init(st);
   __syncthreads();
   for (uint32_t round = 1;; ++round) {
-    const uint32_t total = run_round<WIDE, CNT, MW>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+    const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB>(D, st, round, gw, nw, lane,
+                                                                                 ws_all[wib], acc);
     if (total == 0) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
@@ -1049,7 +1055,8 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
-  const uint32_t total = run_round<WIDE, CNT, MW>(D, st, round, gw, nw, lane, ws_all[wib], acc);
+  const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE>(D, st, round, gw, nw, lane, ws_all[wib],
+                                                                         acc);
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);
