@@ -181,7 +181,10 @@ struct Dev {
   uint32_t max_rounds;
   uint32_t wide;                // max log2(words per row) over the batch's modules: 0 = all narrow,
                                 // >= 1: some module has > 64 instances (row-occupancy path)
-  uint32_t hiocc;               // 1: narrow batch of >= HIOCC_NODES nodes, 4-CTA/SM instantiation
+  uint32_t hiocc;               // 1: launch the 4-CTA/SM narrow instantiation (batches >= HIOCC_NODES)
+  uint32_t round0;              // first round of this launch (hybrid launches resume mid-build)
+  uint32_t sw_lo, sw_hi;        // hybrid: leave at the start of a round with < sw_lo / >= sw_hi items
+                                // (bar[3] = that round), 0 = off
   uint32_t flags;               // F_* scheduling switches of the build (ablation variants)
   uint32_t count;               // 1: evaluate the byte models (alg/dense bytes, atomics) on the device
   unsigned long long* trace;    // optional per-round trace: {globaltimer ns, items << 32 | nodes}

@@ -53,6 +53,7 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #define GD_CONT_DENSE 1        // continue into narrow (one word per row) destinations too (light rounds)
 #endif
 constexpr uint32_t NO_CONT = 0xffffffffu;
+constexpr uint32_t ROUND_SWITCH = 0xffffffffu;   // run_round: leave this launch before the round
 
 struct Acc {                   // per-warp counters (shared memory), flushed once per kernel
   unsigned long long alg;      // touched-word model bytes
@@ -947,6 +948,10 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     return 0;
   }
   if (D.max_rounds && round > D.max_rounds) return total;
+  if ((D.sw_lo && total < D.sw_lo) || (D.sw_hi && total >= D.sw_hi)) {   // hybrid: hand over
+    if (blockIdx.x == 0 && threadIdx.x == 0) D.bar[3] = round;
+    return ROUND_SWITCH;
+  }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     const uint32_t nodes = D.counts[cur * CNT_STRIDE + CNT_NODES];
 #pragma unroll
@@ -1030,10 +1035,10 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
   __syncthreads();
-  for (uint32_t round = 1;; ++round) {
+  for (uint32_t round = D.round0;; ++round) {
     const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB>(D, st, round, gw, nw, lane,
                                                                                  ws_all[wib], acc);
-    if (total == 0) break;
+    if (total == 0 || total == ROUND_SWITCH) break;
     if (D.max_rounds && round > D.max_rounds) {
       if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
       break;
@@ -1057,6 +1062,7 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
   __syncthreads();
   const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE>(D, st, round, gw, nw, lane, ws_all[wib],
                                                                          acc);
+  if (total == ROUND_SWITCH) { flush_acc(D, acc); return; }
   if (total && D.max_rounds && round > D.max_rounds && blockIdx.x == 0 && threadIdx.x == 0)
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);

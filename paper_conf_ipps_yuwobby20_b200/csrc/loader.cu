@@ -29,6 +29,17 @@ using namespace gd;
 
 namespace {
 
+#ifndef GD_HYBRID
+#define GD_HYBRID 1          // large narrow batches alternate the 3- and 4-CTA/SM instantiations
+#endif
+constexpr uint32_t HYB_SWITCHES = 8;
+#ifndef GD_HYB_HI
+#define GD_HYB_HI 16         // heavy round: >= GD_HYB_HI/4 waves of items (3-CTA grid)
+#endif
+#ifndef GD_HYB_LO
+#define GD_HYB_LO 4          // light round: < GD_HYB_LO/4 waves
+#endif
+
 thread_local std::string g_err;
 
 // GDROID_TIMING=1: print host-side phase times of gdroid_load_* to stderr
@@ -1025,6 +1036,8 @@ struct gdroid_app {
   uint64_t launches = 0;
   bool built = false, pending = false;
   int max_blocks = 0;
+  int max_blocks_lo = 0;              // hybrid (large narrow batches): grid of the 3-CTA/SM instantiation
+  uint32_t* h_bar = nullptr;          // pinned readback of the barrier words (hybrid hand-over)
   // PLAIN variant (plain.cu): set-based state, present when loaded with gdroid_load_icfg_plain
   PlainDev P{};
   void* d_plain = nullptr;            // uploaded inputs + sets, locks, stamps, queues, scratch, heap
@@ -1046,6 +1059,7 @@ void free_app(gdroid_app* a) {
   if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
   delete a->h_stats;
+  if (a->h_bar) cudaFreeHost(a->h_bar);
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
   cudaSetDevice(cur);
@@ -1366,6 +1380,8 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   }
   D.hiocc = (D.wide == 0 && N >= HIOCC_NODES) ? 1u : 0u;
   a->max_blocks = fixpoint_max_blocks(device, D.wide, D.hiocc);
+  a->max_blocks_lo = fixpoint_max_blocks(device, D.wide, 0u);
+  if (D.hiocc && cudaMallocHost(&a->h_bar, 64) != cudaSuccess) return fail(set_err(GDROID_E_OOM, "pinned barrier readback"));
   PHASE("device state + k_rebase/k_edges");
   *out = a;
   return GDROID_OK;
@@ -1412,7 +1428,36 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   CU(launch_seed(D, s));
   a->launches++;
   CU(cudaEventRecord(a->ev[1], s));
-  if (o.loop_mode == 0) {
+  D.round0 = 1;
+  D.sw_lo = D.sw_hi = 0;
+  if (o.loop_mode == 0 && D.hiocc && GD_HYBRID && (D.flags & F_CONT)) {
+    // Hybrid (large narrow batches, default variant): light rounds run in the 3-CTA/SM
+    // instantiation with narrow continuation, heavy rounds (>= 4 waves of items) in the 4-CTA/SM
+    // one; a launch leaves at the first round of the other kind (bar[3] = that round) and the
+    // next launch resumes there.  At most HYB_SWITCHES hand-overs per build.
+    uint32_t blocks_lo = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks_lo) : (uint32_t)a->max_blocks_lo;
+    const uint32_t nw_lo = blocks_lo * (THREADS / 32);
+    bool heavy = false;
+    for (uint32_t sw = 0;; ++sw) {
+      const bool last = sw >= HYB_SWITCHES;
+      D.sw_lo = (heavy && !last) ? GD_HYB_LO * nw_lo / 4u : 0u;
+      D.sw_hi = (!heavy && !last) ? GD_HYB_HI * nw_lo / 4u : 0u;
+      D.hiocc = heavy ? 1u : 0u;
+      CU(cudaMemsetAsync(D.bar + 3, 0, 4, s));
+      const cudaError_t e = launch_fixpoint(D, heavy ? blocks : blocks_lo, s);
+      D.hiocc = 1u;
+      if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "k_fixpoint: %s", cudaGetErrorString(e));
+      a->launches++;
+      if (last) break;
+      CU(cudaMemcpyAsync(a->h_bar, D.bar, 16, cudaMemcpyDeviceToHost, s));
+      CU(cudaStreamSynchronize(s));
+      if (a->h_bar[3] == 0) break;                 // finished (empty worklist or round limit)
+      D.round0 = a->h_bar[3];
+      heavy = !heavy;
+    }
+    D.round0 = 1;
+    D.sw_lo = D.sw_hi = 0;
+  } else if (o.loop_mode == 0) {
     CU(launch_fixpoint(D, blocks, s));
     a->launches++;
   } else {
