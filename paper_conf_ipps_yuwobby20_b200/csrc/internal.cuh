@@ -13,7 +13,10 @@ constexpr int NCLS = 5;            // GRP classes + 2 interpr
 enum Cls : uint8_t { C_ONETIME = 0, C_SINGLE = 1, C_DOUBLE = 2, C_CALL = 3, C_EXIT = 4 };
 constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]; slot CNT_NODES = nodes queued
 constexpr int CNT_NODES = 5;
-constexpr uint32_t HIOCC_NODES = 1u << 20;   // batches this large are item-throughput bound
+#ifndef GD_HIOCC_NODES
+#define GD_HIOCC_NODES (1u << 17)
+#endif
+constexpr uint32_t HIOCC_NODES = GD_HIOCC_NODES;   // batches this large are item-throughput bound
 #ifndef GD_THREADS
 #define GD_THREADS 256
 #endif
