@@ -345,7 +345,7 @@ def run_ours(args):
         "gpu_launches": int(stats[-1]["kernel_launches"]) * args.steps,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "kernel": "k_fixpoint",
-                     "bytes_model": "touched-word (SURVEY §8(d)); per launch = one step; counted by one untimed build with the counting kernel instantiation, timed launches run without the counters",
+                     "bytes_model": "touched-word (SURVEY §8(d)); per launch = one step's fixed point (1-3 k_fixpoint launches under the hybrid light/heavy schedule, DESIGN.md §5.4; achieved = bytes / their summed CUDA-event time, traffic = ncu DRAM bytes summed over them); counted by one untimed build with the counting kernel instantiation, timed launches run without the counters",
                      "alg_bytes_per_launch": alg, "dense_bytes_per_launch": dense,
                      "dense_achieved": dense / (statistics.mean(fix_ns) / 1e9) / 1e9,
                      "peak_source": peak_src, "traffic_workload": traffic_wl},

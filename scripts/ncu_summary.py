@@ -74,6 +74,10 @@ def main():
     if len(sys.argv) > 5:
         summary["bench_workload"] = sys.argv[5]
         summary["apps_per_rank"] = int(sys.argv[6]) if len(sys.argv) > 6 else 1
+    # Several captured launches of one kernel (the hybrid schedule runs k_fixpoint 1-3 times per
+    # build) are summed: dram_bytes_per_launch = bytes of one build (all its
+    # launches); the other metrics are those of the longest launch.
+    tscale = {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0}
     for d, u in raw(rep):
         name = kname(d.get("Kernel Name", "?"))
         m = {k: d.get(k) for k in KEYS if k in d}
@@ -84,7 +88,25 @@ def main():
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
         m["dram_bytes_per_launch"] = rd * scale.get(u.get("dram__bytes_read.sum"), 1) + \
             wr * scale.get(u.get("dram__bytes_write.sum"), 1)
+        ms = float(d.get("gpu__time_duration.sum", "0").replace(",", "") or 0) * \
+            tscale.get(u.get("gpu__time_duration.sum"), 1.0)
+        if name in summary:
+            prev = summary[name]
+            m["launches_captured"] = prev["launches_captured"] + 1
+            m["total_ms_captured"] = prev["total_ms_captured"] + ms
+            m["dram_bytes_per_launch"] += prev["dram_bytes_per_launch"]
+            if prev["_ms"] > ms:
+                keep = {k: m[k] for k in ("launches_captured", "total_ms_captured", "dram_bytes_per_launch")}
+                m = dict(prev, **keep)
+                ms = prev["_ms"]
+        else:
+            m["launches_captured"] = 1
+            m["total_ms_captured"] = ms
+        m["_ms"] = ms
         summary[name] = m
+    for m in summary.values():
+        if isinstance(m, dict):
+            m.pop("_ms", None)
     with open(prefix + ".json", "w") as fh:
         json.dump(summary, fh, indent=1)
     print(json.dumps(summary, indent=1))
