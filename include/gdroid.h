@@ -92,7 +92,9 @@ typedef struct {
 
 /* Build options; an all-zero struct (or NULL) means defaults. */
 typedef struct {
-  uint32_t async;        /* 1: enqueue only, complete with gdroid_sync                      */
+  uint32_t async;        /* 1: enqueue only, complete with gdroid_sync (narrow batches of
+                            >= 2^17 nodes with the default variant still wait on the stream
+                            at each light/heavy hand-over)                   */
   uint32_t max_rounds;   /* 0 = unlimited                                                   */
   uint32_t blocks;       /* persistent-kernel CTAs (0 = SMs x occupancy)                     */
   uint32_t loop_mode;    /* 0 = persistent cooperative kernel (default), 1 = host-launched
