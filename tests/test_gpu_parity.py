@@ -238,3 +238,25 @@ def test_loader_sorted_key_paths(monkeypatch):
         r = oracle.build_idfg(g)
         _assert_same(app, k, g, r, g.name)
         assert int(digs[k]) == r.app_digest
+
+
+def test_hybrid_schedule_limits_and_async():
+    """Large narrow batches run the hybrid light/heavy launches: a round limit
+    still stops the build (GDROID_E_LIMIT), an async build completes through gdroid_sync, a
+    small grid gives the same fixed point, and every run matches the stored oracle digest."""
+    import json
+    import os
+    from synth import generator as G
+    fx = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "oracle_digests.json")))
+    g = G.preset("median")
+    app = gd.load(g)
+    with pytest.raises(gd.GdroidError) as e:
+        app.build(max_rounds=5)
+    assert e.value.code == -8
+    assert app.build(asynchronous=True) is None
+    st = app.sync()
+    assert st["rounds"] > 0 and st["kernel_launches"] >= 3
+    assert str(int(app.app_digests()[0])) == fx["median"]["app_digest"]
+    app.build(blocks=37)
+    assert str(int(app.app_digests()[0])) == fx["median"]["app_digest"]
+    app.free()
