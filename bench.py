@@ -45,7 +45,7 @@ def parse():
                     help="ablation variant (SURVEY §8(f) 1); plain needs one app per rank")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     return ap.parse_args()
 
 
