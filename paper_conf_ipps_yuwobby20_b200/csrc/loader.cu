@@ -1037,7 +1037,8 @@ struct gdroid_app {
   bool built = false, pending = false;
   int max_blocks = 0;
   int max_blocks_lo = 0;              // hybrid (large narrow batches): grid of the 3-CTA/SM instantiation
-  uint32_t* h_bar = nullptr;          // pinned readback of the barrier words (hybrid hand-over)
+  uint32_t h_bar[4] = {0, 0, 0, 0};   // readback of the barrier words (hybrid hand-over; pageable:
+                                      // a per-handle pinned block would make gdroid_free synchronise)
   // PLAIN variant (plain.cu): set-based state, present when loaded with gdroid_load_icfg_plain
   PlainDev P{};
   void* d_plain = nullptr;            // uploaded inputs + sets, locks, stamps, queues, scratch, heap
@@ -1059,7 +1060,6 @@ void free_app(gdroid_app* a) {
   if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
   delete a->h_stats;
-  if (a->h_bar) cudaFreeHost(a->h_bar);
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
   cudaSetDevice(cur);
@@ -1381,7 +1381,6 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.hiocc = (D.wide == 0 && N >= HIOCC_NODES) ? 1u : 0u;
   a->max_blocks = fixpoint_max_blocks(device, D.wide, D.hiocc);
   a->max_blocks_lo = fixpoint_max_blocks(device, D.wide, 0u);
-  if (D.hiocc && cudaMallocHost(&a->h_bar, 64) != cudaSuccess) return fail(set_err(GDROID_E_OOM, "pinned barrier readback"));
   PHASE("device state + k_rebase/k_edges");
   *out = a;
   return GDROID_OK;
