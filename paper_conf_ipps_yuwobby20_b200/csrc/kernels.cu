@@ -49,6 +49,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_PRE2
 #define GD_PRE2 1              // ... and of the second edge
 #endif
+#ifndef GD_BAR_NS
+#define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
+#endif
 #ifndef GD_CONT_DENSE
 #define GD_CONT_DENSE 1        // continue into narrow (one word per row) destinations too (light rounds)
 #endif
@@ -908,7 +911,9 @@ __device__ __forceinline__ void grid_sync(uint32_t* bar, uint32_t nblocks) {
       __threadfence();
       atomicAdd(bar + 1, 1u);
     } else {
-      while (*vgen == gen) __nanosleep(20);
+      while (*vgen == gen) {
+        if constexpr (GD_BAR_NS > 0) __nanosleep(GD_BAR_NS);
+      }
     }
     __threadfence();                       // acquire: later loads see other SMs' writes
   }
