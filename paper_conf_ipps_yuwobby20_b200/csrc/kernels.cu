@@ -225,7 +225,7 @@ __device__ __forceinline__ void stage_publish(const Dev& D, CtaStage& st, uint32
 // OR KW words into IN(dst): a (possibly stale) load, then RED.OR only where bits are missing.
 // Words of row `kill` are dropped (C2R).  Returns the number of non-zero words in the low
 // 16 bits and the number of REDs issued in the high bits.
-__device__ __forceinline__ uint32_t or_chunk(uint64_t* __restrict__ Z, const uint64_t (&y)[KW], uint32_t c0,
+__device__ __forceinline__ uint32_t or_chunk(uint64_t* Z, const uint64_t (&y)[KW], uint32_t c0,
                                              int lane, int kill, uint32_t logW, uint64_t& mbits, uint32_t msh) {
   uint64_t cur[KW];
 #pragma unroll
@@ -295,8 +295,10 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
                              uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
   const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B, rows = B >> logW;
-  const uint64_t* __restrict__ X = D.facts + R.off;
-  const uint64_t* __restrict__ OCC = X + occ_offset(B);
+  // The fact store is read and RED.OR-ed by the same kernel (self loops write IN(src) within
+  // one item): no __restrict__ / const-cache loads on it, only plain coherent LDG.
+  const uint64_t* X = D.facts + R.off;
+  const uint64_t* OCC = X + occ_offset(B);
   const uint32_t nocc = occ_words(rows);
   const uint32_t kind = R.kind;
   // ---- transfer setup: generated row t (mode 1 replace / 2 or-in) or FSTORE rows (mode 3)
@@ -417,47 +419,50 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
             }
           }
         }
-        // target rows
-        int rt[3] = {-1, -1, -1};
-        if (ek == GE_INTRA) rt[0] = (int)r;
-        else if (ek == GE_C2R) rt[0] = ((int)r == R.r0) ? -1 : (int)r;
+        // Target rows.  Every edge kind maps source row r to at most one target row, except
+        // CALL locals: one local passed as several actuals feeds every such parameter
+        // (param_j <- arg_j for all j), so CALL scans all npar actuals.
+        int rt = -1;
+        const bool call_local = ek == GE_CALL && r < L;
+        if (ek == GE_INTRA) rt = (int)r;
+        else if (ek == GE_C2R) rt = ((int)r == R.r0) ? -1 : (int)r;
         else if (r >= L) {
           const uint32_t gs = r - L;
           const int gt = proj ? rowinv[gs] : (int)gs;       // π: source global row -> target row
-          if (gt >= 0) rt[0] = (int)Lt + gt;
+          if (gt >= 0) rt = (int)Lt + gt;
         } else if (ek == GE_RET) {
-          if (r == L - 1 && lhs >= 0) rt[0] = lhs;
+          if (r == L - 1 && lhs >= 0) rt = lhs;
+        }
+        if (rt < 0 && !call_local) continue;
+        uint64_t out[MW];                                   // the row in the target's columns
+        if (!proj) {
+#pragma unroll
+          for (int s2 = 0; s2 < MW; ++s2) out[s2] = y[s2];
         } else {
-          int k2 = 0;
-          for (uint32_t jj = 0; jj < npar && k2 < 3; ++jj) {
-            const int a = npar > 3 ? D.args[D.arg_ptr[n] + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
-            if (a == (int)r) rt[k2++] = (int)jj;
+#pragma unroll
+          for (int s2 = 0; s2 < MW; ++s2) out[s2] = 0;
+          for (uint32_t j = 0; j < W; ++j) {
+            uint64_t b = 0;
+#pragma unroll
+            for (int jj = 0; jj < MW; ++jj) if ((uint32_t)jj == j) b = y[jj];
+            while (b) {
+              const int bit = __ffsll((long long)b) - 1;
+              b &= b - 1;
+              const int cd = ws.cmap[j * 64 + bit];
+              if (cd < 0) continue;
+#pragma unroll
+              for (int s2 = 0; s2 < MW; ++s2)
+                if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
+            }
           }
         }
-#pragma unroll
-        for (int q = 0; q < 3; ++q) {
-          if (rt[q] < 0) continue;
-          if (!proj) {
-            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], y, nz, red, g, D.smask + ep->dst);
-          } else {
-            uint64_t out[MW];
-#pragma unroll
-            for (int s2 = 0; s2 < MW; ++s2) out[s2] = 0;
-            for (uint32_t j = 0; j < W; ++j) {
-              uint64_t b = 0;
-#pragma unroll
-              for (int jj = 0; jj < MW; ++jj) if ((uint32_t)jj == j) b = y[jj];
-              while (b) {
-                const int bit = __ffsll((long long)b) - 1;
-                b &= b - 1;
-                const int cd = ws.cmap[j * 64 + bit];
-                if (cd < 0) continue;
-#pragma unroll
-                for (int s2 = 0; s2 < MW; ++s2)
-                  if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
-              }
-            }
-            emit_row_words(Z, Bt, logWt, (uint32_t)rt[q], out, nz, red, g, D.smask + ep->dst);
+        if (!call_local) {
+          emit_row_words(Z, Bt, logWt, (uint32_t)rt, out, nz, red, g, D.smask + ep->dst);
+        } else {
+          const uint32_t a0 = npar > 3 ? D.arg_ptr[n] : 0u;
+          for (uint32_t jj = 0; jj < npar; ++jj) {        // param_jj <- arg_jj whenever arg_jj = r
+            const int a = npar > 3 ? D.args[a0 + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
+            if (a == (int)r) emit_row_words(Z, Bt, logWt, jj, out, nz, red, g, D.smask + ep->dst);
           }
         }
       }
@@ -509,7 +514,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
                                                    uint32_t round, uint32_t nxt, int lane, Acc& acc,
                                                    bool cont_ok) {
   const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
-  const uint64_t* __restrict__ X = D.facts + R.off;
+  const uint64_t* X = D.facts + R.off;             // coherent loads (no __restrict__: see process_wide)
   uint64_t y[KW], p0[KW], p1[KW];
   const uint64_t off0 = shfl64(me.off, 0), off1 = shfl64(me.off, 1);
 #pragma unroll
@@ -651,7 +656,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
   constexpr uint32_t logW = 0u, W = 1u;
-  const uint64_t* __restrict__ X = D.facts + R.off;
+  const uint64_t* X = D.facts + R.off;             // coherent loads (no __restrict__: see process_wide)
   uint32_t cont_v = NO_CONT;                                // node to continue into (warp-uniform)
 
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
@@ -961,9 +966,10 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     const uint32_t nodes = D.counts[cur * CNT_STRIDE + CNT_NODES];
 #pragma unroll
     for (int c = 0; c < CNT_STRIDE; ++c) D.counts[clr * CNT_STRIDE + c] = 0;
-    D.stats->rounds += 1;
-    D.stats->visits += nodes;
-    D.stats->hist[nodes <= 32 ? 0 : (nodes <= 64 ? 1 : 2)] += 1;
+    // atomics: in loop_mode 1 other CTAs of this launch may already add continuation visits
+    atomicAdd(&D.stats->rounds, 1ull);
+    atomicAdd(&D.stats->visits, (unsigned long long)nodes);
+    atomicAdd(&D.stats->hist[nodes <= 32 ? 0 : (nodes <= 64 ? 1 : 2)], 1ull);
     if (round <= D.trace_cap) {
       unsigned long long ns;
       asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
@@ -1039,13 +1045,25 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   Acc& acc = acc_all[wib];
   if (lane == 0) acc = Acc{0, 0, 0, 0};
   stage_init(st);
+  uint32_t round0 = D.round0;
+  if (D.hyb) {                 // hybrid sequence: resume where the previous launch handed over
+    round0 = *(volatile uint32_t*)(D.bar + 3);
+    if (round0 == 0) return;   // (uniform: bar[3] changes only when this launch ends, see below)
+  }
   __syncthreads();
-  for (uint32_t round = D.round0;; ++round) {
+  for (uint32_t round = round0;; ++round) {
     const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB>(D, st, round, gw, nw, lane,
                                                                                  ws_all[wib], acc);
-    if (total == 0 || total == ROUND_SWITCH) break;
+    if (total == ROUND_SWITCH) break;                 // bar[3] = this round (run_round)
+    if (total == 0) {                                 // fixed point: later launches return at once
+      if (D.hyb && blockIdx.x == 0 && threadIdx.x == 0) D.bar[3] = 0;
+      break;
+    }
     if (D.max_rounds && round > D.max_rounds) {
-      if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
+      if (blockIdx.x == 0 && threadIdx.x == 0) {
+        D.stats->limit_hit = 1;
+        if (D.hyb) D.bar[3] = 0;
+      }
       break;
     }
     stage_publish(D, st, (round + 1) % 3);
@@ -1144,6 +1162,7 @@ __global__ void k_seed(Dev D) {
     flush_pushes(D, st, lane, act, e, info, true, 0u, 1u);
   }
   stage_publish(D, st, 1u);
+  if (threadIdx.x == 0) D.bar[3] = 1;     // hybrid sequences start at round 1
 }
 
 // (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp's nodes are

@@ -75,7 +75,7 @@ struct Gen {
   std::vector<std::vector<uint32_t>> mod_sites;        // instances created by each module
   std::vector<std::unordered_set<uint32_t>> mod_neighbors;
   std::vector<std::vector<uint32_t>> planned;          // planned callees per method
-  std::vector<std::vector<uint32_t>> by_arity[4];      // per component: methods by arity
+  std::vector<std::vector<uint32_t>> by_arity[9];      // per component: methods by arity (0..8)
   std::vector<uint32_t> comp_of_method, comp_begin, comp_end;
   std::vector<std::pair<uint32_t, uint32_t>> pending_ret;  // (callee, retsite) RET edges
   std::vector<std::pair<uint32_t, uint32_t>> pending_call; // (call node, callee) CALL edges
@@ -142,8 +142,16 @@ struct Gen {
     int32_t lhs = R.uni() < 0.7 ? loc(def_local()) : -1;
     int c = node(cm, CALL, lhs);
     int r = node(cm, RETSITE, lhs, -1, -1, c);
-    for (uint32_t j = 0; j < ar; ++j)
-      call_args[c].push_back(R.uni() < 0.85 ? loc(use_local()) : -1);
+    // actuals: a used local (85 %) or a non-reference value (-1); 15 % of the calls with two or
+    // more parameters pass one local for several of them (setPadding(p, p, p, p)-style), so a
+    // source row can feed many parameter rows (C3)
+    if (ar >= 2 && R.uni() < 0.15) {
+      const int32_t rep = loc(use_local());
+      for (uint32_t j = 0; j < ar; ++j) call_args[c].push_back(R.uni() < 0.8 ? rep : (R.uni() < 0.5 ? -1 : loc(use_local())));
+    } else {
+      for (uint32_t j = 0; j < ar; ++j)
+        call_args[c].push_back(R.uni() < 0.85 ? loc(use_local()) : -1);
+    }
     for (uint32_t t : targets) {
       pending_call.push_back({(uint32_t)c, t});               // m_entry[t] may not exist yet
       pending_ret.push_back({t, (uint32_t)r});
@@ -289,10 +297,12 @@ struct Gen {
       if (!mod_statics[d].empty() && R.uni() < 0.5) mod_statics[d + 1].push_back(mod_statics[d][0]);
     for (auto& s : mod_statics) { std::sort(s.begin(), s.end()); s.erase(std::unique(s.begin(), s.end()), s.end()); }
     m_nparams.resize(M); m_nlocals.resize(M);
-    for (int a = 0; a < 4; ++a) by_arity[a].resize(K);
+    for (int a = 0; a < 9; ++a) by_arity[a].resize(K);
     for (uint32_t m = 0; m < M; ++m) {
       double u = R.uni();
-      uint32_t np = m == comp_begin[comp_of_method[m]] ? 0 : (u < 0.2 ? 0 : u < 0.55 ? 1 : u < 0.85 ? 2 : 3);
+      // arity 0..8 (Android APIs take up to ~8 arguments; 8 % of the methods take 4 or more)
+      uint32_t np = m == comp_begin[comp_of_method[m]] ? 0
+                  : (u < 0.2 ? 0 : u < 0.53 ? 1 : u < 0.80 ? 2 : u < 0.92 ? 3 : 4 + R.below(5));
       m_nparams[m] = np;
       m_nlocals[m] = np + std::max<uint32_t>(P.temps_per_method, 1) + 1;
       by_arity[np][comp_of_method[m]].push_back(m);

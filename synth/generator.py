@@ -28,7 +28,7 @@ _SRC = os.path.join(_HERE, "gen.cpp")
 _LIB = os.path.join(_HERE, "libgdrgen.so")
 _lock = threading.Lock()
 _lib = None
-GEN_VERSION = 1
+GEN_VERSION = 2   # 2: arity 0..8 with repeated actuals (round 2)
 
 
 def build(force: bool = False) -> str:

@@ -118,7 +118,7 @@ def random_inline_pair(seed: int):
     type_fields = [rng.sample(range(nf), rng.randint(1, nf)) for _ in range(n_types)]
     n_stat = rng.randint(0, 2)
     nl0 = rng.randint(2, 4)       # includes (unused) RET0
-    np1 = rng.randint(1, 2)
+    np1 = rng.choice((1, 1, 2, 2, 3, 4, 5, 6))   # arity up to 6 (> 3: the args-table path)
     nl1 = np1 + rng.randint(0, 2) + 1
     kinds0 = [NOP, PRIM, CONST, NEW, COPY, SLOAD, SSTORE, FLOAD, FSTORE, ALOAD, ASTORE]
     kinds1 = kinds0 + [RETV, RETV]
@@ -153,7 +153,11 @@ def random_inline_pair(seed: int):
         u1 = lambda: cee(r2.randrange(nl1 - 1))
         a_nodes = [_emit(r2, b, m0, k, u0, u0, types, sites) for k in A]
         lhs_i = r2.randrange(nl0 - 1)
-        args = [r2.randrange(nl0 - 1) if r2.random() < 0.8 else -1 for _ in range(np1)]
+        if np1 >= 2 and r2.random() < 0.4:         # one caller local passed as several actuals
+            rep = r2.randrange(nl0 - 1)
+            args = [rep if r2.random() < 0.8 else -1 for _ in range(np1)]
+        else:
+            args = [r2.randrange(nl0 - 1) if r2.random() < 0.8 else -1 for _ in range(np1)]
         b_nodes = [_emit(r2, b, m0, k, u0, u0, types, sites) for k in Bk]
         c_nodes = []
         for k in Ck:

@@ -39,7 +39,7 @@ def random_tiny(seed: int, n_methods: int = None, n_modules: int = None,
     meths = []
     for m in range(M):
         d = mods[m % D] if m < D else rng.choice(mods)
-        np_ = rng.randint(0, 2)
+        np_ = rng.choice((0, 0, 1, 1, 2, 2, 3, 4, 5))       # arity 0..5
         nl = np_ + rng.randint(1, 2) + 1
         meths.append(b.add_method(d, np_, nl))
     kinds = kinds or _STMT_KINDS
@@ -56,13 +56,16 @@ def random_tiny(seed: int, n_methods: int = None, n_modules: int = None,
         for _ in range(rng.randint(1, max_stmts)):
             k = rng.choice(kinds)
             if k == "CALL":
-                np_ = rng.randint(0, 2)
+                np_ = rng.choice(sorted({b.methods[t].n_params for t in meths}))
                 cands = [t for t in meths if b.methods[t].n_params == np_]
-                if not cands:
-                    continue
                 targets = rng.sample(cands, rng.randint(1, min(2, len(cands))))
                 lhs = loc() if rng.random() < 0.7 else None
-                args = [loc() if rng.random() < 0.8 else -1 for _ in range(np_)]
+                if np_ >= 2 and rng.random() < 0.35:     # one local passed as several actuals
+                    rep = loc()
+                    args = [rep if rng.random() < 0.8 else (-1 if rng.random() < 0.5 else loc())
+                            for _ in range(np_)]
+                else:
+                    args = [loc() if rng.random() < 0.8 else -1 for _ in range(np_)]
                 c, r = b.call(m, lhs, args, targets)
                 heads.append((c, r))
                 seq.append((c, r))
