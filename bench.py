@@ -3,17 +3,21 @@
 
 Metric (BASELINE.json): "IDFG build ms/app and node-visits/s (1 GPU); corpus apps/s at
 1/2/4/8 B200".  A *step* is one pass of the whole hot path (zero the
-fact store, seed, fixed point, digests) over one batch of synthetic apps resident in HBM.
+fact store, seed, fixed point, digests) over the workload, inputs resident in HBM.
 
 Workloads (--workload):
-  corpus  (default) each rank builds a fixed shard of B apps of the seeded 1000-app corpus
-          (BASELINE.json configs[4]; apps 0..B*N-1, LPT-sharded by estimated size) as ONE
-          batch handle: weak scaling (per-rank app count fixed as N grows).
-  median / small / worst   one app of that preset per rank (replicas).
-value = apps built by all ranks / max-over-ranks device time of the K timed steps.
+  corpus1000 (default) the seeded 1000-app corpus of BASELINE.json configs[4] (LogNormal
+          sizes, 20K-2M nodes, the clipped 1.5 % tail in the worst-case |Q| = 256 shape),
+          LPT-sharded over the ranks by estimated cost: STRONG scaling (the corpus is fixed,
+          N ranks split it).  Every rank keeps all its batches' tables in HBM; a batch holds a
+          fact store only while it builds.  value = 1000 apps / max-over-ranks
+          device time per step.  Rank 0 also builds the small / median / worst presets alone
+          (the metric's "IDFG build ms/app and node-visits/s (1 GPU)", `per_config`).
+  corpus8  the round-1 workload: 8 apps per rank as one batch (weak scaling).
+  small / median / worst   one app of that preset per rank (replicas).
 
 --impl reference runs the CPU oracle (oracle/, the reference arm of this tier) on a bounded
-sample of the same workload on the host cores; rank 0 only.
+sample of the same workload on the host cores (rank 0 only).
 """
 from __future__ import annotations
 
@@ -29,49 +33,83 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+# single-thread oracle throughput on narrow corpus apps (~10.6 us per node, tests/golden/
+# corpus_digests.json oracle_s): sizes the bounded CPU samples
+ORACLE_NODES_PER_CORE_S = 9.0e4
 METRIC = "IDFG build ms/app and node-visits/s (1 GPU); corpus apps/s at 1/2/4/8 B200"
+CORPUS_CACHE = os.path.join(ROOT, "tests", "golden", "corpus_digests.json")
+PRESET_CACHE = os.path.join(ROOT, "tests", "golden", "oracle_digests.json")
 
 
-def parse():
+def parse(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--workload", default="corpus", choices=["corpus", "median", "small", "worst"])
-    ap.add_argument("--apps-per-rank", type=int, default=8)
+    ap.add_argument("--workload", default="corpus1000",
+                    choices=["corpus1000", "corpus8", "median", "small", "worst"])
+    ap.add_argument("--n-apps", type=int, default=1000, help="corpus1000: apps of the corpus")
+    ap.add_argument("--apps-per-rank", type=int, default=8, help="corpus8: apps per rank")
+    ap.add_argument("--node-budget", type=int, default=4_000_000, help="narrow apps per batch (nodes)")
+    ap.add_argument("--wide-per-batch", type=int, default=1)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--loop-mode", type=int, default=0)
-    ap.add_argument("--variant", default="default", choices=["default", "mat", "mat_grp", "gdroid", "plain"],
-                    help="ablation variant (SURVEY §8(f) 1); plain needs one app per rank")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-seconds", type=float, default=12.0)
-    ap.add_argument("--e2e-steps", type=int, default=5)
-    return ap.parse_args()
+    ap.add_argument("--no-per-config", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--e2e-steps", type=int, default=1)
+    ap.add_argument("--e2e-readback", default="facts", choices=["facts", "digests"])
+    ap.add_argument("--gen-threads", type=int, default=0)
+    return ap.parse_args(argv)
+
+
+def host_threads():
+    return len(os.sched_getaffinity(0))
+
+
+def cpu_model():
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
 
 
 # ------------------------------------------------------------------ workload construction
-def workload_apps(args, rank, world):
-    """Returns (list of Icfg for this rank, description dict).  Generation is not timed."""
+def workload(args, world):
+    """(plan, make_app, desc).  Generation is never timed."""
+    from paper_conf_ipps_yuwobby20_b200 import corpus
     from synth import generator as G
-    if args.workload != "corpus":
-        g = G.preset(args.workload)
-        return [g], {"workload": f"{args.workload} app (seed {G.PRESETS[args.workload].seed})",
-                     "apps_per_rank": 1}
-    B = args.apps_per_rank
-    n_total = B * world
-    sizes = G.corpus_sizes(n_total)
-    order = sorted(range(n_total), key=lambda i: -sizes[i])       # LPT by estimated cost
-    loads = [0] * world
-    shard = [[] for _ in range(world)]
-    for i in order:
-        r = min(range(world), key=lambda q: (loads[q], q) if len(shard[q]) < B else (1 << 62, q))
-        shard[r].append(i)
-        loads[r] += sizes[i]
-    mine = sorted(shard[rank])
-    apps = [G.corpus_app(i) for i in mine]
-    return apps, {"workload": f"corpus shard: apps {n_total} of the seeded 1000-app corpus "
-                              f"(seeds 1000..{1000 + n_total - 1}), {B} per rank",
-                  "apps_per_rank": B, "app_ids": mine}
+    if args.workload == "corpus1000":
+        n = args.n_apps
+        cfgs = [G.corpus_config(i) for i in range(n)]
+        sizes = G.corpus_sizes(n)
+        wide = [c.q_cap > 64 for c in cfgs]
+        plan = corpus.plan_corpus(sizes, wide, world, node_budget=args.node_budget,
+                                  wide_per_batch=args.wide_per_batch)
+        desc = {"workload": f"corpus{n}: the seeded {n}-app corpus (BASELINE.json configs[4]; seeds "
+                            f"1000..{999 + n}; {sum(wide)} worst-shaped apps), LPT-sharded over "
+                            f"{world} rank(s), strong scaling",
+                "n_apps": n, "node_budget": args.node_budget, "wide_per_batch": args.wide_per_batch}
+        return plan, G.corpus_app, desc, "strong"
+    if args.workload == "corpus8":
+        B = args.apps_per_rank
+        n = B * world
+        sizes = G.corpus_sizes(n)
+        wide = [G.corpus_config(i).q_cap > 64 for i in range(n)]
+        plan = corpus.plan_corpus(sizes, wide, world, node_budget=1 << 62, per_rank=B)
+        plan.batches = [[sorted(s)] for s in plan.shards]          # one batch per rank
+        desc = {"workload": f"corpus shard: {B} apps per rank of the seeded corpus (seeds 1000..{999 + n}), "
+                            f"one batch per rank, weak scaling", "apps_per_rank": B}
+        return plan, G.corpus_app, desc, "weak"
+    # presets: one app per rank (replicas), app id = rank
+    cfg = G.PRESETS[args.workload]
+    plan = corpus.Plan(world, world, [0] * world, [cfg.q_cap > 64] * world,
+                       [[r] for r in range(world)], [[[r]] for r in range(world)])
+    desc = {"workload": f"{args.workload} app (seed {cfg.seed}), one per rank (replicas)"}
+    return plan, (lambda i: G.preset(args.workload)), desc, "weak"
 
 
 # ------------------------------------------------------------------ clocks sampling
@@ -134,15 +172,15 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def ncu_traffic(workload, apps_per_rank):
-    """Per-launch DRAM bytes of k_fixpoint from the committed ncu summary of THIS workload
-    (profiles/ncu_summary.json, written by scripts/ncu_summary.py), else None."""
+def ncu_traffic(workload):
+    """DRAM bytes of k_fixpoint per step of THIS workload from the committed ncu summary
+    (profiles/ncu_summary.json, written by scripts/ncu_summary.py), else (None, None)."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
     try:
         with open(p) as fh:
             d = json.load(fh)
         for cap in d.get("captures", [d]):
-            if cap.get("bench_workload") == workload and cap.get("apps_per_rank", apps_per_rank) == apps_per_rank:
+            if cap.get("bench_workload") == workload:
                 return cap.get("k_fixpoint", {}).get("dram_bytes_per_launch"), cap.get("workload")
     except Exception:
         pass
@@ -150,224 +188,274 @@ def ncu_traffic(workload, apps_per_rank):
 
 
 # ------------------------------------------------------------------ CPU oracle legs
-def oracle_sample(apps, seconds):
-    """Time the oracle (as it stands, single-threaded) on apps of the workload, cycling through
-    them until about `seconds` of CPU work (at most 64 runs)."""
+def oracle_sample_ids(plan, make_app_cost, budget_nodes):
+    """A size-stratified sample of the workload's narrow apps (evenly spaced in size order)
+    whose node count is about budget_nodes.  Worst-shaped apps (~800 s of one core each) are
+    excluded from the timed sample and reported separately."""
+    ids = sorted((i for s in plan.shards for i in s if not plan.wide[i]), key=lambda i: plan.sizes[i])
+    if not ids:
+        return []
+    tot = sum(plan.sizes[i] for i in ids)
+    k = max(1, min(len(ids), round(len(ids) * budget_nodes / max(tot, 1))))
+    step = len(ids) / k
+    return sorted({ids[int(j * step + step / 2)] for j in range(k)})
+
+
+def oracle_pool(apps, threads):
+    """Run the oracle (as it stands, single-threaded code) on every app with `threads`
+    concurrent workers; returns (wall s, Σ oracle s, Σ visits, digests)."""
+    from concurrent.futures import ThreadPoolExecutor
     import oracle
     t0 = time.perf_counter()
-    done, visits, app_s = 0, 0, []
-    while done < 64:
-        g = apps[done % len(apps)]
-        r = oracle.build_idfg(g)
-        done += 1
-        visits += r.visits
-        app_s.append(r.seconds)
-        if time.perf_counter() - t0 > seconds:
-            break
+    with ThreadPoolExecutor(max_workers=threads) as ex:
+        res = list(ex.map(oracle.run_timed, apps))
     wall = time.perf_counter() - t0
-    return {"apps": done, "wall_s": wall, "visits": visits, "oracle_s": sum(app_s),
-            "digests": None}
+    return wall, sum(r[0] for r in res), sum(r[1] for r in res), [r[2] for r in res]
 
 
 def run_reference(args):
-    """--impl reference: the oracle on host cores, same config/metric; rank 0 only."""
+    """--impl reference: the oracle on the host cores, same workload/metric; rank 0 only.
+    Each step = one bounded, size-stratified sample of the workload's apps run by P threads."""
     rank = int(os.environ.get("RANK", "0"))
-    world = int(os.environ.get("WORLD_SIZE", "1"))
     if rank != 0:
         return
-    apps, desc = workload_apps(args, 0, 1)
     import oracle
     oracle.build()
-    for i in range(args.warmup):
-        oracle.build_idfg(apps[i % len(apps)])
-    t0 = time.perf_counter()
-    visits = 0
-    for s in range(args.steps):                                  # one app per step (bounded)
-        r = oracle.build_idfg(apps[s % len(apps)])
-        visits += r.visits
-    dt = time.perf_counter() - t0
-    v = args.steps / dt
+    plan, make_app, desc, scaling = workload(args, 1)
+    P = host_threads()
+    per_step_nodes = ORACLE_NODES_PER_CORE_S * P * 4.0   # ~4 s of P threads per step
+    ids = oracle_sample_ids(plan, None, per_step_nodes * (args.steps + args.warmup))
+    if not ids:                                          # a preset workload: its one app
+        ids = plan.shards[0]
+    apps = [make_app(i) for i in ids]
+    nsteps = args.steps + args.warmup
+    chunks = [apps[j::nsteps] for j in range(nsteps)] if len(apps) >= nsteps else [apps] * nsteps
+    for j in range(args.warmup):
+        oracle_pool(chunks[j], P)
+    wall, n_apps, visits, nodes = 0.0, 0, 0, 0
+    for j in range(args.warmup, nsteps):
+        w, _, v, _ = oracle_pool(chunks[j], P)
+        wall += w
+        n_apps += len(chunks[j])
+        visits += v
+        nodes += sum(a.n_nodes for a in chunks[j])
+    v = n_apps / wall
+    sample = (f"{n_apps} apps in {args.steps} steps (size-stratified sample of the workload's "
+              f"narrow apps, {nodes} nodes), oracle on {P} host threads")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "apps/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+            "ms_per_step": wall / args.steps * 1e3, "higher_is_better": True, "scaling": scaling,
             "vs_baseline": None, "dtype": "u64", "data": "synthetic (seeded generator)",
-            "config": {**{k: v2 for k, v2 in desc.items() if k != "app_ids"},
-                       "step": "oracle on one app of the workload (bounded sample)"},
-            "node_visits_per_s": visits / dt,
-            "cpu_baseline": {"value": v, "unit": "apps/s", "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} apps of the workload, single-threaded C++ oracle"},
+            "config": {**desc, "step": "oracle on a bounded sample of the workload"},
+            "node_visits_per_s": visits / wall,
+            "cpu_baseline": {"value": v, "unit": "apps/s", "cores": P, "kind": "oracle",
+                             "sample": sample, "cpu_model": cpu_model()},
             "e2e": {"value": v, "unit": "apps/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
 # ------------------------------------------------------------------ the GPU arm
+def per_config_runs(device, stream, reps=5):
+    """The metric's single-GPU figures: each preset built alone (1 warm-up, `reps` timed
+    builds, CUDA events of the build; median), checked against the stored oracle digests."""
+    import paper_conf_ipps_yuwobby20_b200 as gd
+    from synth import generator as G
+    cache = json.load(open(PRESET_CACHE)) if os.path.exists(PRESET_CACHE) else {}
+    out = {}
+    for name in ("small", "median", "worst"):
+        g = G.preset(name)
+        app = gd.load(g, device=device, stream=stream)
+        app.build(byte_model=False)
+        st = [app.build(byte_model=False) for _ in range(reps)]
+        cnt = app.build(byte_model=True)
+        dig = int(app.app_digests()[0])
+        ref = cache.get(name, {})
+        ms = statistics.median(s["build_ns"] for s in st) / 1e6
+        fix_ms = statistics.median(s["fixpoint_ns"] for s in st) / 1e6
+        out[name] = {"nodes": g.n_nodes, "ms_per_app": ms, "fixpoint_ms": fix_ms,
+                     "node_visits_per_s": st[-1]["node_visits"] / (ms / 1e3),
+                     "rounds": st[-1]["rounds"], "us_per_round": 1e3 * fix_ms / max(1, st[-1]["rounds"]),
+                     "alg_gbs": cnt["alg_bytes"] / (fix_ms / 1e3) / 1e9,
+                     "parity": ("ok" if str(dig) == ref.get("app_digest") else
+                                ("MISMATCH" if ref else "no oracle cache"))}
+        app.free()
+    return out
+
+
 def run_ours(args):
     import numpy as np
     import torch
     import torch.distributed as dist
 
-    import paper_conf_ipps_yuwobby20_b200 as gd
+    from paper_conf_ipps_yuwobby20_b200 import corpus
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    # ranks on one host share its cores: the library's loader pool gets an equal share
     per_host = int(os.environ.get("LOCAL_WORLD_SIZE", "1"))
-    os.environ.setdefault("GDROID_HOST_THREADS", str(max(1, len(os.sched_getaffinity(0)) // max(1, per_host))))
+    nthreads = max(1, host_threads() // max(1, per_host))
+    os.environ.setdefault("GDROID_HOST_THREADS", str(nthreads))
     assert torch.cuda.is_available(), "bench needs a GPU"
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
-    apps, desc = workload_apps(args, rank, world)
-    n_apps = len(apps)
-    nodes = sum(g.n_nodes for g in apps)
-    input_bytes = sum(g.nbytes() for g in apps)
-
-    plain = args.variant == "plain"
-    assert not plain or len(apps) == 1, "--variant plain takes one app per rank (--apps-per-rank 1)"
-    app = gd.load(apps, device=local, stream=stream.cuda_stream, plain=plain)   # inputs resident in HBM
-    for _ in range(args.warmup):
-        app.build(loop_mode=args.loop_mode, variant=args.variant, byte_model=False)
-    torch.cuda.synchronize()
 
     def barrier():
         if world > 1:
             dist.barrier()
 
-    stats = []
-    with Clocks(local) as clk:
-        barrier()
-        torch.cuda.synchronize()
+    plan, make_app, desc, scaling = workload(args, world)
+    my_batches = plan.batches[rank]
+    my_ids = [i for b in my_batches for i in b]
+    apps = corpus.make_apps(my_ids, make_app, threads=args.gen_threads or nthreads)
+    shard = corpus.DeviceShard(my_batches, apps, device=local, stream=stream.cuda_stream)
+    nodes = sum(shard.nodes)
+    torch.cuda.synchronize()
+
+    def timer(fn):
         ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
         ev0.record(stream)
-        for _ in range(args.steps):
-            stats.append(app.build(loop_mode=args.loop_mode, variant=args.variant, byte_model=False))
+        fn()
         ev1.record(stream)
         torch.cuda.synchronize()
-        barrier()
-    my_ms = ev0.elapsed_time(ev1)
-    digests = app.app_digests()
-    # the byte models (SURVEY §8(d)) are counted by one extra, untimed build of the same
-    # workload with the counting instantiation of the kernel (same fixed point and schedule)
-    counted = app.build(loop_mode=args.loop_mode, variant=args.variant, byte_model=True)
-    assert np.array_equal(app.app_digests(), digests)
+        return ev0.elapsed_time(ev1)
 
-    # e2e: the public C-ABI calls with HOST buffers, every step: gdroid_load_batch (host tables +
-    # pinned H2D), gdroid_build_idfg, gdroid_app_digests (D2H of the result).  Steps are
-    # double-buffered like the paper's dual-buffering (PAPER.md:544-580): a loader thread loads
-    # step i+1 on its own stream while step i builds.
-    import queue as _queue
-    import threading as _threading
-    e2e_ms, e2e_parts = [], []
+    with Clocks(local) as clk:
+        res = corpus.run_rank(shard, args.steps, args.warmup, barrier, timer)
+    clocks = clk.summary()
+    stats, counted = res.stats, res.counted
+    my_ms = res.step_ms[0]
+    visits = sum(s["node_visits"] for s in stats)
+    fix_ns = sum(s["fixpoint_ns"] for s in stats)
+    alg = sum(s["alg_bytes"] for s in counted)
+    dense = sum(s["dense_bytes"] for s in counted)
+    launches = sum(s["kernel_launches"] for s in stats)
+    batch_ms = [s["build_ns"] / 1e6 for s in stats]
+    # per-app IDFG time: apps of a batch share its rounds; an app's share is its node fraction
+    app_ms = []
+    for b, s, nn in zip(my_batches, stats, shard.nodes):
+        for i in b:
+            app_ms.append(s["build_ns"] / 1e6 * apps[i].n_nodes / max(1, nn))
+    rec = corpus.pack_record(apps=len(my_ids), visits=visits, alg_bytes=alg, build_ns=int(my_ms * 1e6),
+                             wall_ns=int(my_ms * 1e6), max_app_ns=int(max(batch_ms) * 1e6),
+                             digest_sum=sum(res.digests.values()), errors=0)
+    recs = corpus.unpack_records(corpus.gather_records(rec, dev if world > 1 else None))
+    dig_all, dig_mask = corpus.gather_digests(plan.n_apps, res.digests, dev if world > 1 else None)
+    shard.free()
+
+    # e2e through the public API from host arrays: load (host tables + pinned H2D) of batch i+1
+    # overlapped with build + fact readback of batch i
+    e2e = None
     if args.e2e_steps > 0:
-        streams = [torch.cuda.Stream(device=local), torch.cuda.Stream(device=local)]
-        q = _queue.Queue(maxsize=1)
-        load_ms = []
-
-        def loader():
-            for i in range(args.e2e_steps + 1):          # +1: the first load primes the pipeline
-                t = time.perf_counter()
-                a = gd.load(apps, device=local, stream=streams[i % 2].cuda_stream, plain=plain)
-                load_ms.append((time.perf_counter() - t) * 1e3)
-                q.put(a)
-
-        th = _threading.Thread(target=loader, daemon=True)
         barrier()
         torch.cuda.synchronize()
-        th.start()
-        first = q.get()                                  # not timed: pipeline fill
-        first.build(loop_mode=args.loop_mode, variant=args.variant, byte_model=False)
-        assert np.array_equal(first.app_digests(), digests)
-        first.free()
+        d2h = h2d = 0
         t0 = time.perf_counter()
-        for i in range(args.e2e_steps):
-            tb = time.perf_counter()
-            a2 = q.get()
-            a2.build(loop_mode=args.loop_mode, variant=args.variant, byte_model=False)
-            tc = time.perf_counter()
-            d2 = a2.app_digests()                        # D2H of the result
-            a2.free()
-            assert np.array_equal(d2, digests)
-            e2e_parts.append(((tc - tb) * 1e3,))
-        e2e_total = (time.perf_counter() - t0) * 1e3
-        th.join()
-        e2e_ms = [e2e_total / args.e2e_steps]
-        e2e_parts = [(statistics.median(load_ms[1:]), statistics.median(x[0] for x in e2e_parts), 0.0)]
-    e2e_mine = statistics.median(e2e_ms) if e2e_ms else float("nan")
+        for _ in range(args.e2e_steps):
+            out = corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback)
+            for br in out:
+                for k, i in enumerate(br.app_ids):
+                    if int(br.digests[k]) != res.digests[i]:
+                        raise RuntimeError(f"e2e digest of app {i} differs from the device-resident run")
+                d2h += br.d2h_bytes
+                h2d += br.h2d_bytes
+        torch.cuda.synchronize()
+        e2e_ms = (time.perf_counter() - t0) * 1e3 / args.e2e_steps
+        t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+        if world > 1:
+            g = [torch.zeros_like(t) for _ in range(world)]
+            dist.all_gather(g, t)
+            e2e_max = max(float(x) for x in g)
+        else:
+            e2e_max = e2e_ms
+        e2e = {"ms": e2e_max, "d2h": d2h // args.e2e_steps, "h2d": h2d // args.e2e_steps}
 
-    fix_ns = [s["fixpoint_ns"] for s in stats]
-    alg = counted["alg_bytes"]
-    dense = counted["dense_bytes"]
-    visits = stats[-1]["node_visits"]
-    rec = torch.tensor([my_ms, e2e_mine, float(n_apps), float(visits), float(nodes),
-                        float(statistics.mean(fix_ns)), float(alg)], dtype=torch.float64,
-                       device="cuda")
-    if world > 1:                                         # NCCL gather of per-rank records
-        gathered = [torch.zeros_like(rec) for _ in range(world)]
-        dist.all_gather(gathered, rec)
-        dig = torch.tensor(digests.view(np.int64), device="cuda")
-        dig_all = [torch.zeros_like(dig) for _ in range(world)]
-        dist.all_gather(dig_all, dig)
-        recs = torch.stack(gathered).cpu().numpy()
-    else:
-        recs = rec.unsqueeze(0).cpu().numpy()
     if rank != 0:
+        barrier()
         if world > 1:
             dist.destroy_process_group()
         return
 
-    max_ms = float(recs[:, 0].max())
-    total_apps = float(recs[:, 2].sum())
+    tot = corpus.combine(recs)
+    max_ms = max(r["wall_ns"] for r in recs) / 1e6
+    total_apps = tot["apps"]
     ms_step = max_ms / args.steps
     value = total_apps * args.steps / (max_ms / 1e3)
-    e2e_max = float(recs[:, 1].max())
-    fix_ms = statistics.mean(fix_ns) / 1e6
     peak, peak_src = measured_peak()
-    achieved = alg / (statistics.mean(fix_ns) / 1e9) / 1e9     # GB/s, touched-word model
-    traffic, traffic_wl = ncu_traffic(args.workload, desc["apps_per_rank"])
-    clocks = clk.summary()
+    achieved = alg / (fix_ns / 1e9) / 1e9 if fix_ns else 0.0
+    traffic, traffic_wl = ncu_traffic(args.workload)
+    parity = None
+    if args.workload.startswith("corpus") and os.path.exists(CORPUS_CACHE):
+        cache = json.load(open(CORPUS_CACHE))
+        parity = corpus.check_digests(dig_all, dig_mask, cache["apps"]) if \
+            cache.get("gen_version") == __import__("synth").generator.GEN_VERSION else {"stale_cache": True}
+    pct = lambda xs, q: float(np.percentile(np.asarray(xs), q)) if xs else None
     line = {
         "metric": METRIC, "value": value, "unit": "apps/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_step,
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+        "higher_is_better": True, "scaling": scaling, "vs_baseline": None, "dtype": "u64",
         "data": "synthetic (seeded generator, Android-app-shaped ICFGs)",
-        "config": {**{k: v for k, v in desc.items() if k != "app_ids"},
-                   "nodes_per_rank": nodes, "input_bytes_per_rank": input_bytes,
-                   "fact_store_bytes_per_rank": stats[-1]["fact_bytes"],
-                   "l2": "fact store > L2 (126 MB) per step; re-zeroed each step",
-                   "parallelism": f"apps sharded over {world} GPU(s), no data-path collective",
-                   "loop_mode": args.loop_mode, "variant": args.variant},
+        "config": {**desc, "batches_per_rank": [len(b) for b in plan.batches],
+                   "nodes_rank0": nodes, "input_bytes_rank0": shard.input_bytes,
+                   "l2": "fact stores > L2 (126 MB) per batch; re-zeroed each build",
+                   "parallelism": f"apps sharded over {world} GPU(s), no data-path collective"},
         "ms_per_app": ms_step / (total_apps / world),
-        "node_visits_per_s": float(recs[:, 3].sum()) * args.steps / (max_ms / 1e3),
-        "rounds_per_step": stats[-1]["rounds"],
-        "fixpoint_ms_per_step": fix_ms,
-        "gpu_launches": int(stats[-1]["kernel_launches"]) * args.steps,
+        "node_visits_per_s": tot["visits"] * args.steps / (max_ms / 1e3),
+        "app_ms_rank0": {"p50": pct(app_ms, 50), "p90": pct(app_ms, 90), "p99": pct(app_ms, 99),
+                         "max": max(app_ms) if app_ms else None,
+                         "note": "an app's share of its batch's build time (apps of a batch share rounds), by node fraction"},
+        "batch_ms_rank0": {"n": len(batch_ms), "sum": sum(batch_ms), "max": max(batch_ms),
+                           "wide": sum(ms for b, ms in zip(my_batches, batch_ms) if plan.wide[b[0]])},
+        "rounds_rank0": sum(s["rounds"] for s in stats),
+        "fixpoint_ms_per_step_rank0": fix_ns / 1e6,
+        "gpu_launches": launches * args.steps,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "kernel": "k_fixpoint",
-                     "bytes_model": "touched-word (SURVEY §8(d)); per launch = one step's fixed point (1-3 k_fixpoint launches under the hybrid light/heavy schedule, DESIGN.md §5.4; achieved = bytes / their summed CUDA-event time, traffic = ncu DRAM bytes summed over them); counted by one untimed build with the counting kernel instantiation, timed launches run without the counters",
+                     "bytes_model": "touched-word (SURVEY §8(d)), counted on the device by one untimed "
+                                    "build of every batch with the counting instantiation; per launch = one "
+                                    "step's k_fixpoint launches summed (achieved = bytes / their summed "
+                                    "CUDA-event time; traffic = ncu DRAM bytes of the same launches)",
                      "alg_bytes_per_launch": alg, "dense_bytes_per_launch": dense,
-                     "dense_achieved": dense / (statistics.mean(fix_ns) / 1e9) / 1e9,
+                     "dense_achieved": dense / (fix_ns / 1e9) / 1e9 if fix_ns else 0.0,
                      "peak_source": peak_src, "traffic_workload": traffic_wl},
-        "e2e": {"value": total_apps / (e2e_max / 1e3), "unit": "apps/s",
-                "h2d_bytes_per_step": input_bytes, "d2h_bytes_per_step": 8 * n_apps + 128,
-                "ms_per_step": e2e_max,
-                "pipeline": "double-buffered: load of step i+1 overlaps build of step i",
-                "breakdown_ms": dict(zip(("load", "wait+build+readback"),
-                                         [round(x, 2) for x in e2e_parts[0][:2]]))
-                                if e2e_parts else None},
+        "parity": parity,
         "clocks": clocks,
     }
+    if e2e:
+        line["e2e"] = {"value": total_apps / (e2e["ms"] / 1e3), "unit": "apps/s",
+                       "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
+                       "ms_per_step": e2e["ms"], "readback": args.e2e_readback,
+                       "pipeline": "loader thread: generate-free host tables + pinned H2D of batch i+1 "
+                                   "overlapped with build + gdroid_read_all_facts of batch i"}
+    if not args.no_per_config and args.workload == "corpus1000":
+        line["per_config"] = per_config_runs(local, stream.cuda_stream)
     if not args.no_cpu_baseline:
         import oracle
         oracle.build()
-        s = oracle_sample(apps, args.cpu_seconds)
-        line["cpu_baseline"] = {"value": s["apps"] / s["wall_s"], "unit": "apps/s", "cores": 1,
-                                "kind": "oracle",
-                                "sample": f"{s['apps']} oracle run(s) over rank 0's {len(apps)} app(s), "
-                                          f"single-threaded ({s['wall_s']:.1f} s)",
-                                "node_visits_per_s": s["visits"] / s["wall_s"]}
+        P = host_threads()
+        ids = oracle_sample_ids(plan, None, ORACLE_NODES_PER_CORE_S * P * args.cpu_seconds)
+        sample_apps = [apps[i] if i in apps else make_app(i) for i in ids]
+        if not sample_apps and not plan.wide[my_ids[0]]:
+            ids, sample_apps = [my_ids[0]], [apps[my_ids[0]]]
+    if not args.no_cpu_baseline and not sample_apps:
+        line["cpu_baseline"] = {"value": None, "unit": "apps/s", "cores": P, "kind": "oracle",
+                                "sample": "not timed: a worst-shaped app takes ~800 s of one core "
+                                          "(tests/golden/oracle_digests.json records the oracle's time)"}
+    elif not args.no_cpu_baseline:
+        wall, osec, ovis, odig = oracle_pool(sample_apps, P)
+        ok = sum(1 for i, d in zip(ids, odig) if i in res.digests and d == res.digests[i])
+        line["cpu_baseline"] = {
+            "value": len(sample_apps) / wall, "unit": "apps/s", "cores": P, "kind": "oracle",
+            "cpu_model": cpu_model(),
+            "sample": f"{len(sample_apps)} apps ({sum(a.n_nodes for a in sample_apps)} nodes), a size-stratified "
+                      f"sample of the workload's narrow apps, oracle on {P} host threads, {wall:.1f} s wall; "
+                      f"the {sum(plan.wide)} worst-shaped apps are not in the timed sample",
+            "node_visits_per_s": ovis / wall, "digests_equal_gpu": f"{ok}/{len(ids)}"}
     print(json.dumps(line), flush=True)
+    barrier()
     if world > 1:
         dist.destroy_process_group()
 

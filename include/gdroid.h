@@ -33,7 +33,7 @@
 extern "C" {
 #endif
 
-#define GDROID_ABI_VERSION 1u
+#define GDROID_ABI_VERSION 2u   /* 2: gdroid_build_opts.release_facts, gdroid_release_facts */
 
 typedef enum {
   GDROID_OK = 0,
@@ -92,9 +92,9 @@ typedef struct {
 
 /* Build options; an all-zero struct (or NULL) means defaults. */
 typedef struct {
-  uint32_t async;        /* 1: enqueue only, complete with gdroid_sync (narrow batches of
-                            >= 2^17 nodes with the default variant still wait on the stream
-                            at each light/heavy hand-over)                   */
+  uint32_t async;        /* 1: enqueue only, complete with gdroid_sync.  The light/heavy
+                            hand-overs of large narrow batches are decided
+                            on the device, so nothing in a build waits on the host.        */
   uint32_t max_rounds;   /* 0 = unlimited                                                   */
   uint32_t blocks;       /* persistent-kernel CTAs (0 = SMs x occupancy)                     */
   uint32_t loop_mode;    /* 0 = persistent cooperative kernel (default), 1 = host-launched
@@ -106,6 +106,12 @@ typedef struct {
                             and atomics of the stats are then 0); rounds and visits are
                             always counted.  A separate kernel instantiation without the
                             counting code (fewer instructions per visit).                  */
+  uint32_t release_facts;/* 1: after the digests, return the fact store to the device's
+                            stream-ordered memory pool (gdroid_release_facts); the digests
+                            stay readable, the facts do not (GDROID_E_STATE) until the next
+                            build re-allocates and rebuilds them.  Lets a corpus keep every
+                            app's tables resident while only the batch being built holds a
+                            fact store.                                       */
 } gdroid_build_opts;
 
 /* Variants (Fig. 8-12), recast on B200:
@@ -160,6 +166,11 @@ gdroid_status gdroid_load_icfg_plain(const gdroid_icfg_desc* desc, int device, v
 gdroid_status gdroid_build_idfg(gdroid_app* app, const gdroid_build_opts* opts,
                                 gdroid_build_stats* stats);
 gdroid_status gdroid_sync(gdroid_app* app, gdroid_build_stats* stats);
+/* Free the handle's fact store (stream-ordered, cudaFreeAsync on the handle's stream; the
+ * library raises the device pool's release threshold so the memory stays reserved for the
+ * next allocation).  Tables, digests and stats remain; gdroid_read_* return GDROID_E_STATE
+ * until the next gdroid_build_idfg, which re-allocates the store.  Idempotent. */
+gdroid_status gdroid_release_facts(gdroid_app* app);
 /* Facts of one node of app k as strictly ascending (slot_gid << 32 | inst_gid).
  * pairs == NULL: size query.  cap < needed: GDROID_E_SMALLBUF with *n_pairs set. */
 gdroid_status gdroid_read_facts(const gdroid_app* app, uint32_t node, uint64_t* pairs,
@@ -172,6 +183,9 @@ gdroid_status gdroid_read_all_facts(const gdroid_app* app, uint32_t k, uint64_t*
 /* Per-node digests d(n) = sum over IN(n) of mix64(mix64(n) ^ pair),
  * computed on the device at the end of the build; per_node may be NULL. */
 gdroid_status gdroid_node_digests(const gdroid_app* app, uint64_t* per_node, uint64_t* app_digest);
+/* The same for app k of a batch: per_node[n_nodes(k)] indexed by the app's own node ids. */
+gdroid_status gdroid_node_digests_in(const gdroid_app* app, uint32_t k, uint64_t* per_node,
+                                     uint64_t* app_digest);
 gdroid_status gdroid_app_digests(const gdroid_app* app, uint64_t* per_app /* [n_apps] */);
 uint32_t      gdroid_n_apps(const gdroid_app* app);
 /* Diagnostics: record a per-round trace in the next builds (cap rounds, 0 = off), then read

@@ -158,6 +158,24 @@ def build_idfg(g, order: int = 0, seed: int = 0) -> OracleResult:
     return r
 
 
+def run_timed(g, order: int = 0):
+    """The oracle's fixed point with only (seconds, visits, app digest) returned — no pair
+    copy-out; used by bench.py's cpu_baseline / --impl reference legs (thread pools: the
+    ctypes call releases the GIL and the oracle keeps no shared mutable state)."""
+    L = lib()
+    d, keep = _desc(g)
+    h = C.c_void_p()
+    rc = L.oracle_build(C.byref(d), order, 0, C.byref(h))
+    if rc != 0:
+        raise OracleError(rc, L.oracle_last_error().decode())
+    try:
+        app = C.c_uint64(0)
+        L.oracle_digests(h, None, C.byref(app))
+        return float(L.oracle_seconds(h)), int(L.oracle_visits(h)), int(app.value)
+    finally:
+        L.oracle_free(h)
+
+
 def check_postfix(g, r: OracleResult) -> int:
     d, keep = _desc(g)
     return int(lib().oracle_check_postfix(C.byref(d), r._h))

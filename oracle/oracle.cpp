@@ -483,114 +483,37 @@ uint64_t oracle_check_postfix(const oracle_icfg* g, const oracle_result* r) {
   return bad;
 }
 
+// Round-synchronous (BSP) variant of Alg. 1 for the Fig. 2 pin (reading A12): every round
+// processes the whole current list in order; successors that grew or were never reached (A5)
+// form the next list, each once.  Same fixed point as the FIFO worklist.
 int64_t oracle_bsp_rounds(const oracle_icfg* g, uint32_t* seq, uint64_t cap, uint32_t* lens, uint64_t lens_cap) {
-  uint64_t visits = 0;
-  return oracle_bsp_rounds_policy(g, 0, seq, cap, lens, lens_cap, &visits);
-}
-
-// BSP rounds with a scheduling policy (experiments; results are policy-independent):
-// 0 = process the whole current list; 1 = defer a node to the next round when one of its
-// predecessors with a smaller node id is also in the current list (MER-style postponement,
-// PAPER.md:1039-1082; the smallest id of a list is never deferred, so progress is guaranteed).
-int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq, uint64_t cap, uint32_t* lens,
-                                 uint64_t lens_cap, uint64_t* visits) {
   Universe U;
   U.init(g);
   int rc = validate(U);
   if (rc) return rc;
   const uint32_t N = g->n_nodes;
-  std::vector<std::vector<uint32_t>> preds(N);
-  for (uint32_t p = 0; p < N; ++p)
-    for (uint64_t e = g->row_ptr[p]; e < g->row_ptr[p + 1]; ++e) preds[g->col[e]].push_back(p);
-  // policy 3 (| window << 8): priority window.  prio(n) = reverse-postorder index of a DFS from
-  // the component entries; a round processes only the listed nodes with prio < min_c + window,
-  // min_c = smallest prio listed in the node's component; the rest are carried over.
-  const int pol = policy & 0xff;
-  const uint32_t window = (uint32_t)policy >> 8;
-  std::vector<uint32_t> prio((pol == 3 || pol == 4) ? N : 0, 0), comp((pol == 3 || pol == 4) ? N : 0, 0);
-  if ((pol == 3 || pol == 4)) {
-    std::vector<uint32_t> post;
-    std::vector<char> seen(N, 0);
-    std::vector<std::pair<uint32_t, uint64_t>> st;
-    for (uint32_t i = 0; i < g->n_entries; ++i) {
-      const uint32_t e = g->entries[i];
-      if (seen[e]) continue;
-      seen[e] = 1;
-      comp[e] = i;
-      st.push_back({e, g->row_ptr[e]});
-      while (!st.empty()) {
-        auto& top = st.back();
-        if (top.second < g->row_ptr[top.first + 1]) {
-          const uint32_t s = g->col[top.second++];
-          if (!seen[s]) { seen[s] = 1; comp[s] = i; st.push_back({s, g->row_ptr[s]}); }
-        } else {
-          post.push_back(top.first);
-          st.pop_back();
-        }
-      }
-    }
-    for (size_t k2 = 0; k2 < post.size(); ++k2) prio[post[k2]] = (uint32_t)(post.size() - 1 - k2);
-    if (pol == 4) for (uint32_t n = 0; n < N; ++n) prio[n] = n;   // policy 4: node id order
-  }
-  std::vector<uint32_t> cmin((pol == 3 || pol == 4) ? g->n_entries : 0, 0xffffffffu);
   std::vector<PairSet> IN(N);
-  std::vector<char> visited(N, 0), in_next(N, 0), in_cur(N, 0);
+  std::vector<char> visited(N, 0), in_next(N, 0);
   std::vector<uint32_t> cur, nxt;
   for (uint32_t i = 0; i < g->n_entries; ++i)
     if (std::find(cur.begin(), cur.end(), g->entries[i]) == cur.end()) cur.push_back(g->entries[i]);
   uint64_t k = 0;
   int64_t rounds = 0;
-  *visits = 0;
   while (!cur.empty()) {
     if ((uint64_t)rounds < lens_cap) lens[rounds] = (uint32_t)cur.size();
-    if (pol != 2 && pol != 5) for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
+    for (uint32_t n : cur) { if (k < cap) seq[k] = n; ++k; }
     ++rounds;
     nxt.clear();
-    uint32_t max_depth = 0;
-    for (uint32_t n : cur) in_cur[n] = 1;
-    std::vector<uint32_t> cont_round((pol == 2 || pol == 5) ? N : 0, 0);
-    if ((pol == 3 || pol == 4)) {
-      for (uint32_t n : cur) cmin[comp[n]] = 0xffffffffu;
-      for (uint32_t n : cur) cmin[comp[n]] = std::min(cmin[comp[n]], prio[n]);
-    }
-    for (uint32_t n0 : cur) {
-      bool defer = false;
-      if (pol == 1)
-        for (uint32_t p : preds[n0]) if (p < n0 && in_cur[p]) { defer = true; break; }
-      if ((pol == 3 || pol == 4)) defer = prio[n0] >= cmin[comp[n0]] + window;
-      if (defer) {
-        if (!in_next[n0]) { nxt.push_back(n0); in_next[n0] = 1; }
-        continue;
-      }
-      // policy 2: continue depth-first into a grown successor of a single-successor node
-      uint32_t n = n0;
-      const int max_dep = (pol == 2 || pol == 5) && window ? (int)window : 64;
-      for (int depth = 0; depth < max_dep; ++depth) {
-        visited[n] = 1;
-        ++*visits;
-        PairSet Y = transfer(U, n, IN[n]);
-        int64_t cont = -1;
-        for (uint64_t e = g->row_ptr[n]; e < g->row_ptr[n + 1]; ++e) {
-          uint32_t s = g->col[e];
-          PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
-          bool grew = merge_union(IN[s], Z);
-          if (!(grew || !visited[s])) continue;
-          if ((pol == 2 || pol == 5) && cont < 0 && depth + 1 < max_dep &&
-              (pol == 5 || g->row_ptr[n + 1] - g->row_ptr[n] == 1) && !in_cur[s] &&
-              cont_round[s] != (uint32_t)rounds) {
-            cont_round[s] = (uint32_t)rounds;
-            cont = s;
-            continue;
-          }
-          if (!in_next[s]) { nxt.push_back(s); in_next[s] = 1; }
-        }
-        if (depth + 1 > (int)max_depth) max_depth = depth + 1;
-        if (cont < 0) break;
-        n = (uint32_t)cont;
+    for (uint32_t n : cur) {
+      visited[n] = 1;
+      PairSet Y = transfer(U, n, IN[n]);
+      for (uint64_t e = g->row_ptr[n]; e < g->row_ptr[n + 1]; ++e) {
+        uint32_t s = g->col[e];
+        PairSet Z = edge_transform(U, n, s, g->edge_kind[e], Y);
+        bool grew = merge_union(IN[s], Z);
+        if ((grew || !visited[s]) && !in_next[s]) { nxt.push_back(s); in_next[s] = 1; }
       }
     }
-    if ((pol == 2 || pol == 5) && (uint64_t)(rounds - 1) < cap) seq[rounds - 1] = max_depth;   // chain depth
-    for (uint32_t n : cur) in_cur[n] = 0;
     for (uint32_t s : nxt) in_next[s] = 0;
     cur.swap(nxt);
   }

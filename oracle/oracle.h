@@ -64,10 +64,6 @@ uint64_t oracle_check_postfix(const oracle_icfg* g, const oracle_result* r);
 int64_t oracle_bsp_rounds(const oracle_icfg* g, uint32_t* seq, uint64_t cap,
                           uint32_t* lens, uint64_t lens_cap);
 
-/* Same with a scheduling policy (0 = all, 1 = defer nodes with a smaller-id predecessor in the
- * current list); *visits = nodes processed.  The fixed point is policy-independent. */
-int64_t oracle_bsp_rounds_policy(const oracle_icfg* g, int policy, uint32_t* seq, uint64_t cap,
-                                 uint32_t* lens, uint64_t lens_cap, uint64_t* visits);
 
 /* Fig. 7 MER primitive: given the current worklist wl[0..n) and the
  * destinations dst[0..nd) produced by processing its head list, form the next worklist:

@@ -14,7 +14,7 @@ import numpy as np
 
 from ._build import LIB
 
-ABI_VERSION = 1
+ABI_VERSION = 2
 STATUS = {0: "OK", -1: "E_INVALID", -2: "E_POOL", -3: "E_OOM", -4: "E_CUDA", -5: "E_STATE",
           -6: "E_RANGE", -7: "E_SMALLBUF", -8: "E_LIMIT"}
 
@@ -33,7 +33,8 @@ class IcfgDesc(C.Structure):
 
 class BuildOpts(C.Structure):
     _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
-                ("loop_mode", C.c_uint32), ("variant", C.c_uint32), ("no_byte_model", C.c_uint32)]
+                ("loop_mode", C.c_uint32), ("variant", C.c_uint32), ("no_byte_model", C.c_uint32),
+                ("release_facts", C.c_uint32)]
 
 
 class BuildStats(C.Structure):
@@ -79,10 +80,12 @@ def lib():
             L.gdroid_load_icfg_plain.restype = C.c_int
         L.gdroid_build_idfg.argtypes = [P, P, P]
         L.gdroid_sync.argtypes = [P, P]
+        L.gdroid_release_facts.argtypes = [P]
         L.gdroid_read_facts.argtypes = [P, C.c_uint32, P, C.c_uint64, P]
         L.gdroid_read_facts_in.argtypes = [P, C.c_uint32, C.c_uint32, P, C.c_uint64, P]
         L.gdroid_read_all_facts.argtypes = [P, C.c_uint32, P, P, C.c_uint64]
         L.gdroid_node_digests.argtypes = [P, P, P]
+        L.gdroid_node_digests_in.argtypes = [P, C.c_uint32, P, P]
         L.gdroid_app_digests.argtypes = [P, P]
         L.gdroid_n_apps.argtypes = [P]
         L.gdroid_n_apps.restype = C.c_uint32
@@ -96,9 +99,9 @@ def lib():
         L.gdroid_free.restype = None
         L.gdroid_last_error.restype = C.c_char_p
         L.gdroid_abi_version.restype = C.c_uint32
-        for f in ("gdroid_load_batch", "gdroid_load_icfg", "gdroid_build_idfg", "gdroid_sync",
+        for f in ("gdroid_load_batch", "gdroid_load_icfg", "gdroid_build_idfg", "gdroid_sync", "gdroid_release_facts",
                   "gdroid_read_facts", "gdroid_read_facts_in", "gdroid_read_all_facts",
-                  "gdroid_node_digests", "gdroid_app_digests"):
+                  "gdroid_node_digests", "gdroid_node_digests_in", "gdroid_app_digests"):
             getattr(L, f).restype = C.c_int
         _lib = L
     return _lib
@@ -157,15 +160,20 @@ class App:
         self.stats: Optional[dict] = None
 
     def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
-              asynchronous: bool = False, variant=0, byte_model: bool = True) -> Optional[dict]:
+              asynchronous: bool = False, variant=0, byte_model: bool = True,
+              release_facts: bool = False) -> Optional[dict]:
         o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant),
-                      0 if byte_model else 1)
+                      0 if byte_model else 1, 1 if release_facts else 0)
         s = BuildStats()
         _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
         if asynchronous:
             return None
         self.stats = s.as_dict()
         return self.stats
+
+    def release_facts(self):
+        """gdroid_release_facts: return the fact store to the device pool (digests stay)."""
+        _check(lib().gdroid_release_facts(self._h))
 
     def sync(self) -> dict:
         s = BuildStats()
@@ -181,19 +189,24 @@ class App:
         _check(L.gdroid_read_facts_in(self._h, k, node, _ptr(out), cnt.value, C.byref(cnt)))
         return out[:cnt.value]
 
-    def read_all_facts(self, k: int = 0) -> Tuple[np.ndarray, np.ndarray]:
+    def read_all_facts(self, k: int = 0, ptr_out: Optional[np.ndarray] = None,
+                       pairs_buf=None) -> Tuple[np.ndarray, np.ndarray]:
+        """All facts of app k (CSR ptr[n_nodes+1], pairs).  ptr_out: a caller uint64 array of
+        n_nodes+1; pairs_buf: an object with .get(n) -> uint64 array of n (e.g. a reusable
+        pinned buffer), else fresh numpy arrays."""
         L = lib()
-        ptr = np.zeros(self.n_nodes[k] + 1, dtype=np.uint64)
+        ptr = ptr_out if ptr_out is not None else np.zeros(self.n_nodes[k] + 1, dtype=np.uint64)
+        assert ptr.dtype == np.uint64 and ptr.size == self.n_nodes[k] + 1 and ptr.flags.c_contiguous
         _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), None, 0))
         tot = int(ptr[-1])
-        pairs = np.zeros(max(tot, 1), dtype=np.uint64)
-        _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), _ptr(pairs), tot))
+        pairs = pairs_buf.get(tot) if pairs_buf is not None else np.zeros(max(tot, 1), dtype=np.uint64)[:tot]
+        _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), _ptr(pairs) if tot else None, tot))
         return ptr, pairs[:tot]
 
-    def node_digests(self) -> Tuple[np.ndarray, int]:
-        per = np.zeros(self.n_nodes[0], dtype=np.uint64)
+    def node_digests(self, k: int = 0) -> Tuple[np.ndarray, int]:
+        per = np.zeros(self.n_nodes[k], dtype=np.uint64)
         app = C.c_uint64(0)
-        _check(lib().gdroid_node_digests(self._h, _ptr(per), C.byref(app)))
+        _check(lib().gdroid_node_digests_in(self._h, k, _ptr(per), C.byref(app)))
         return per, int(app.value)
 
     def app_digests(self) -> np.ndarray:

@@ -15,13 +15,28 @@ FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std
          "-shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v"]
 
 
+FLAGS_FILE = LIB + ".flags"     # the extra nvcc flags the in-tree library was built with
+
+
+def _built_flags():
+    try:
+        with open(FLAGS_FILE) as fh:
+            return fh.read().strip()
+    except OSError:
+        return None
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Rebuild when a source is newer than the library OR the library was built with other
+    extra flags (GDROID_NVCC_FLAGS, used by A/B scripts) than the ones requested now, so an A/B
+    variant left in the tree is never reused by a default build."""
     newest = max(os.path.getmtime(p) for p in DEPS)
-    force = force or bool(os.environ.get("GDROID_NVCC_FLAGS"))
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest:
+    extra = os.environ.get("GDROID_NVCC_FLAGS", "").split()
+    want = " ".join(extra)
+    if (not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= newest
+            and _built_flags() == want):
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
-    extra = os.environ.get("GDROID_NVCC_FLAGS", "").split()
     cmd = [NVCC, *FLAGS, *extra, "-I", os.path.join(ROOT, "include"), "-o", tmp, *SOURCES]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
@@ -31,6 +46,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     with open(os.path.join(HERE, "ptxas_info.txt"), "w") as fh:
         fh.write(r.stderr)
     os.replace(tmp, LIB)
+    with open(FLAGS_FILE, "w") as fh:
+        fh.write(want + "\n")
     return LIB
 
 

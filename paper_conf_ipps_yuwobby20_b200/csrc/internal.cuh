@@ -185,7 +185,8 @@ struct Dev {
   uint32_t wide;                // max log2(words per row) over the batch's modules: 0 = all narrow,
                                 // >= 1: some module has > 64 instances (row-occupancy path)
   uint32_t hiocc;               // 1: launch the 4-CTA/SM narrow instantiation (batches >= HIOCC_NODES)
-  uint32_t round0;              // first round of this launch (hybrid launches resume mid-build)
+  uint32_t round0;              // first round of this launch (non-hybrid: 1)
+  uint32_t hyb;                 // 1: hybrid launch sequence: start at round bar[3], return if it is 0
   uint32_t sw_lo, sw_hi;        // hybrid: leave at the start of a round with < sw_lo / >= sw_hi items
                                 // (bar[3] = that round), 0 = off
   uint32_t flags;               // F_* scheduling switches of the build (ablation variants)

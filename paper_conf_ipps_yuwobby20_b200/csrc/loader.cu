@@ -1015,6 +1015,54 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
 
 size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
 
+// Pinned, portable host slots for the per-build stats readback, recycled across handles: the
+// D2H copy at the end of a build is then truly asynchronous (a pageable destination would make
+// cudaMemcpyAsync return only after the build), and gdroid_free needs no cudaFreeHost (which
+// would synchronise the device).  Slabs live for the process.
+struct StatsSlots {
+  std::mutex m;
+  std::vector<DevStats*> free_;
+  DevStats* get() {
+    std::lock_guard<std::mutex> lk(m);
+    if (free_.empty()) {
+      constexpr int SLAB = 64;
+      void* p = nullptr;
+      if (cudaHostAlloc(&p, SLAB * sizeof(DevStats), cudaHostAllocPortable) != cudaSuccess) return nullptr;
+      for (int i = SLAB - 1; i >= 0; --i) free_.push_back((DevStats*)p + i);
+    }
+    DevStats* r = free_.back();
+    free_.pop_back();
+    *r = DevStats{};
+    return r;
+  }
+  void put(DevStats* p) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(m);
+    free_.push_back(p);
+  }
+};
+// Raise the release threshold of the device's default memory pool once, so fact stores freed
+// with cudaFreeAsync (gdroid_release_facts) stay reserved and the next cudaMallocAsync of a
+// batch reuses them without an OS allocation.
+void keep_pool_reserved(int device) {
+  static std::mutex m;
+  static std::vector<char> done;
+  std::lock_guard<std::mutex> lk(m);
+  if ((int)done.size() <= device) done.resize(device + 1, 0);
+  if (done[device]) return;
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t thr = ~0ull;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  }
+  done[device] = 1;
+}
+
+StatsSlots& stats_slots() {
+  static StatsSlots* s = new StatsSlots();   // never destroyed (pinned slabs outlive static teardown)
+  return *s;
+}
+
 }  // namespace
 
 struct gdroid_app {
@@ -1024,10 +1072,11 @@ struct gdroid_app {
   std::vector<uint32_t> app_base;     // [n_apps+1] global node id ranges
   Dev D{};
   void* d_tables = nullptr;
-  uint64_t* d_facts = nullptr;
+  uint64_t* d_facts = nullptr;        // nullptr after gdroid_release_facts (re-allocated by build)
+  uint64_t fact_alloc_bytes = 0;
   void* d_state = nullptr;            // stamp, queue, counts, stats, bar, digests
   uint32_t cls_count[NCLS] = {};      // work items per GRP class (queue segment sizes)
-  DevStats* h_stats = nullptr;        // pinned
+  DevStats* h_stats = nullptr;        // pinned slot (StatsSlots)
   uint64_t* d_scratch = nullptr;
   size_t scratch_bytes = 0;
   cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
@@ -1035,10 +1084,10 @@ struct gdroid_app {
   uint64_t h2d_ns = 0;
   uint64_t launches = 0;
   bool built = false, pending = false;
+  bool digests_ok = false;            // a build completed (digests readable even if facts released)
+  bool release_pending = false;
   int max_blocks = 0;
   int max_blocks_lo = 0;              // hybrid (large narrow batches): grid of the 3-CTA/SM instantiation
-  uint32_t h_bar[4] = {0, 0, 0, 0};   // readback of the barrier words (hybrid hand-over; pageable:
-                                      // a per-handle pinned block would make gdroid_free synchronise)
   // PLAIN variant (plain.cu): set-based state, present when loaded with gdroid_load_icfg_plain
   PlainDev P{};
   void* d_plain = nullptr;            // uploaded inputs + sets, locks, stamps, queues, scratch, heap
@@ -1059,7 +1108,8 @@ void free_app(gdroid_app* a) {
   if (a->d_scratch) cudaFree(a->d_scratch);
   if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
-  delete a->h_stats;
+  if (a->pending) cudaStreamSynchronize(a->stream);   // the stats copy targets the slot
+  stats_slots().put(a->h_stats);
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
   cudaSetDevice(cur);
@@ -1098,7 +1148,8 @@ gdroid_status finish_stats(gdroid_app* a, gdroid_build_stats* out) {
   s.kernel_launches = a->launches;
   a->last = s;
   a->pending = false;
-  a->built = true;
+  a->built = a->d_facts != nullptr;                   // released facts cannot be read back
+  a->digests_ok = true;
   if (out) *out = s;
   if (h.limit_hit) return set_err(GDROID_E_LIMIT, "max_rounds (%u) exceeded; facts are an under-approximation", a->D.max_rounds);
   return GDROID_OK;
@@ -1228,6 +1279,7 @@ gdroid_status build_plain(gdroid_app* a, const gdroid_build_opts& o, gdroid_buil
   CU(cudaMemcpyAsync(&err, P.err, 4, cudaMemcpyDeviceToHost, s));
   CU(cudaStreamSynchronize(s));
   a->pending = true;
+  a->digests_ok = false;
   a->last_plain = true;
   gdroid_status st = finish_stats(a, stats);
   a->last.fact_bytes = a->h_stats->dense_bytes;
@@ -1355,7 +1407,9 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
 
   // ---- fact store + mutable state
   {
-    cudaError_t e = cudaMallocAsync(&a->d_facts, std::max<uint64_t>(Lo.fact_words, 4) * 8, a->stream);
+    keep_pool_reserved(device);
+    a->fact_alloc_bytes = std::max<uint64_t>(Lo.fact_words, 4) * 8;
+    cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(Lo.fact_words * 8), cudaGetErrorString(e)));
     D.facts = a->d_facts;
     size_t s_mask = align256((size_t)N * 8);
@@ -1374,7 +1428,8 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     D.bar = (uint32_t*)S; S += s_bar;
     D.node_digest = (uint64_t*)S; S += s_nd;
     D.app_digest = (unsigned long long*)S;
-    a->h_stats = new DevStats();
+    a->h_stats = stats_slots().get();
+    if (!a->h_stats) return fail(set_err(GDROID_E_OOM, "pinned stats slot"));
     for (auto& ev : a->ev)
       if (cudaEventCreate(&ev) != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "cudaEventCreate failed"));
   }
@@ -1415,6 +1470,11 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   const uint32_t N = D.n_nodes;
   uint32_t blocks = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks) : (uint32_t)a->max_blocks;
   a->launches = 0;
+  if (!a->d_facts) {                                  // released by an earlier build: re-allocate
+    const cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, s);
+    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e));
+    D.facts = a->d_facts;
+  }
   CU(cudaEventRecord(a->ev[0], s));
   // (a2) zero the fact matrices and the worklist state
   CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
@@ -1434,27 +1494,25 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
     // instantiation with narrow continuation, heavy rounds (>= 4 waves of items) in the 4-CTA/SM
     // one; a launch leaves at the first round of the other kind (bar[3] = that round) and the
     // next launch resumes there.  At most HYB_SWITCHES hand-overs per build.
+    // The hand-over is device-side: every launch of the alternating sequence is enqueued up
+    // front (no host round trip); a launch starts at the round in bar[3] (k_seed sets 1) and
+    // returns at once when bar[3] = 0 (an earlier launch reached the fixed point or the limit).
     uint32_t blocks_lo = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks_lo) : (uint32_t)a->max_blocks_lo;
     const uint32_t nw_lo = blocks_lo * (THREADS / 32);
     bool heavy = false;
-    for (uint32_t sw = 0;; ++sw) {
-      const bool last = sw >= HYB_SWITCHES;
+    D.hyb = 1u;
+    for (uint32_t sw = 0; sw <= HYB_SWITCHES; ++sw) {
+      const bool last = sw == HYB_SWITCHES;
       D.sw_lo = (heavy && !last) ? GD_HYB_LO * nw_lo / 4u : 0u;
       D.sw_hi = (!heavy && !last) ? GD_HYB_HI * nw_lo / 4u : 0u;
       D.hiocc = heavy ? 1u : 0u;
-      CU(cudaMemsetAsync(D.bar + 3, 0, 4, s));
       const cudaError_t e = launch_fixpoint(D, heavy ? blocks : blocks_lo, s);
       D.hiocc = 1u;
-      if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "k_fixpoint: %s", cudaGetErrorString(e));
+      if (e != cudaSuccess) { D.hyb = 0u; return set_err(GDROID_E_CUDA, "k_fixpoint: %s", cudaGetErrorString(e)); }
       a->launches++;
-      if (last) break;
-      CU(cudaMemcpyAsync(a->h_bar, D.bar, 16, cudaMemcpyDeviceToHost, s));
-      CU(cudaStreamSynchronize(s));
-      if (a->h_bar[3] == 0) break;                 // finished (empty worklist or round limit)
-      D.round0 = a->h_bar[3];
       heavy = !heavy;
     }
-    D.round0 = 1;
+    D.hyb = 0u;
     D.sw_lo = D.sw_hi = 0;
   } else if (o.loop_mode == 0) {
     CU(launch_fixpoint(D, blocks, s));
@@ -1487,6 +1545,13 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   CU(cudaMemcpyAsync(a->h_stats, D.stats, sizeof(DevStats), cudaMemcpyDeviceToHost, s));
   a->pending = true;
   a->built = false;
+  a->digests_ok = false;
+  a->release_pending = o.release_facts != 0;
+  if (o.release_facts) {                              // stream-ordered: after the digest kernel
+    CU(cudaFreeAsync(a->d_facts, s));
+    a->d_facts = nullptr;
+    D.facts = nullptr;
+  }
   if (o.async) return GDROID_OK;
   CU(cudaStreamSynchronize(s));
   return finish_stats(a, stats);
@@ -1498,6 +1563,18 @@ gdroid_status gdroid_sync(gdroid_app* a, gdroid_build_stats* stats) {
   DeviceGuard guard(a->device);
   CU(cudaStreamSynchronize(a->stream));
   return finish_stats(a, stats);
+}
+
+gdroid_status gdroid_release_facts(gdroid_app* a) {
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
+  if (!a->d_facts) return GDROID_OK;
+  DeviceGuard guard(a->device);
+  CU(cudaFreeAsync(a->d_facts, a->stream));
+  a->d_facts = nullptr;
+  a->D.facts = nullptr;
+  a->built = false;                                   // digests stay readable
+  return GDROID_OK;
 }
 
 uint32_t gdroid_n_apps(const gdroid_app* a) { return a ? a->n_apps : 0; }
@@ -1570,22 +1647,27 @@ gdroid_status gdroid_read_facts(const gdroid_app* a, uint32_t node, uint64_t* pa
   return gdroid_read_facts_in(a, 0, node, pairs, cap, n_pairs);
 }
 
-gdroid_status gdroid_node_digests(const gdroid_app* ca, uint64_t* per_node, uint64_t* app_digest) {
+gdroid_status gdroid_node_digests_in(const gdroid_app* ca, uint32_t k, uint64_t* per_node, uint64_t* app_digest) {
   gdroid_app* a = const_cast<gdroid_app*>(ca);
   if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
-  if (!a->built) return set_err(GDROID_E_STATE, "digests read before a completed build");
+  if (!a->digests_ok) return set_err(GDROID_E_STATE, "digests read before a completed build");
+  if (k >= a->n_apps) return set_err(GDROID_E_RANGE, "app index %u >= %u", k, a->n_apps);
   DeviceGuard guard(a->device);
-  const uint32_t n = a->app_base[1] - a->app_base[0];
-  if (per_node) CU(cudaMemcpyAsync(per_node, a->D.node_digest, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
-  if (app_digest) CU(cudaMemcpyAsync(app_digest, a->D.app_digest, 8, cudaMemcpyDeviceToHost, a->stream));
+  const uint32_t n0 = a->app_base[k], n = a->app_base[k + 1] - n0;
+  if (per_node) CU(cudaMemcpyAsync(per_node, a->D.node_digest + n0, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
+  if (app_digest) CU(cudaMemcpyAsync(app_digest, a->D.app_digest + k, 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));
   return GDROID_OK;
+}
+
+gdroid_status gdroid_node_digests(const gdroid_app* a, uint64_t* per_node, uint64_t* app_digest) {
+  return gdroid_node_digests_in(a, 0, per_node, app_digest);
 }
 
 gdroid_status gdroid_app_digests(const gdroid_app* ca, uint64_t* per_app) {
   gdroid_app* a = const_cast<gdroid_app*>(ca);
   if (!a || !per_app) return set_err(GDROID_E_INVALID, "NULL argument");
-  if (!a->built) return set_err(GDROID_E_STATE, "digests read before a completed build");
+  if (!a->digests_ok) return set_err(GDROID_E_STATE, "digests read before a completed build");
   DeviceGuard guard(a->device);
   CU(cudaMemcpyAsync(per_app, a->D.app_digest, (size_t)a->n_apps * 8, cudaMemcpyDeviceToHost, a->stream));
   CU(cudaStreamSynchronize(a->stream));

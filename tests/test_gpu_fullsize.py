@@ -31,10 +31,24 @@ def _mix64(z):
 
 
 def _node_hash(per_node):
+    """Order-sensitive hash of a per-node digest array (scripts/make_oracle_digests.py's
+    node_hash), vectorised: uint64 arithmetic wraps mod 2^64 like the Python original."""
+    d = np.asarray(per_node, dtype=np.uint64)
+    with np.errstate(over="ignore"):
+        z = (np.arange(len(d), dtype=np.uint64) * np.uint64(0x9E3779B97F4A7C15)) ^ d
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+        return int(z.sum(dtype=np.uint64))
+
+
+def test_node_hash_matches_python_definition():
+    rng = np.random.default_rng(5)
+    per = rng.integers(0, 2**63, size=1000, dtype=np.uint64) * np.uint64(3)
     h = 0
-    for i, d in enumerate(per_node.tolist()):
+    for i, d in enumerate(per.tolist()):
         h = (h + _mix64((i * 0x9E3779B97F4A7C15) ^ d)) & M
-    return h
+    assert _node_hash(per) == h
 
 
 def _fixture():
@@ -102,38 +116,65 @@ def test_corpus_run_shard_pipeline():
 
 
 # ---- the 1000-app corpus (BASELINE.json configs[4]) against tests/golden/corpus_digests.json
-# (written by scripts/make_corpus_digests.py, which calls only oracle/).  The clipped tail of 15
-# worst-shaped apps (|Q| = 256, ~800 s of oracle each) is covered by the `worst` preset entry.
+# (written by scripts/make_corpus_digests.py, which calls only oracle/), in the launch
+# configuration bench.py times: corpus.plan_corpus batches (narrow apps under a 4M-node
+# budget, each worst-shaped app alone) built by corpus.DeviceShard (tables resident, fact
+# store released after every build).  Every app: app digest AND the order-sensitive hash of
+# its per-node digest array (so every node's set is checked).
 CFIX = os.path.join(HERE, "golden", "corpus_digests.json")
 
 
-def _corpus_check(ids):
+def _corpus_check(ids, node_budget=4_000_000):
+    from paper_conf_ipps_yuwobby20_b200 import corpus
     if not os.path.exists(CFIX):
         pytest.skip("no stored corpus digests")
     fx = json.load(open(CFIX))
     assert fx["gen_version"] == G.GEN_VERSION
     ids = [i for i in ids if str(i) in fx["apps"]]
     assert ids
-    for b0 in range(0, len(ids), 8):
-        batch = ids[b0:b0 + 8]
-        gs = [G.corpus_app(i) for i in batch]
-        app = gd.load(gs)
-        app.build()
-        digs = app.app_digests()
-        for k, (i, g) in enumerate(zip(batch, gs)):
+    n = max(ids) + 1
+    sizes = G.corpus_sizes(n)
+    wide = [G.corpus_config(i).q_cap > 64 for i in range(n)]
+    plan = corpus.plan_corpus(sizes, wide, 1, node_budget=node_budget, app_ids=ids)
+    checked = 0
+    for b in plan.batches[0]:
+        apps = {i: G.corpus_app(i) for i in b}
+        sh = corpus.DeviceShard([b], apps)
+        sh.step()
+        sh.finish()
+        h = sh.handles[0]
+        digs = h.app_digests()
+        for k, i in enumerate(b):
             ref = fx["apps"][str(i)]
-            assert g.n_nodes == ref["n_nodes"]
+            assert apps[i].n_nodes == ref["n_nodes"]
             assert str(int(digs[k])) == ref["app_digest"], f"corpus{i}"
-        app.free()
-    return len(ids)
+            per, _ = h.node_digests(k)
+            assert str(_node_hash(per)) == ref["node_digest_hash"], f"corpus{i} per-node"
+            checked += 1
+        sh.free()
+    return checked
 
 
 def test_corpus_digest_sample():
-    """Every 20th app of the corpus (50 apps, 20K-2M nodes), in 8-app batches as bench.py runs them."""
+    """Every 20th app of the corpus (50 apps, 20K-2M nodes)."""
     assert _corpus_check(list(range(0, 1000, 20))) >= 45
 
 
-@pytest.mark.skipif(bool(os.environ.get("GDROID_QUICK")), reason="GDROID_QUICK set (about 75 s on a B200)")
+def test_corpus_wide_apps():
+    """The worst-shaped corpus apps (|Q| = 256) that the cache holds, each alone."""
+    from synth import generator as G2
+    wide = [i for i in range(1000) if G2.corpus_config(i).q_cap > 64]
+    fx = json.load(open(CFIX)) if os.path.exists(CFIX) else {"apps": {}}
+    have = [i for i in wide if str(i) in fx["apps"]]
+    if not have:
+        pytest.skip("no wide corpus apps in the cache yet")
+    if os.environ.get("GDROID_QUICK"):
+        have = have[:2]
+    assert _corpus_check(have) == len(have)
+
+
+@pytest.mark.skipif(bool(os.environ.get("GDROID_QUICK")), reason="GDROID_QUICK set (minutes on a B200)")
 def test_corpus_digest_all():
-    """All 985 narrow apps of the 1000-app corpus (profiles/r01_full_corpus_parity.log)."""
-    assert _corpus_check(list(range(1000))) == 985
+    """All 1000 apps of the corpus that the cache holds (profiles/r02_full_corpus_parity.log)."""
+    fx = json.load(open(CFIX)) if os.path.exists(CFIX) else {"apps": {}}
+    assert _corpus_check(list(range(1000))) == len(fx["apps"]) >= 985

@@ -30,7 +30,7 @@ def test_header_symbols_exported():
     assert len(names) >= 12
     for nm in names:
         assert hasattr(L, nm), nm
-    assert L.gdroid_abi_version() == 1
+    assert L.gdroid_abi_version() == 2
 
 
 def _load_status(g):
