@@ -350,12 +350,16 @@ def run_ours(args):
     # overlapped with build + fact readback of batch i
     e2e = None
     if args.e2e_steps > 0:
+        bufs = corpus.ReadbackBuffers()
+        corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback,
+                             bufs=bufs)                  # untimed warm-up: sizes the pinned buffers
         barrier()
         torch.cuda.synchronize()
         d2h = h2d = 0
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
-            out = corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback)
+            out = corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback,
+                                       bufs=bufs)
             for br in out:
                 for k, i in enumerate(br.app_ids):
                     if int(br.digests[k]) != res.digests[i]:
@@ -428,8 +432,9 @@ def run_ours(args):
         line["e2e"] = {"value": total_apps / (e2e["ms"] / 1e3), "unit": "apps/s",
                        "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
                        "ms_per_step": e2e["ms"], "readback": args.e2e_readback,
-                       "pipeline": "loader thread: generate-free host tables + pinned H2D of batch i+1 "
-                                   "overlapped with build + gdroid_read_all_facts of batch i"}
+                       "pipeline": "loader thread: host tables + pinned H2D of batch i+1 overlapped with the "
+                                   "build of batch i; gdroid_read_batch_facts of batch i (pinned) overlapped "
+                                   "with the build of batch i+1; one untimed warm-up pass sizes the buffers"}
     if not args.no_per_config and args.workload == "corpus1000":
         line["per_config"] = per_config_runs(local, stream.cuda_stream)
     if not args.no_cpu_baseline:

@@ -112,6 +112,14 @@ typedef struct {
                             build re-allocates and rebuilds them.  Lets a corpus keep every
                             app's tables resident while only the batch being built holds a
                             fact store.                                       */
+  uint32_t keep_facts;   /* 1: incremental build: the fact store keeps its
+                            content (an earlier build of this handle, or gdroid_import_facts),
+                            the worklist history persists, and the first round queues only
+                            the seeds staged with gdroid_stage_seeds (plus the entries on the
+                            handle's first build).  IN only grows, so this continues the same
+                            monotone iteration: the out-of-core sub-graph loop (§III-A1,
+                            PAPER.md:524-580) runs each sub-graph this way until no seed
+                            changes.                                                         */
 } gdroid_build_opts;
 
 /* Variants (Fig. 8-12), recast on B200:
@@ -166,6 +174,30 @@ gdroid_status gdroid_load_icfg_plain(const gdroid_icfg_desc* desc, int device, v
 gdroid_status gdroid_build_idfg(gdroid_app* app, const gdroid_build_opts* opts,
                                 gdroid_build_stats* stats);
 gdroid_status gdroid_sync(gdroid_app* app, gdroid_build_stats* stats);
+/* ---- incremental builds and out-of-core sub-graphs ----
+ * Stage seeds for the next keep_facts build of app k: for each of the n nodes (app-local ids),
+ * the pairs pairs[ptr[i] .. ptr[i+1]) (slot_gid << 32 | inst_gid, the app's gids) are OR-ed
+ * into IN(node) and the node is queued even if it gets no pair (first reach, reading A5).
+ * Arrays are read during the call.  A pair outside the node's pools makes that build return
+ * GDROID_E_POOL. */
+gdroid_status gdroid_stage_seeds(gdroid_app* app, uint32_t k, uint32_t n, const uint32_t* nodes,
+                                 const uint64_t* ptr, const uint64_t* pairs);
+/* Facts of the listed nodes of app k (app-local ids): ptr[n+1] and pairs, two-call like
+ * gdroid_read_all_facts (the boundary proxies of out-of-core sub-graphs). */
+gdroid_status gdroid_read_nodes_facts(const gdroid_app* app, uint32_t k, uint32_t n,
+                                      const uint32_t* nodes, uint64_t* ptr, uint64_t* pairs,
+                                      uint64_t cap);
+/* out[i] = 1 if node nodes[i] of app k was ever queued (reached) by the builds so far. */
+gdroid_status gdroid_read_reached(const gdroid_app* app, uint32_t k, uint32_t n,
+                                  const uint32_t* nodes, uint8_t* out);
+/* Raw copies of the whole device fact store (gdroid_fact_bytes bytes, the library's own
+ * layout) to / from caller host memory, enqueued on the handle's stream (pinned memory: an
+ * asynchronous DMA; complete with gdroid_stream_sync).  Import re-allocates a released store;
+ * a keep_facts build then continues from the imported facts. */
+gdroid_status gdroid_export_facts(const gdroid_app* app, void* host, uint64_t bytes);
+gdroid_status gdroid_import_facts(gdroid_app* app, const void* host, uint64_t bytes);
+gdroid_status gdroid_stream_sync(gdroid_app* app);
+uint64_t      gdroid_fact_bytes(const gdroid_app* app);
 /* Free the handle's fact store (stream-ordered, cudaFreeAsync on the handle's stream; the
  * library raises the device pool's release threshold so the memory stays reserved for the
  * next allocation).  Tables, digests and stats remain; gdroid_read_* return GDROID_E_STATE
@@ -180,6 +212,13 @@ gdroid_status gdroid_read_facts_in(const gdroid_app* app, uint32_t k, uint32_t n
 /* All facts of app k: ptr[n_nodes+1] and pairs (two-call: pairs == NULL fills ptr only). */
 gdroid_status gdroid_read_all_facts(const gdroid_app* app, uint32_t k, uint64_t* ptr,
                                     uint64_t* pairs, uint64_t cap);
+/* All facts of EVERY app of the batch as one CSR over the batch's nodes in load order (app k
+ * owns rows sum_{j<k} n_nodes(j) ..): ptr[N_batch+1], pairs as in gdroid_read_all_facts (each
+ * app in its own slot / instance gids).  Two-call: pairs == NULL fills ptr only (the per-node
+ * counts stay on the device for the fetch).  Pinned caller buffers give full-rate copies
+ * (Alg. 3 l.17 h_fact <- d_fact_mat). */
+gdroid_status gdroid_read_batch_facts(const gdroid_app* app, uint64_t* ptr, uint64_t* pairs,
+                                      uint64_t cap);
 /* Per-node digests d(n) = sum over IN(n) of mix64(mix64(n) ^ pair),
  * computed on the device at the end of the build; per_node may be NULL. */
 gdroid_status gdroid_node_digests(const gdroid_app* app, uint64_t* per_node, uint64_t* app_digest);

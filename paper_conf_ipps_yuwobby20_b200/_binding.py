@@ -34,7 +34,7 @@ class IcfgDesc(C.Structure):
 class BuildOpts(C.Structure):
     _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
                 ("loop_mode", C.c_uint32), ("variant", C.c_uint32), ("no_byte_model", C.c_uint32),
-                ("release_facts", C.c_uint32)]
+                ("release_facts", C.c_uint32), ("keep_facts", C.c_uint32)]
 
 
 class BuildStats(C.Structure):
@@ -81,9 +81,18 @@ def lib():
         L.gdroid_build_idfg.argtypes = [P, P, P]
         L.gdroid_sync.argtypes = [P, P]
         L.gdroid_release_facts.argtypes = [P]
+        L.gdroid_stage_seeds.argtypes = [P, C.c_uint32, C.c_uint32, P, P, P]
+        L.gdroid_read_reached.argtypes = [P, C.c_uint32, C.c_uint32, P, P]
+        L.gdroid_read_nodes_facts.argtypes = [P, C.c_uint32, C.c_uint32, P, P, P, C.c_uint64]
+        L.gdroid_export_facts.argtypes = [P, P, C.c_uint64]
+        L.gdroid_import_facts.argtypes = [P, P, C.c_uint64]
+        L.gdroid_stream_sync.argtypes = [P]
+        L.gdroid_fact_bytes.argtypes = [P]
+        L.gdroid_fact_bytes.restype = C.c_uint64
         L.gdroid_read_facts.argtypes = [P, C.c_uint32, P, C.c_uint64, P]
         L.gdroid_read_facts_in.argtypes = [P, C.c_uint32, C.c_uint32, P, C.c_uint64, P]
         L.gdroid_read_all_facts.argtypes = [P, C.c_uint32, P, P, C.c_uint64]
+        L.gdroid_read_batch_facts.argtypes = [P, P, P, C.c_uint64]
         L.gdroid_node_digests.argtypes = [P, P, P]
         L.gdroid_node_digests_in.argtypes = [P, C.c_uint32, P, P]
         L.gdroid_app_digests.argtypes = [P, P]
@@ -100,7 +109,9 @@ def lib():
         L.gdroid_last_error.restype = C.c_char_p
         L.gdroid_abi_version.restype = C.c_uint32
         for f in ("gdroid_load_batch", "gdroid_load_icfg", "gdroid_build_idfg", "gdroid_sync", "gdroid_release_facts",
-                  "gdroid_read_facts", "gdroid_read_facts_in", "gdroid_read_all_facts",
+                  "gdroid_stage_seeds", "gdroid_read_reached", "gdroid_read_nodes_facts", "gdroid_export_facts", "gdroid_import_facts",
+                  "gdroid_stream_sync",
+                  "gdroid_read_facts", "gdroid_read_facts_in", "gdroid_read_all_facts", "gdroid_read_batch_facts",
                   "gdroid_node_digests", "gdroid_node_digests_in", "gdroid_app_digests"):
             getattr(L, f).restype = C.c_int
         _lib = L
@@ -161,15 +172,54 @@ class App:
 
     def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
               asynchronous: bool = False, variant=0, byte_model: bool = True,
-              release_facts: bool = False) -> Optional[dict]:
+              release_facts: bool = False, keep_facts: bool = False) -> Optional[dict]:
         o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant),
-                      0 if byte_model else 1, 1 if release_facts else 0)
+                      0 if byte_model else 1, 1 if release_facts else 0, 1 if keep_facts else 0)
         s = BuildStats()
         _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
         if asynchronous:
             return None
         self.stats = s.as_dict()
         return self.stats
+
+    # ---- incremental builds / out-of-core sub-graphs (gdroid_stage_seeds & co.)
+    def stage_seeds(self, nodes, ptr, pairs, k: int = 0):
+        nodes = np.ascontiguousarray(nodes, dtype=np.uint32)
+        ptr = np.ascontiguousarray(ptr, dtype=np.uint64)
+        pairs = np.ascontiguousarray(pairs, dtype=np.uint64)
+        assert len(ptr) == len(nodes) + 1
+        _check(lib().gdroid_stage_seeds(self._h, k, len(nodes), _ptr(nodes), _ptr(ptr), _ptr(pairs)))
+
+    def read_reached(self, nodes, k: int = 0) -> np.ndarray:
+        nodes = np.ascontiguousarray(nodes, dtype=np.uint32)
+        out = np.zeros(max(len(nodes), 1), dtype=np.uint8)
+        _check(lib().gdroid_read_reached(self._h, k, len(nodes), _ptr(nodes), _ptr(out)))
+        return out[:len(nodes)].astype(bool)
+
+    def read_nodes_facts(self, nodes, k: int = 0) -> Tuple[np.ndarray, np.ndarray]:
+        nodes = np.ascontiguousarray(nodes, dtype=np.uint32)
+        L = lib()
+        ptr = np.zeros(len(nodes) + 1, dtype=np.uint64)
+        _check(L.gdroid_read_nodes_facts(self._h, k, len(nodes), _ptr(nodes), _ptr(ptr), None, 0))
+        tot = int(ptr[-1])
+        pairs = np.zeros(max(tot, 1), dtype=np.uint64)
+        _check(L.gdroid_read_nodes_facts(self._h, k, len(nodes), _ptr(nodes), _ptr(ptr), _ptr(pairs), tot))
+        return ptr, pairs[:tot]
+
+    @property
+    def fact_bytes(self) -> int:
+        return int(lib().gdroid_fact_bytes(self._h))
+
+    def export_facts(self, host: np.ndarray):
+        assert host.flags.c_contiguous and host.nbytes == self.fact_bytes
+        _check(lib().gdroid_export_facts(self._h, _ptr(host), host.nbytes))
+
+    def import_facts(self, host: np.ndarray):
+        assert host.flags.c_contiguous and host.nbytes == self.fact_bytes
+        _check(lib().gdroid_import_facts(self._h, _ptr(host), host.nbytes))
+
+    def stream_sync(self):
+        _check(lib().gdroid_stream_sync(self._h))
 
     def release_facts(self):
         """gdroid_release_facts: return the fact store to the device pool (digests stay)."""
@@ -201,6 +251,19 @@ class App:
         tot = int(ptr[-1])
         pairs = pairs_buf.get(tot) if pairs_buf is not None else np.zeros(max(tot, 1), dtype=np.uint64)[:tot]
         _check(L.gdroid_read_all_facts(self._h, k, _ptr(ptr), _ptr(pairs) if tot else None, tot))
+        return ptr, pairs[:tot]
+
+    def read_batch_facts(self, ptr_buf=None, pairs_buf=None) -> Tuple[np.ndarray, np.ndarray]:
+        """gdroid_read_batch_facts: (ptr[N_batch+1], pairs) over all apps of the handle; the
+        buffers (objects with .get(n) -> uint64 array, e.g. reusable pinned memory) are
+        optional."""
+        L = lib()
+        n = sum(self.n_nodes)
+        ptr = ptr_buf.get(n + 1) if ptr_buf is not None else np.zeros(n + 1, dtype=np.uint64)
+        _check(L.gdroid_read_batch_facts(self._h, _ptr(ptr), None, 0))
+        tot = int(ptr[-1])
+        pairs = pairs_buf.get(tot) if pairs_buf is not None else np.zeros(max(tot, 1), dtype=np.uint64)[:tot]
+        _check(L.gdroid_read_batch_facts(self._h, _ptr(ptr), _ptr(pairs) if tot else None, tot))
         return ptr, pairs[:tot]
 
     def node_digests(self, k: int = 0) -> Tuple[np.ndarray, int]:

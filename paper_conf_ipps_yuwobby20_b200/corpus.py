@@ -284,8 +284,9 @@ class BatchResult:
     h2d_bytes: int = 0
 
 
-class _PinnedBuf:
-    """Growable pinned host buffer (uint64) for fact readback."""
+class PinnedBuf:
+    """Growable pinned host buffer (uint64) for fact readback; reused across batches and steps
+    (pinning is slow, so an untimed warm-up pass sizes it)."""
 
     def __init__(self):
         self.t = None
@@ -293,22 +294,30 @@ class _PinnedBuf:
     def get(self, n: int) -> np.ndarray:
         import torch
         if self.t is None or self.t.numel() < n:
-            self.t = torch.empty(max(n, 1 << 20), dtype=torch.int64, pin_memory=True)
+            self.t = None
+            self.t = torch.empty(max(int(n * 1.1), 1 << 20), dtype=torch.int64, pin_memory=True)
         return self.t.numpy().view(np.uint64)[:n]
 
 
+class ReadbackBuffers:
+    def __init__(self):
+        self.ptr, self.pairs = PinnedBuf(), PinnedBuf()
+
+
 def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], device: int = 0,
-                  readback: str = "facts", on_facts: Optional[Callable] = None) -> List[BatchResult]:
+                  readback: str = "facts", on_facts: Optional[Callable] = None,
+                  bufs: Optional[ReadbackBuffers] = None) -> List[BatchResult]:
     """End to end through the public API: a loader thread generates batch i+1 and uploads it
-    (gdroid_load_batch on its own stream) while batch i builds on the GPU; then every app's
-    facts come back (gdroid_read_all_facts into pinned buffers: Alg. 3 l.17 h_fact <- d_fact,
-    PAPER.md:768), or only its digests (readback='digests').  A loader failure is re-raised
-    in the caller (never a hang)."""
+    (gdroid_load_batch on its own stream: the paper's dual buffering) while
+    batch i builds; batch i's facts come back (gdroid_read_batch_facts into pinned buffers:
+    Alg. 3 l.17 h_fact <- d_fact) while batch i+1 builds on the other stream.
+    readback='digests' reads only the app digests.  A loader failure is re-raised here."""
     import torch
     from . import _binding as gd
     q: "Queue" = Queue(maxsize=1)
     streams = [torch.cuda.Stream(device=device), torch.cuda.Stream(device=device)]
     stop = threading.Event()
+    bufs = bufs or ReadbackBuffers()
 
     def loader():
         try:
@@ -325,10 +334,27 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
         finally:
             q.put(None)
 
+    out: List[BatchResult] = []
+
+    def finish(prev):
+        ids, app, st, t0, load_ms, nn, ib = prev
+        dig = app.app_digests()
+        d2h = 8 * len(ids)
+        if readback == "facts":
+            ptr, pairs = app.read_batch_facts(bufs.ptr, bufs.pairs)
+            d2h += ptr.nbytes + pairs.nbytes
+            if on_facts is not None:
+                base = 0
+                for k, i in enumerate(ids):
+                    p = ptr[base:base + nn[k] + 1]
+                    on_facts(i, p - p[0], pairs[int(p[0]):int(p[-1])])
+                    base += nn[k]
+        app.free()
+        out.append(BatchResult(list(ids), dig, st, (time.perf_counter() - t0) * 1e3 + load_ms, d2h, ib))
+
     th = threading.Thread(target=loader, daemon=True)
     th.start()
-    out: List[BatchResult] = []
-    ptr_buf, pair_buf = _PinnedBuf(), _PinnedBuf()
+    prev = None
     try:
         while True:
             item = q.get()
@@ -338,28 +364,27 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
                 raise item
             ids, app, load_ms, nn, ib = item
             t0 = time.perf_counter()
-            st = app.build()
-            dig = app.app_digests()
-            d2h = 8 * len(ids)
-            if readback == "facts":
-                for k in range(len(ids)):
-                    ptr, pairs = app.read_all_facts(k, ptr_out=ptr_buf.get(nn[k] + 1),
-                                                    pairs_buf=pair_buf)
-                    d2h += ptr.nbytes + pairs.nbytes
-                    if on_facts is not None:
-                        on_facts(ids[k], ptr, pairs)
-            app.free()
-            out.append(BatchResult(list(ids), dig, st, (time.perf_counter() - t0) * 1e3 + load_ms,
-                                   d2h, ib))
+            app.build(asynchronous=True)
+            if prev is not None:                          # read back i while i+1 builds
+                finish(prev)
+                prev = None
+            st = app.sync()
+            prev = (ids, app, st, t0, load_ms, nn, ib)
+        if prev is not None:
+            finish(prev)
+            prev = None
     finally:
         stop.set()
-        while th.is_alive():                               # drain so the loader can finish
+        if prev is not None:
+            prev[1].free()
+        while th.is_alive() or not q.empty():             # drain so the loader can finish
             try:
                 it = q.get(timeout=0.1)
                 if isinstance(it, tuple):
                     it[1].free()
             except Exception:
-                pass
+                if not th.is_alive():
+                    break
         th.join()
     return out
 

@@ -73,13 +73,16 @@ __host__ __device__ __forceinline__ uint32_t occ_words(uint32_t rows) { return (
 // INTRA/C2R edges share one transfer evaluation, so their chunks hold up to 4 edges; CALL
 // and RET edges each re-map the whole block, so CALL and EXIT nodes get one edge per chunk.
 constexpr uint32_t EDGES_PER_CHUNK = 4;
-__host__ __device__ __forceinline__ uint32_t chunk_edges(uint32_t deg, uint32_t cls) {
+// Wide blocks (logW >= 1) are never split: their visit consumes Δ(src) once (semi-naive, DESIGN.md
+// §5.5), so one warp must propagate it along every out-edge.
+__host__ __device__ __forceinline__ uint32_t chunk_edges(uint32_t deg, uint32_t cls, uint32_t logW) {
+  if (logW >= 1) return deg > 0 ? deg : 1u;
   const uint32_t e = (deg + 31) >> 5;
   const uint32_t lo = (cls == 3u || cls == 4u) ? 1u : EDGES_PER_CHUNK;   // C_CALL, C_EXIT
   return e > lo ? e : lo;
 }
-__host__ __device__ __forceinline__ uint32_t n_chunks_of(uint32_t deg, uint32_t cls) {
-  return deg == 0 ? 1u : (deg + chunk_edges(deg, cls) - 1) / chunk_edges(deg, cls);
+__host__ __device__ __forceinline__ uint32_t n_chunks_of(uint32_t deg, uint32_t cls, uint32_t logW) {
+  return deg == 0 ? 1u : (deg + chunk_edges(deg, cls, logW) - 1) / chunk_edges(deg, cls, logW);
 }
 
 // Chunk 0's INTRA/C2R out-edges of a narrow node, held beside its NodeRec (4 x 16 B = one
@@ -139,7 +142,7 @@ constexpr uint32_t NO_XMAP = 0xffffffffu;
 constexpr uint32_t F_GRP = 1u, F_MER = 2u, F_CONT = 4u;
 
 struct DevStats {
-  unsigned long long rounds, visits, alg_bytes, dense_bytes, atomics, hist[3], limit_hit, pad;
+  unsigned long long rounds, visits, alg_bytes, dense_bytes, atomics, hist[3], limit_hit, seed_err;
   unsigned long long phase[8];  // GD_PHASES builds: cycles in setup / edges / push / round end, items
 };
 
@@ -166,6 +169,8 @@ struct Dev {
   const uint32_t* node_method;  // [N] (digest / readback only)
   const int32_t* frow;          // field-row tables: frow[r3 + c] = global row of (col c, f) | -1
   uint64_t* facts;
+  uint64_t* delta;              // wide batches: Δ store, same layout as facts (bits that reached
+                                // IN(n) since n's last visit); nullptr if narrow
   uint64_t* smask;              // [N] narrow blocks: bit i = word group i (mshift_of(B)) may be non-zero
   uint32_t* stamp;              // [N] last round a node was queued for (0 = never)
   uint32_t* cont;               // [N] last round a warp continued into the node (0 = never)
@@ -185,7 +190,11 @@ struct Dev {
   uint32_t wide;                // max log2(words per row) over the batch's modules: 0 = all narrow,
                                 // >= 1: some module has > 64 instances (row-occupancy path)
   uint32_t hiocc;               // 1: launch the 4-CTA/SM narrow instantiation (batches >= HIOCC_NODES)
-  uint32_t round0;              // first round of this launch (non-hybrid: 1)
+  const uint32_t* seed_nodes;   // staged seed nodes queued by k_seed (incremental builds)
+  const uint32_t* seed_pairs;   // [3 n] (node, slot gid, instance gid) OR-ed in by k_apply_seeds
+  uint32_t n_seed_nodes, n_seed_pairs;
+  uint32_t push_entries;        // 1: k_seed queues the component entries (fresh builds)
+  uint32_t round0;              // first round of this build / launch (1 for a fresh build)
   uint32_t hyb;                 // 1: hybrid launch sequence: start at round bar[3], return if it is 0
   uint32_t sw_lo, sw_hi;        // hybrid: leave at the start of a round with < sw_lo / >= sw_hi items
                                 // (bar[3] = that round), 0 = off
@@ -239,9 +248,10 @@ cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_digest(const Dev& D, cudaStream_t s);
-cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
+cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s,
+                        const uint32_t* list = nullptr);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,
-                          uint64_t* pairs, cudaStream_t s);
+                          uint64_t* pairs, cudaStream_t s, const uint32_t* list = nullptr);
 int fixpoint_max_blocks(int device, uint32_t wide, uint32_t hiocc);
 
 }  // namespace gd

@@ -65,12 +65,14 @@ struct Acc {                   // per-warp counters (shared memory), flushed onc
   unsigned long long cont;     // items processed by continuation (visits not in the queue)
 };
 
-struct WarpScratch {
+template <bool WIDE>
+struct WarpScratchT {
   uint64_t rv[MAXW];           // FSTORE base row v
   uint64_t rw[MAXW];           // FSTORE / FLOAD value row w
   uint64_t gen[MAXW];          // generated row (wide path)
   int16_t cmap[64 * MAXW];     // projection column map of the current cross-module edge
-  uint16_t rowlist[1024];      // rows visited by the wide path
+  uint16_t rowlist[WIDE ? 1024 : 1];        // wide: candidate rows, then the rows with OUT_Δ != 0
+  uint32_t gbits[WIDE ? 32 : 1];            // wide: update() per edge of the item (<= 1024 edges)
 };
 
 // warp-uniform counter updates: lane 0 adds the warp's total
@@ -89,6 +91,11 @@ struct CtaStage {              // per-CTA staged worklist appends of the current
 // fire-and-forget 64-bit OR at L2 (RED; no return value, no scoreboard wait)
 __device__ __forceinline__ void red_or(uint64_t* p, uint64_t v) {
   asm volatile("red.relaxed.gpu.global.or.b64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
+}
+
+// fire-and-forget 64-bit AND at L2 (clears the Δ bits a visit consumed)
+__device__ __forceinline__ void red_and(uint64_t* p, uint64_t v) {
+  asm volatile("red.relaxed.gpu.global.and.b64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
 
 __device__ __forceinline__ uint64_t warp_or64(uint64_t v) {
@@ -264,10 +271,12 @@ __device__ __forceinline__ void set_mask(const Dev& D, uint32_t dst, uint64_t mb
 // occupancy bit.  Same results as the dense path, bytes proportional to non-zero rows.
 constexpr int WROWS = 1024;    // row-list capacity per warp (rows of one block)
 
+// OR one row into IN(dst) (wide or narrow target).  Wide targets (logWt >= 1) also get the
+// new bits in Δ(dst) (Zd: the target's block in the Δ store), which their next visit consumes.
 template <int MW>
 __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_t logWt, uint32_t rt,
                                                const uint64_t (&v)[MW], uint32_t& nz, uint32_t& red, bool& g,
-                                               uint64_t* mask_t) {
+                                               uint64_t* mask_t, uint64_t* Zd) {
   const uint32_t Wt = 1u << logWt;
   uint64_t* row = Z + ((uint64_t)rt << logWt);
   uint64_t cur[MW];
@@ -284,24 +293,40 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
     if (j >= (int)Wt || !v[j]) continue;
     ++nz;
     if (cur[j]) was_zero = false;
-    if (v[j] & ~cur[j]) { red_or(row + j, v[j]); ++red; g = true; wrote = true; }
+    const uint64_t nb = v[j] & ~cur[j];
+    if (nb) {
+      red_or(row + j, v[j]);
+      if (logWt >= 1) red_or(Zd + ((uint64_t)rt << logWt) + j, nb);   // Δ(dst) of a wide target
+      ++red; g = true; wrote = true;
+    }
   }
   if (logWt >= 1 && was_zero) red_or(Z + occ_offset(Bt) + (rt >> 6), 1ull << (rt & 63));   // occupancy
   if (GD_SMASK && logWt == 0 && was_zero && wrote) red_or(mask_t, 1ull << (rt >> mshift_of(Bt)));
 }
 
+// Semi-naive (Δ) visit of a wide block.  IN(src) supplies the transfer
+// function's operand rows and the candidate rows (its row-occupancy bitmap); the visit
+// propagates only OUT_Δ = (Δ(src) \ KILL) ∪ GEN(IN(src)) where Δ(src) holds the bits that
+// reached IN(src) since its last visit.  Every f of §3 C2 is (X \ KILL) ∪ GEN(X) with GEN
+// monotone and every edge transform distributes over ∪, so f(IN_old ∪ Δ) ⊆ f(IN_old) ∪ OUT_Δ:
+// successors already hold T_e(f(IN_old)) from earlier visits and receive T_e(OUT_Δ) now —
+// the same least fixed point (C4) with work proportional to the new facts.  Δ bits are
+// consumed with RED.AND of exactly the bits read; bits arriving later stay for the next visit
+// (their writer also queued the node).
 template <bool CNT, int MW>
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
-                             bool first, uint32_t round, uint32_t nxt, int lane, WarpScratch& ws, Acc& acc,
+                             bool first, uint32_t round, uint32_t nxt, int lane, WarpScratchT<true>& ws, Acc& acc,
                              uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
   const uint32_t logW = R.logW, W = 1u << logW, L = R.L, B = R.B, rows = B >> logW;
   // The fact store is read and RED.OR-ed by the same kernel (self loops write IN(src) within
   // one item): no __restrict__ / const-cache loads on it, only plain coherent LDG.
   const uint64_t* X = D.facts + R.off;
+  uint64_t* DX = D.delta + R.off;
   const uint64_t* OCC = X + occ_offset(B);
   const uint32_t nocc = occ_words(rows);
   const uint32_t kind = R.kind;
-  // ---- transfer setup: generated row t (mode 1 replace / 2 or-in) or FSTORE rows (mode 3)
+  // ---- transfer setup on IN(src): generated row t (mode 1 replace / 2 or-in) or FSTORE rows
+  //      (mode 3).  The full GEN is emitted on every visit (a superset of its new part).
   int mode = 0, t = -1;
   uint32_t hwords = 0;
   if (lane < MAXW) ws.gen[lane] = 0;
@@ -341,8 +366,9 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
       ws.rw[lane] = X[((uint64_t)R.r1 << logW) + lane];
     }
   }
+  if (lane < 32) ws.gbits[lane] = 0;
   __syncwarp();
-  // ---- row list: flagged rows, then the generated rows that are not flagged yet
+  // ---- candidate rows: IN-occupied rows (Δ ⊆ IN), then generated rows not occupied yet
   const unsigned lt_mask = (1u << lane) - 1u;
   const uint64_t my_occ = lane < (int)nocc ? OCC[lane] : 0ull;   // nocc <= 32 (loader: rows <= WROWS)
   uint32_t cnt = 0;
@@ -373,14 +399,62 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
 
   uint32_t nzx = 0, nz = 0, red = 0;
   unsigned long long dense_l0 = first ? 8ull * B : 0ull;
-  for (uint32_t eb = e0; eb < e1; eb += 32) {
-    const uint32_t ne = min(32u, e1 - eb);
-    const uint32_t my_info = lane < (int)ne ? D.edges[eb + lane].info : 0u;
-    unsigned gmask = 0;
-    for (uint32_t i = 0; i < ne; ++i) {
-      const Edge* ep = D.edges + eb + i;
+  // OUT_Δ row of candidate row r: Δ(src) row r (killed for mode-1 row t), plus the GEN rows
+  auto out_delta = [&](uint32_t r, uint64_t (&y)[MW], bool consume) {
+    uint64_t* drow = DX + ((uint64_t)r << logW);
+#pragma unroll
+    for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? drow[j] : 0ull;
+    if (consume) {
+#pragma unroll
+      for (int j = 0; j < MW; ++j)
+        if (y[j]) { red_and(drow + j, ~y[j]); ++nzx; }      // consume exactly the bits read
+    }
+    if (mode == 1 && (int)r == t) {                          // Δ row t killed, GEN instead
+#pragma unroll
+      for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? ws.gen[j] : 0ull;
+    } else if (mode == 2 && (int)r == t) {
+#pragma unroll
+      for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.gen[j];
+    } else if (mode == 3 && r >= L + R.n_stat) {
+      const uint32_t gg = r - L;
+      if (D.grow_field[R.grow_off + gg] == R.r2) {
+        const int c = D.grow_col[R.grow_off + gg];
+        if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) {
+#pragma unroll
+          for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.rw[j];
+        }
+      }
+    }
+    bool any = false;
+#pragma unroll
+    for (int j = 0; j < MW; ++j) any |= (y[j] != 0);
+    return any;
+  };
+  // ---- pass 1: keep the candidate rows whose OUT_Δ is non-empty (compacted in place; a row
+  //      that gains Δ bits after this scan keeps them for the node's next visit)
+  uint32_t kept = 0;
+  for (uint32_t p0 = 0; p0 < cnt; p0 += 32) {
+    const uint32_t p = p0 + lane;
+    uint64_t y[MW];
+    const uint32_t r = p < cnt ? ws.rowlist[p] : 0u;
+    const bool keep = p < cnt && out_delta(r, y, false);
+    const unsigned km = __ballot_sync(FULL, keep);
+    if (keep) ws.rowlist[kept + __popc(km & lt_mask)] = (uint16_t)r;   // (behind every read)
+    kept += __popc(km);
+  }
+  __syncwarp();
+  // ---- pass 2: 32 kept rows at a time (one per lane): consume their Δ bits and propagate
+  //      OUT_Δ along every edge of the item
+  for (uint32_t q0 = 0; q0 < kept; q0 += 32) {
+    const bool mine = q0 + lane < kept;
+    const uint32_t rr = mine ? ws.rowlist[q0 + lane] : 0u;
+    uint64_t yv[MW];
+    const bool live = mine && out_delta(rr, yv, true);
+    for (uint32_t e = e0; e < e1; ++e) {
+      const Edge* ep = D.edges + e;
       const uint32_t ek = ep->info & 3u;
       uint64_t* Z = D.facts + ep->off;
+      uint64_t* Zd = D.delta + ep->off;
       const uint32_t Bt = ep->B, Lt = ep->L, logWt = ep->logW;
       const int aux = ep->aux;
       const uint32_t xoff = ep->xoff;
@@ -393,89 +467,72 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
       const uint32_t npar = (ek == GE_CALL) ? (uint32_t)aux : 0u;
       const int lhs = (ek == GE_RET) ? aux : -1;
       bool g = false;
-      for (uint32_t p = lane; p < cnt; p += 32) {
-        const uint32_t r = ws.rowlist[p];
-        // Y row r = f(X) row r
-        uint64_t y[MW];
-#pragma unroll
-        for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? X[((uint64_t)r << logW) + j] : 0ull;
-        if (first && eb == e0 && i == 0) {
-#pragma unroll
-          for (int j = 0; j < MW; ++j) nzx += (j < (int)W && y[j] != 0);
-        }
-        if (mode == 1 && (int)r == t) {
-#pragma unroll
-          for (int j = 0; j < MW; ++j) y[j] = (j < (int)W) ? ws.gen[j] : 0ull;
-        } else if (mode == 2 && (int)r == t) {
-#pragma unroll
-          for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.gen[j];
-        } else if (mode == 3 && r >= L + R.n_stat) {
-          const uint32_t gg = r - L;
-          if (D.grow_field[R.grow_off + gg] == R.r2) {
-            const int c = D.grow_col[R.grow_off + gg];
-            if ((ws.rv[c >> 6] >> (c & 63)) & 1ull) {
-#pragma unroll
-              for (int j = 0; j < MW; ++j) if (j < (int)W) y[j] |= ws.rw[j];
-            }
-          }
-        }
-        // Target rows.  Every edge kind maps source row r to at most one target row, except
+      if (live) {
+        // Target rows.  Every edge kind maps source row rr to at most one target row, except
         // CALL locals: one local passed as several actuals feeds every such parameter
         // (param_j <- arg_j for all j), so CALL scans all npar actuals.
         int rt = -1;
-        const bool call_local = ek == GE_CALL && r < L;
-        if (ek == GE_INTRA) rt = (int)r;
-        else if (ek == GE_C2R) rt = ((int)r == R.r0) ? -1 : (int)r;
-        else if (r >= L) {
-          const uint32_t gs = r - L;
+        const bool call_local = ek == GE_CALL && rr < L;
+        if (ek == GE_INTRA) rt = (int)rr;
+        else if (ek == GE_C2R) rt = ((int)rr == R.r0) ? -1 : (int)rr;
+        else if (rr >= L) {
+          const uint32_t gs = rr - L;
           const int gt = proj ? rowinv[gs] : (int)gs;       // π: source global row -> target row
           if (gt >= 0) rt = (int)Lt + gt;
         } else if (ek == GE_RET) {
-          if (r == L - 1 && lhs >= 0) rt = lhs;
+          if (rr == L - 1 && lhs >= 0) rt = lhs;
         }
-        if (rt < 0 && !call_local) continue;
-        uint64_t out[MW];                                   // the row in the target's columns
-        if (!proj) {
+        if (rt >= 0 || call_local) {
+          uint64_t out[MW];                                 // the row in the target's columns
+          if (!proj) {
 #pragma unroll
-          for (int s2 = 0; s2 < MW; ++s2) out[s2] = y[s2];
-        } else {
+            for (int s2 = 0; s2 < MW; ++s2) out[s2] = yv[s2];
+          } else {
 #pragma unroll
-          for (int s2 = 0; s2 < MW; ++s2) out[s2] = 0;
-          for (uint32_t j = 0; j < W; ++j) {
-            uint64_t b = 0;
+            for (int s2 = 0; s2 < MW; ++s2) out[s2] = 0;
+            for (uint32_t j = 0; j < W; ++j) {
+              uint64_t b = 0;
 #pragma unroll
-            for (int jj = 0; jj < MW; ++jj) if ((uint32_t)jj == j) b = y[jj];
-            while (b) {
-              const int bit = __ffsll((long long)b) - 1;
-              b &= b - 1;
-              const int cd = ws.cmap[j * 64 + bit];
-              if (cd < 0) continue;
+              for (int jj = 0; jj < MW; ++jj) if ((uint32_t)jj == j) b = yv[jj];
+              while (b) {
+                const int bit = __ffsll((long long)b) - 1;
+                b &= b - 1;
+                const int cd = ws.cmap[j * 64 + bit];
+                if (cd < 0) continue;
 #pragma unroll
-              for (int s2 = 0; s2 < MW; ++s2)
-                if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
+                for (int s2 = 0; s2 < MW; ++s2)
+                  if (s2 == (cd >> 6)) out[s2] |= 1ull << (cd & 63);
+              }
             }
           }
-        }
-        if (!call_local) {
-          emit_row_words(Z, Bt, logWt, (uint32_t)rt, out, nz, red, g, D.smask + ep->dst);
-        } else {
-          const uint32_t a0 = npar > 3 ? D.arg_ptr[n] : 0u;
-          for (uint32_t jj = 0; jj < npar; ++jj) {        // param_jj <- arg_jj whenever arg_jj = r
-            const int a = npar > 3 ? D.args[a0 + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
-            if (a == (int)r) emit_row_words(Z, Bt, logWt, jj, out, nz, red, g, D.smask + ep->dst);
+          if (!call_local) {
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt, out, nz, red, g, D.smask + ep->dst, Zd);
+          } else {
+            const uint32_t a0 = npar > 3 ? D.arg_ptr[n] : 0u;
+            for (uint32_t jj = 0; jj < npar; ++jj) {        // param_jj <- arg_jj whenever arg_jj = rr
+              const int a = npar > 3 ? D.args[a0 + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
+              if (a == (int)rr) emit_row_words(Z, Bt, logWt, jj, out, nz, red, g, D.smask + ep->dst, Zd);
+            }
           }
         }
       }
       if (proj) __syncwarp();
-      g = __any_sync(FULL, g);
-      if (g) gmask |= 1u << i;
-      dense_l0 += 16ull * Bt;
+      if (__any_sync(FULL, g) && lane == 0 && e - e0 < 1024u) ws.gbits[(e - e0) >> 5] |= 1u << ((e - e0) & 31u);
+      if (q0 == 0) dense_l0 += 16ull * Bt;
     }
+  }
+  __syncwarp();
+  for (uint32_t eb = e0; eb < e1; eb += 32) {               // update() / first reach -> pushes
+    const uint32_t ne = min(32u, e1 - eb);
+    const uint32_t gm = eb - e0 < 1024u ? ws.gbits[(eb - e0) >> 5] : ~0u;   // beyond: push (safe)
+    const uint32_t my_info = lane < (int)ne ? D.edges[eb + lane].info : 0u;
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gmask >> lane) & 1u, round, nxt, cont, cont_dense);
+    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gm >> lane) & 1u, round, nxt, cont, cont_dense);
   }
   if constexpr (CNT) {                     // byte models (dead code, removed, when !CNT)
-    acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
+    // touched words of the semi-naive visit: Δ(src) words read and cleared, T_e(OUT_Δ) words
+    // read and OR-ed into IN(dst) (+ Δ(dst)), heap rows gathered, occupancy words
+    acc_add(acc.alg, 24u * nz + 16u * nzx + 8u * hwords + 8u * nocc + (lane == 0 ? alg_l0 : 0u));
     acc_add(acc.atom, red);
     if (lane == 0) acc.dense += dense_l0 + alg_l0;
   }
@@ -627,13 +684,13 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
 // ---------------------------------------------------------------------------------- one item
 template <bool WIDE, bool CNT, int MW, bool CD>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
-                                 uint32_t nxt, int lane, WarpScratch& ws, Acc& acc, bool allow_cont,
+                                 uint32_t nxt, int lane, WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
   const uint64_t mk = GD_SMASK ? __ldcg(D.smask + n) : ~0ull;   // (issued with the NodeRec load)
   const NodeRec R = D.nodes[n];
   InlEdge me{0u, 0u, 0ull};                                 // inline chunk-0 edge of this lane (same hop)
   if (GD_INL && !WIDE && lane < 4) me = D.inl[4 * n + lane];
-  const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls);
+  const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls, R.logW);
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
   const bool first = ci == 0;
   const uint32_t L = R.L, B = R.B;
@@ -881,7 +938,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                     if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
                 }
               }
-              emit_row_words(Z, Bt, logWt, r, out, nz, red, g, D.smask + ep->dst);   // occupancy
+              emit_row_words(Z, Bt, logWt, r, out, nz, red, g, D.smask + ep->dst, D.delta + off);   // occupancy, Δ
             }
           }
         }
@@ -938,7 +995,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
 template <bool WIDE, bool CNT, int MW, bool CD>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
-                                              uint32_t nw, int lane, WarpScratch& ws, Acc& acc) {
+                                              uint32_t nw, int lane, WarpScratchT<WIDE>& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
   uint32_t cnt[NCLS];
   uint32_t total = 0;
@@ -1001,7 +1058,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       uint32_t info = 0;
       if (lane == 0) {
         const NodeRec R = D.nodes[n];
-        info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls) - 1) << 5);
+        info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls, R.logW) - 1) << 5);
       }
       flush_pushes(D, st, lane, lane == 0, n, info, true, round, nxt);
       item += nw;
@@ -1023,7 +1080,8 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
                                               depth < GD_CONT_DEPTH, cont_ok);
         if (c == NO_CONT) break;
         __syncwarp();                      // this warp's ORs into IN(c) are visible to all lanes
-        __threadfence_block();
+        if constexpr (WIDE) __threadfence();   // + its Δ(c) bits (the visit consumes them): L2 order
+        else __threadfence_block();
         n = c;
         ci = 0;
         if (lane == 0) acc.cont += 1;
@@ -1037,7 +1095,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
 
 template <bool WIDE, bool CNT, int MW, int MINB>
 __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
-  __shared__ WarpScratch ws_all[WARPS];
+  __shared__ WarpScratchT<WIDE> ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
   __shared__ CtaStage st;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1074,7 +1132,7 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
 
 template <bool WIDE, bool CNT, int MW>
 __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t round) {
-  __shared__ WarpScratch ws_all[WARPS];
+  __shared__ WarpScratchT<WIDE> ws_all[WARPS];
   __shared__ Acc acc_all[WARPS];
   __shared__ CtaStage st;
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1120,14 +1178,14 @@ __global__ void k_edges(Dev D, Edge* edges, InlEdge* inl, NodeRec* nodes, const 
   for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < D.n_nodes; n += stride) {
     const NodeRec R = nodes[n];
     const uint32_t base = D.app_node_base[R.app];
-    const uint32_t deg = R.e1 - R.e0, n0 = min(deg, chunk_edges(deg, R.cls));
+    const uint32_t deg = R.e1 - R.e0, n0 = min(deg, chunk_edges(deg, R.cls, R.logW));
     bool inl_ok = deg > 0 && n0 <= 4 && R.logW == 0 && R.B <= INL_MAX_B;
     InlEdge rec[4];
     for (uint32_t e = R.e0; e < R.e1; ++e) {
       const uint32_t s = base + ecol[e], ek = ekind[e];
       const NodeRec& RS = nodes[s];
       const uint32_t cls = RS.cls, logW = RS.logW;
-      const uint32_t nch = n_chunks_of(RS.e1 - RS.e0, cls);
+      const uint32_t nch = n_chunks_of(RS.e1 - RS.e0, cls, logW);
       Edge E2;
       E2.dst = s;
       E2.info = ek | (cls << 2) | ((nch - 1) << 5) | (logW >= 1 ? INFO_WIDE : 0u);
@@ -1146,23 +1204,66 @@ __global__ void k_edges(Dev D, Edge* edges, InlEdge* inl, NodeRec* nodes, const 
 
 // (a2) seed round 1 with the component entries (Alg. 1 l.9)
 __global__ void k_seed(Dev D) {
+  // The first round of this build is D.round0 (1, or after the rounds of earlier builds of an
+  // incremental handle): entries (fresh builds) and staged seed nodes (gdroid_stage_seeds) are
+  // queued for it, stamped round0, in queue slot round0 % 3.
   __shared__ CtaStage st;
   const int lane = threadIdx.x & 31;
+  const uint32_t r0 = D.round0;
   stage_init(st);
   __syncthreads();
-  for (uint32_t i0 = 0; i0 < D.n_entries; i0 += 32) {
+  const uint32_t ne = D.push_entries ? D.n_entries : 0u, nt = ne + D.n_seed_nodes;
+  for (uint32_t i0 = 0; i0 < nt; i0 += 32) {
     const uint32_t i = i0 + lane;
-    const bool act = i < D.n_entries;
-    const uint32_t e = act ? D.entries[i] : 0u;
+    const bool act = i < nt;
+    const uint32_t e = act ? (i < ne ? D.entries[i] : D.seed_nodes[i - ne]) : 0u;
     uint32_t info = 0;
     if (act) {
       const NodeRec R = D.nodes[e];
-      info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls) - 1) << 5);
+      info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls, R.logW) - 1) << 5);
     }
-    flush_pushes(D, st, lane, act, e, info, true, 0u, 1u);
+    flush_pushes(D, st, lane, act, e, info, true, r0 - 1, r0 % 3);
   }
-  stage_publish(D, st, 1u);
-  if (threadIdx.x == 0) D.bar[3] = 1;     // hybrid sequences start at round 1
+  stage_publish(D, st, r0 % 3);
+  if (threadIdx.x == 0) D.bar[3] = r0;    // hybrid sequences start here
+}
+
+// Staged seed facts (gdroid_stage_seeds): OR pair (slot gid, instance gid) into IN(node) —
+// and into Δ(node) and the row-occupancy bitmap for wide blocks — before the build's first
+// round.  One thread per pair: slot -> row (method local, else binary search of the module's
+// ascending global-row gids), instance -> column (binary search of the sorted pool).  A pair
+// outside the node's pools P_m x Q_m sets stats->seed_err (GDROID_E_POOL).
+__global__ void k_apply_seeds(Dev D) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= D.n_seed_pairs) return;
+  const uint32_t node = D.seed_pairs[3 * i], slot = D.seed_pairs[3 * i + 1], inst = D.seed_pairs[3 * i + 2];
+  const NodeRec R = D.nodes[node];
+  const uint32_t L = R.L, rows = R.B >> R.logW;
+  int64_t row = -1;
+  if (slot - R.local_base < L) row = slot - R.local_base;
+  else {
+    uint32_t lo = 0, hi = rows - L;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (D.grow_gid[R.grow_off + mid] < slot) lo = mid + 1; else hi = mid;
+    }
+    if (lo < rows - L && D.grow_gid[R.grow_off + lo] == slot) row = L + lo;
+  }
+  uint32_t lo = 0, hi = R.n_cols;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (D.col_gid[R.col_off + mid] < inst) lo = mid + 1; else hi = mid;
+  }
+  if (row < 0 || lo >= R.n_cols || D.col_gid[R.col_off + lo] != inst) {
+    atomicExch(&D.stats->seed_err, 1ull + i);
+    return;
+  }
+  const uint64_t w = ((uint64_t)row << R.logW) + (lo >> 6), bit = 1ull << (lo & 63);
+  atomicOr((unsigned long long*)(D.facts + R.off + w), bit);
+  if (R.logW >= 1) {
+    atomicOr((unsigned long long*)(D.delta + R.off + w), bit);
+    atomicOr((unsigned long long*)(D.facts + R.off + occ_offset(R.B) + (row >> 6)), 1ull << (row & 63));
+  }
 }
 
 // (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp's nodes are
@@ -1206,28 +1307,32 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
   if (lane == 0 && app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
 }
 
-__global__ void k_popc(Dev D, uint32_t n0, uint32_t n1, uint64_t* out) {
+// Readback kernels over nodes n0 .. n1-1, or over list[0 .. n1-n0) when list != nullptr.
+__global__ void k_popc(Dev D, uint32_t n0, uint32_t n1, uint64_t* out, const uint32_t* list) {
   const int lane = threadIdx.x & 31;
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t n = n0 + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < n1; n += nw) {
+  for (uint32_t i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n1 - n0; i += nw) {
+    const uint32_t n = list ? list[i] : n0 + i;
     const NodeRec R = D.nodes[n];
     unsigned long long c = 0;
     for (uint32_t w = lane; w < R.B; w += 32) c += __popcll(D.facts[R.off + w]);
     c = warp_sum64(c);
-    if (lane == 0) out[n - n0] = c;
+    if (lane == 0) out[i] = c;
   }
 }
 
 // bits of IN(n) -> ascending (slot gid << 32 | inst gid): row-major order is ascending because
 // rows are locals < statics < heap in gid order and columns are sorted instance gids.
-__global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs) {
+__global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
+                         const uint32_t* list) {
   const int lane = threadIdx.x & 31;
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
-  for (uint32_t n = n0 + blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < n1; n += nw) {
+  for (uint32_t i = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n1 - n0; i += nw) {
+    const uint32_t n = list ? list[i] : n0 + i;
     const NodeRec R = D.nodes[n];
     const uint32_t local_base = R.local_base;
     const uint32_t logW = R.logW, L = R.L, B = R.B;
-    uint64_t base = ptr[n - n0];
+    uint64_t base = ptr[i];
     for (uint32_t w0 = 0; w0 < B; w0 += 32) {
       const uint32_t w = w0 + lane;
       uint64_t x = w < B ? D.facts[R.off + w] : 0;
@@ -1272,6 +1377,7 @@ cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes
 }
 
 cudaError_t launch_seed(const Dev& D, cudaStream_t s) {
+  if (D.n_seed_pairs) k_apply_seeds<<<(D.n_seed_pairs + 255) / 256, 256, 0, s>>>(D);
   k_seed<<<1, 32, 0, s>>>(D);
   return cudaGetLastError();
 }
@@ -1335,14 +1441,14 @@ cudaError_t launch_digest(const Dev& D, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s) {
-  k_popc<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, out);
+cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s, const uint32_t* list) {
+  k_popc<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, out, list);
   return cudaGetLastError();
 }
 
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
-                          cudaStream_t s) {
-  k_expand<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, ptr, pairs);
+                          cudaStream_t s, const uint32_t* list) {
+  k_expand<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, ptr, pairs, list);
   return cudaGetLastError();
 }
 

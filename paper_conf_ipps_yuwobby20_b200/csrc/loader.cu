@@ -620,6 +620,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     if (words >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "app %u: node %llu: fact block too large", k, (unsigned long long)n);
     if (L > 0xffff) return set_err(GDROID_E_LIMIT, "app %u: node %llu: method with > 65535 locals", k, (unsigned long long)n);
     if (md.logW >= 1 && L + md.n_glob > 1024) return set_err(GDROID_E_LIMIT, "app %u: node %llu: wide block with > 1024 rows", k, (unsigned long long)n);
+    if (d->row_ptr[n + 1] - d->row_ptr[n] > 32768) return set_err(GDROID_E_LIMIT, "app %u: node %llu: out-degree > 32768", k, (unsigned long long)n);
     R.off = H.fact_words + foff[n];
     R.B = (uint32_t)words; R.L = L; R.n_stat = md.n_stat;
     R.e0 = (uint32_t)d->row_ptr[n]; R.e1 = (uint32_t)d->row_ptr[n + 1];
@@ -629,7 +630,7 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
     H.o_nodemeth[n] = mb + (uint32_t)m;
     H.o_rowptr[n + 1] = (uint32_t)d->row_ptr[n + 1];
     H.o_argptr[n + 1] = (uint32_t)a1;
-    cls_cnt[R.cls] += n_chunks_of(R.e1 - R.e0, R.cls);     // work items per GRP class
+    cls_cnt[R.cls] += n_chunks_of(R.e1 - R.e0, R.cls, R.logW);     // work items per GRP class
     return GDROID_OK;
   };
   PHASE("field-row tables");
@@ -1085,6 +1086,17 @@ struct gdroid_app {
   uint64_t launches = 0;
   bool built = false, pending = false;
   bool digests_ok = false;            // a build completed (digests readable even if facts released)
+  uint64_t build_serial = 0;          // completed builds (readback count cache key)
+  // incremental builds / out-of-core sub-graphs
+  bool state_valid = false;           // stamps hold a completed build's history
+  bool facts_valid = false;           // the fact store holds facts (build or import), not garbage
+  uint32_t round_base = 0;            // rounds used by earlier builds of this handle
+  std::vector<uint32_t> seed_nodes;   // staged for the next keep_facts build
+  std::vector<uint32_t> seed_pairs;   // (node, slot gid, inst gid) triples
+  void* h_seed = nullptr;             // pinned staging of the seeds
+  void* d_seed = nullptr;
+  size_t seed_cap = 0;
+  uint64_t counts_build = ~0ull;      // build_serial whose per-node counts are in d_scratch
   bool release_pending = false;
   int max_blocks = 0;
   int max_blocks_lo = 0;              // hybrid (large narrow batches): grid of the 3-CTA/SM instantiation
@@ -1105,10 +1117,12 @@ void free_app(gdroid_app* a) {
   if (a->d_tables) cudaFreeAsync(a->d_tables, a->stream);
   if (a->d_facts) cudaFreeAsync(a->d_facts, a->stream);
   if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
-  if (a->d_scratch) cudaFree(a->d_scratch);
+  if (a->d_scratch) cudaFreeAsync(a->d_scratch, a->stream);
   if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
-  if (a->pending) cudaStreamSynchronize(a->stream);   // the stats copy targets the slot
+  if (a->pending || a->h_seed) cudaStreamSynchronize(a->stream);   // copies target host slots
+  if (a->d_seed) cudaFreeAsync(a->d_seed, a->stream);
+  if (a->h_seed) cudaFreeHost(a->h_seed);
   stats_slots().put(a->h_stats);
   for (auto& e : a->ev)
     if (e) cudaEventDestroy(e);
@@ -1122,13 +1136,36 @@ struct DeviceGuard {
   ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
 };
 
+// Readback scratch: stream-ordered (cudaFreeAsync / cudaMallocAsync on the handle's stream), so
+// growing it never synchronises the device.
 gdroid_status ensure_scratch(gdroid_app* a, size_t bytes) {
   if (a->scratch_bytes >= bytes) return GDROID_OK;
-  if (a->d_scratch) cudaFree(a->d_scratch);
+  if (a->d_scratch) CU(cudaFreeAsync(a->d_scratch, a->stream));
   a->d_scratch = nullptr;
   a->scratch_bytes = 0;
-  CU(cudaMalloc(&a->d_scratch, bytes));
+  CU(cudaMallocAsync(&a->d_scratch, bytes, a->stream));
   a->scratch_bytes = bytes;
+  return GDROID_OK;
+}
+
+gdroid_status ensure_facts(gdroid_app* a) {
+  if (a->d_facts) return GDROID_OK;
+  const cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, a->stream);
+  if (e != cudaSuccess) return set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e));
+  a->D.facts = a->d_facts;
+  a->D.delta = a->D.wide ? a->d_facts + std::max<uint64_t>(a->D.n_words, 4) : nullptr;
+  a->facts_valid = false;
+  return GDROID_OK;
+}
+
+gdroid_status ensure_seed_buf(gdroid_app* a, size_t bytes) {
+  if (a->seed_cap >= bytes) return GDROID_OK;
+  if (a->h_seed) { CU(cudaStreamSynchronize(a->stream)); cudaFreeHost(a->h_seed); a->h_seed = nullptr; }
+  if (a->d_seed) { CU(cudaFreeAsync(a->d_seed, a->stream)); a->d_seed = nullptr; }
+  a->seed_cap = 0;
+  CU(cudaMallocHost(&a->h_seed, bytes));
+  CU(cudaMallocAsync(&a->d_seed, bytes, a->stream));
+  a->seed_cap = bytes;
   return GDROID_OK;
 }
 
@@ -1150,8 +1187,11 @@ gdroid_status finish_stats(gdroid_app* a, gdroid_build_stats* out) {
   a->pending = false;
   a->built = a->d_facts != nullptr;                   // released facts cannot be read back
   a->digests_ok = true;
+  ++a->build_serial;
   if (out) *out = s;
-  if (h.limit_hit) return set_err(GDROID_E_LIMIT, "max_rounds (%u) exceeded; facts are an under-approximation", a->D.max_rounds);
+  a->round_base += (uint32_t)h.rounds + 2;            // incremental builds continue the numbering
+  if (h.seed_err) return set_err(GDROID_E_POOL, "staged seed pair %llu is outside its node's pools (V1-V4)", (unsigned long long)(h.seed_err - 1));
+  if (h.limit_hit) return set_err(GDROID_E_LIMIT, "max_rounds exceeded; facts are an under-approximation");
   return GDROID_OK;
 }
 
@@ -1408,10 +1448,12 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   // ---- fact store + mutable state
   {
     keep_pool_reserved(device);
-    a->fact_alloc_bytes = std::max<uint64_t>(Lo.fact_words, 4) * 8;
+    // wide batches: the Δ store of the semi-naive wide path follows the facts (same layout)
+    a->fact_alloc_bytes = std::max<uint64_t>(Lo.fact_words, 4) * 8 * (Lo.wide ? 2 : 1);
     cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, a->stream);
-    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)(Lo.fact_words * 8), cudaGetErrorString(e)));
+    if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e)));
     D.facts = a->d_facts;
+    D.delta = Lo.wide ? a->d_facts + std::max<uint64_t>(Lo.fact_words, 4) : nullptr;
     size_t s_mask = align256((size_t)N * 8);
     size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
@@ -1470,24 +1512,48 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   const uint32_t N = D.n_nodes;
   uint32_t blocks = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks) : (uint32_t)a->max_blocks;
   a->launches = 0;
-  if (!a->d_facts) {                                  // released by an earlier build: re-allocate
-    const cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, s);
-    if (e != cudaSuccess) return set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e));
-    D.facts = a->d_facts;
-  }
+  gdroid_status est = ensure_facts(a);               // released by an earlier build: re-allocate
+  if (est) return est;
+  // keep_facts (incremental): the fact store keeps its content, the worklist
+  // state persists and round numbers continue, so stamps stay ordered and first-reach history
+  // is kept; only the staged seeds (plus the entries on a handle's first build) are queued.
+  const bool keep = o.keep_facts != 0 && a->state_valid;
   CU(cudaEventRecord(a->ev[0], s));
   // (a2) zero the fact matrices and the worklist state
-  CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
-  CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
-  CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
+  if (!(o.keep_facts && a->facts_valid)) CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
+  if (D.delta) CU(cudaMemsetAsync(D.delta, 0, D.n_words * 8, s));   // empty at every fixed point
+  if (!keep) {
+    CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
+    CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
+    a->round_base = 0;
+  }
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));
   CU(cudaMemsetAsync(D.stats, 0, sizeof(DevStats), s));
   CU(cudaMemsetAsync(D.bar, 0, 256, s));                 // barrier + round descriptor words
   CU(cudaMemsetAsync(D.app_digest, 0, (size_t)a->n_apps * 8, s));
+  D.round0 = a->round_base + 1;
+  D.max_rounds = o.max_rounds ? a->round_base + o.max_rounds : 0u;
+  D.push_entries = keep ? 0u : 1u;
+  if (o.keep_facts && !a->seed_nodes.empty()) {      // staged seeds -> device (stream-ordered copy)
+    const size_t nb = a->seed_nodes.size() * 4, pb = a->seed_pairs.size() * 4;
+    gdroid_status st2 = ensure_seed_buf(a, nb + pb + 8);
+    if (st2) return st2;
+    std::memcpy(a->h_seed, a->seed_nodes.data(), nb);
+    std::memcpy((char*)a->h_seed + nb, a->seed_pairs.data(), pb);
+    CU(cudaMemcpyAsync(a->d_seed, a->h_seed, nb + pb, cudaMemcpyHostToDevice, s));
+    D.seed_nodes = (const uint32_t*)a->d_seed;
+    D.seed_pairs = (const uint32_t*)((char*)a->d_seed + nb);
+    D.n_seed_nodes = (uint32_t)a->seed_nodes.size();
+    D.n_seed_pairs = (uint32_t)(a->seed_pairs.size() / 3);
+  } else {
+    D.n_seed_nodes = D.n_seed_pairs = 0;
+  }
+  a->seed_nodes.clear();
+  a->seed_pairs.clear();
   CU(launch_seed(D, s));
-  a->launches++;
+  a->launches += D.n_seed_pairs ? 2 : 1;
+  D.n_seed_nodes = D.n_seed_pairs = 0;
   CU(cudaEventRecord(a->ev[1], s));
-  D.round0 = 1;
   D.sw_lo = D.sw_hi = 0;
   if (o.loop_mode == 0 && D.hiocc && GD_HYBRID && (D.flags & F_CONT)) {
     // Hybrid (large narrow batches, default variant): light rounds run in the 3-CTA/SM
@@ -1522,7 +1588,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
     const uint32_t K = 64;
     uint32_t* h_counts = nullptr;
     CU(cudaMallocHost(&h_counts, 3 * CNT_STRIDE * 4 + 16));
-    uint32_t round = 1;
+    uint32_t round = D.round0;
     for (;;) {
       for (uint32_t q = 0; q < K; ++q) {
         cudaError_t e = launch_round(D, round + q, blocks, s);
@@ -1547,10 +1613,13 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   a->built = false;
   a->digests_ok = false;
   a->release_pending = o.release_facts != 0;
+  a->state_valid = true;
+  a->facts_valid = true;
   if (o.release_facts) {                              // stream-ordered: after the digest kernel
     CU(cudaFreeAsync(a->d_facts, s));
     a->d_facts = nullptr;
-    D.facts = nullptr;
+    D.facts = D.delta = nullptr;
+    a->facts_valid = false;
   }
   if (o.async) return GDROID_OK;
   CU(cudaStreamSynchronize(s));
@@ -1565,6 +1634,159 @@ gdroid_status gdroid_sync(gdroid_app* a, gdroid_build_stats* stats) {
   return finish_stats(a, stats);
 }
 
+// All facts of every app of the batch in one CSR over the batch's nodes (app k's nodes are
+// rows app_base[k] .. app_base[k+1]-1, each app's pairs in its own gids).  The size query
+// (pairs == NULL) keeps the per-node counts on the device, so the fetch that follows does not
+// count again; both copies go straight between the caller's (ideally pinned) buffers and HBM.
+gdroid_status gdroid_read_batch_facts(const gdroid_app* ca, uint64_t* ptr, uint64_t* pairs, uint64_t cap) {
+  gdroid_app* a = const_cast<gdroid_app*>(ca);
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (!a->built) return set_err(GDROID_E_STATE, "facts read before a completed build");
+  if (!ptr) return set_err(GDROID_E_INVALID, "ptr is NULL");
+  DeviceGuard guard(a->device);
+  const uint32_t n = a->app_base[a->n_apps];
+  const bool cached = pairs && a->counts_build == a->build_serial;
+  if (!cached) {
+    gdroid_status st = ensure_scratch(a, (size_t)(n + 1) * 8);
+    if (st) return st;
+    CU(a->last_plain ? launch_plain_sizes(a->P, 0, n, a->d_scratch, a->stream)
+                     : launch_popc(a->D, 0, n, a->d_scratch, a->stream));
+    CU(cudaMemcpyAsync(ptr + 1, a->d_scratch, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
+    CU(cudaStreamSynchronize(a->stream));
+    ptr[0] = 0;
+    for (uint32_t i = 0; i < n; ++i) ptr[i + 1] += ptr[i];
+    a->counts_build = a->build_serial;
+  }
+  const uint64_t total = ptr[n];
+  if (!pairs) return GDROID_OK;
+  if (cap < total) return set_err(GDROID_E_SMALLBUF, "need %llu pairs, cap %llu", (unsigned long long)total, (unsigned long long)cap);
+  gdroid_status st = ensure_scratch(a, (size_t)(n + 1) * 8 + (size_t)total * 8 + 8);
+  if (st) return st;
+  uint64_t* d_ptr = a->d_scratch;
+  uint64_t* d_pairs = a->d_scratch + (n + 1);
+  CU(cudaMemcpyAsync(d_ptr, ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, a->stream));
+  CU(a->last_plain ? launch_plain_gather(a->P, 0, n, d_ptr, d_pairs, a->stream)
+                   : launch_expand(a->D, 0, n, d_ptr, d_pairs, a->stream));
+  CU(cudaMemcpyAsync(pairs, d_pairs, (size_t)total * 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  return GDROID_OK;
+}
+
+// ---------------------------------------------------------------- incremental / out-of-core
+gdroid_status gdroid_stage_seeds(gdroid_app* a, uint32_t k, uint32_t n, const uint32_t* nodes,
+                                 const uint64_t* ptr, const uint64_t* pairs) {
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (k >= a->n_apps) return set_err(GDROID_E_RANGE, "app index %u >= %u", k, a->n_apps);
+  if (n && (!nodes || !ptr)) return set_err(GDROID_E_INVALID, "nodes / ptr is NULL");
+  const uint32_t n0 = a->app_base[k], nn = a->app_base[k + 1] - n0;
+  for (uint32_t i = 0; i < n; ++i) {
+    if (nodes[i] >= nn) return set_err(GDROID_E_RANGE, "seed %u: node %u >= %u", i, nodes[i], nn);
+    if (ptr[i + 1] < ptr[i]) return set_err(GDROID_E_INVALID, "seed ptr not monotone at %u", i);
+  }
+  for (uint32_t i = 0; i < n; ++i) {
+    a->seed_nodes.push_back(n0 + nodes[i]);
+    for (uint64_t q = ptr[i]; q < ptr[i + 1]; ++q) {
+      a->seed_pairs.push_back(n0 + nodes[i]);
+      a->seed_pairs.push_back((uint32_t)(pairs[q] >> 32));
+      a->seed_pairs.push_back((uint32_t)pairs[q]);
+    }
+  }
+  return GDROID_OK;
+}
+
+// Facts of a list of nodes of app k (app-local ids) as CSR (ptr[n+1], pairs); two-call like
+// gdroid_read_all_facts.  Used to read the boundary proxies of out-of-core sub-graphs.
+gdroid_status gdroid_read_nodes_facts(const gdroid_app* ca, uint32_t k, uint32_t n, const uint32_t* nodes,
+                                      uint64_t* ptr, uint64_t* pairs, uint64_t cap) {
+  gdroid_app* a = const_cast<gdroid_app*>(ca);
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (!a->built) return set_err(GDROID_E_STATE, "facts read before a completed build");
+  if (k >= a->n_apps) return set_err(GDROID_E_RANGE, "app index %u >= %u", k, a->n_apps);
+  if (!ptr || (n && !nodes)) return set_err(GDROID_E_INVALID, "ptr / nodes is NULL");
+  DeviceGuard guard(a->device);
+  const uint32_t n0 = a->app_base[k], nn = a->app_base[k + 1] - n0;
+  std::vector<uint32_t> gl(n);
+  for (uint32_t i = 0; i < n; ++i) {
+    if (nodes[i] >= nn) return set_err(GDROID_E_RANGE, "node %u >= %u", nodes[i], nn);
+    gl[i] = n0 + nodes[i];
+  }
+  ptr[0] = 0;
+  if (n == 0) return GDROID_OK;
+  const size_t lw = (n + 1) / 2 + 1;                  // list words (u32 pairs) at the scratch start
+  gdroid_status st = ensure_scratch(a, (lw + n + 1) * 8);
+  if (st) return st;
+  uint32_t* d_list = (uint32_t*)a->d_scratch;
+  uint64_t* d_cnt = a->d_scratch + lw;
+  CU(cudaMemcpyAsync(d_list, gl.data(), (size_t)n * 4, cudaMemcpyHostToDevice, a->stream));
+  CU(launch_popc(a->D, 0, n, d_cnt, a->stream, d_list));
+  CU(cudaMemcpyAsync(ptr + 1, d_cnt, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  for (uint32_t i = 0; i < n; ++i) ptr[i + 1] += ptr[i];
+  const uint64_t total = ptr[n];
+  if (!pairs) return GDROID_OK;
+  if (cap < total) return set_err(GDROID_E_SMALLBUF, "need %llu pairs, cap %llu", (unsigned long long)total, (unsigned long long)cap);
+  st = ensure_scratch(a, (lw + n + 1 + total + 1) * 8);
+  if (st) return st;
+  d_list = (uint32_t*)a->d_scratch;
+  d_cnt = a->d_scratch + lw;
+  CU(cudaMemcpyAsync(d_list, gl.data(), (size_t)n * 4, cudaMemcpyHostToDevice, a->stream));
+  CU(cudaMemcpyAsync(d_cnt, ptr, (size_t)(n + 1) * 8, cudaMemcpyHostToDevice, a->stream));
+  CU(launch_expand(a->D, 0, n, d_cnt, d_cnt + n + 1, a->stream, d_list));
+  CU(cudaMemcpyAsync(pairs, d_cnt + n + 1, (size_t)total * 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_read_reached(const gdroid_app* ca, uint32_t k, uint32_t n, const uint32_t* nodes, uint8_t* out) {
+  gdroid_app* a = const_cast<gdroid_app*>(ca);
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (!a->digests_ok) return set_err(GDROID_E_STATE, "read before a completed build");
+  if (k >= a->n_apps) return set_err(GDROID_E_RANGE, "app index %u >= %u", k, a->n_apps);
+  DeviceGuard guard(a->device);
+  const uint32_t n0 = a->app_base[k], nn = a->app_base[k + 1] - n0;
+  std::vector<uint32_t> st(nn);
+  CU(cudaMemcpyAsync(st.data(), a->D.stamp + n0, (size_t)nn * 4, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  for (uint32_t i = 0; i < n; ++i) {
+    if (nodes[i] >= nn) return set_err(GDROID_E_RANGE, "node %u >= %u", nodes[i], nn);
+    out[i] = st[nodes[i]] != 0;
+  }
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_export_facts(const gdroid_app* ca, void* host, uint64_t bytes) {
+  gdroid_app* a = const_cast<gdroid_app*>(ca);
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (!a->d_facts || !a->facts_valid) return set_err(GDROID_E_STATE, "no facts to export");
+  if (bytes != a->D.n_words * 8) return set_err(GDROID_E_SMALLBUF, "fact store is %llu B", (unsigned long long)(a->D.n_words * 8));
+  if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
+  DeviceGuard guard(a->device);
+  CU(cudaMemcpyAsync(host, a->d_facts, bytes, cudaMemcpyDeviceToHost, a->stream));
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_import_facts(gdroid_app* a, const void* host, uint64_t bytes) {
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (bytes != a->D.n_words * 8) return set_err(GDROID_E_SMALLBUF, "fact store is %llu B", (unsigned long long)(a->D.n_words * 8));
+  if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
+  DeviceGuard guard(a->device);
+  gdroid_status st = ensure_facts(a);
+  if (st) return st;
+  CU(cudaMemcpyAsync(a->d_facts, host, bytes, cudaMemcpyHostToDevice, a->stream));
+  a->facts_valid = true;
+  a->built = false;                                   // facts no longer those of a build
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_stream_sync(gdroid_app* a) {
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  DeviceGuard guard(a->device);
+  CU(cudaStreamSynchronize(a->stream));
+  return GDROID_OK;
+}
+
+uint64_t gdroid_fact_bytes(const gdroid_app* a) { return a ? a->D.n_words * 8 : 0; }
+
 gdroid_status gdroid_release_facts(gdroid_app* a) {
   if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
   if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
@@ -1572,7 +1794,8 @@ gdroid_status gdroid_release_facts(gdroid_app* a) {
   DeviceGuard guard(a->device);
   CU(cudaFreeAsync(a->d_facts, a->stream));
   a->d_facts = nullptr;
-  a->D.facts = nullptr;
+  a->D.facts = a->D.delta = nullptr;
+  a->facts_valid = false;
   a->built = false;                                   // digests stay readable
   return GDROID_OK;
 }
