@@ -50,7 +50,7 @@ def parse(argv=None):
                     choices=["corpus1000", "corpus8", "median", "small", "worst"])
     ap.add_argument("--n-apps", type=int, default=1000, help="corpus1000: apps of the corpus")
     ap.add_argument("--apps-per-rank", type=int, default=8, help="corpus8: apps per rank")
-    ap.add_argument("--node-budget", type=int, default=4_000_000, help="narrow apps per batch (nodes)")
+    ap.add_argument("--node-budget", type=int, default=16_000_000, help="narrow apps per batch (nodes)")
     ap.add_argument("--wide-per-batch", type=int, default=1)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -132,9 +132,15 @@ typedef struct {
  *   PLAIN    the set-based plain implementation (Alg. 2): per-node sorted
  *            pair arrays with regrowth from a device bump allocator, one thread per node,
  *            per-thread switch over node kinds; needs a handle loaded with
- *            gdroid_load_icfg_plain (one app)                                               */
+ *            gdroid_load_icfg_plain (one app)
+ *   CELL     the paper's own MAT layout (Fig. 5b): one
+ *            cell-major matrix per method (rows = the method's slot pool, columns = its
+ *            instance pool, cell = an n_m-bit mask over the method's statements), run by the
+ *            PLAIN schedule (thread per node: IN(n) gathered from bit n of every cell, unions
+ *            = one atomicOr per pair); the facts are converted to the node-major store for
+ *            readback.  Needs a gdroid_load_icfg_plain handle; fact_bytes = the cell store. */
 typedef enum { GDROID_V_DEFAULT = 0, GDROID_V_MAT = 1, GDROID_V_MAT_GRP = 2, GDROID_V_GDROID = 3,
-               GDROID_V_PLAIN = 4 } gdroid_variant;
+               GDROID_V_PLAIN = 4, GDROID_V_CELL = 5 } gdroid_variant;
 
 /* Device-counted statistics of the last build (DESIGN.md §5 byte models). */
 typedef struct {

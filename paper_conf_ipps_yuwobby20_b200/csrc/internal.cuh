@@ -21,6 +21,10 @@ constexpr uint32_t HIOCC_NODES = GD_HIOCC_NODES;   // batches this large are ite
 #define GD_THREADS 256
 #endif
 constexpr int THREADS = GD_THREADS; // fixed-point kernel block size
+#ifndef GD_SMASK
+#define GD_SMASK 0             // narrow blocks: read only word groups flagged in D.smask (measured
+                               // slower, round 1); 0: D.smask is not allocated
+#endif
 constexpr int WARPS = THREADS / 32;
 
 // One ICFG node (64 B).  Row indices r* are relative to the node's fact block (method-local
@@ -230,11 +234,28 @@ struct PlainDev {
   uint32_t* stamp; uint32_t* queue; uint32_t* counts; uint32_t* bar; uint32_t* err;
   DevStats* stats;
   uint64_t* node_digest; unsigned long long* app_digest;
+  // CELL variant: the paper's cell-major per-method matrix (Fig. 5b,
+  // PAPER.md:871-904): method m owns rows (locals, then the module's global rows in gid order)
+  // x columns (its module's instance pool); cell (r, c) is an n_m-bit mask over m's nodes.
+  uint32_t cell;                // 1: this build runs on the cell store instead of the pair sets
+  uint32_t n_methods;
+  uint64_t* cells;              // the cell store (cell_words words)
+  uint64_t cell_words;
+  const uint64_t* m_coff;       // [M] word offset of method m's matrix
+  const uint32_t* m_rows;       // [M] |P_m|
+  const uint32_t* m_cols;       // [M] |Q_m|
+  const uint32_t* m_wpc;        // [M] words per cell = ceil(n_m / 64)
+  const uint32_t* nidx;         // [N] index of node n among its method's nodes
+  const uint32_t* mnode_ptr;    // [M+1] CSR of each method's nodes in index order
+  const uint32_t* mnodes;
+  const uint32_t* mgrow_ptr;    // [Dm+1] CSR of each module's global-row slot gids (ascending)
+  const uint32_t* mgrow;
 };
 
 int plain_max_blocks(int device);
 cudaError_t launch_plain(const PlainDev& P, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_plain_digest(const PlainDev& P, cudaStream_t s);
+cudaError_t launch_cell_to_mat(const PlainDev& P, const Dev& D, cudaStream_t s);
 cudaError_t launch_plain_sizes(const PlainDev& P, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s);
 cudaError_t launch_plain_gather(const PlainDev& P, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
                                 cudaStream_t s);

@@ -37,9 +37,6 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_CONT_LOAD
 #define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
 #endif
-#ifndef GD_SMASK
-#define GD_SMASK 0             // narrow blocks: read only word groups flagged in D.smask (measured slower)
-#endif
 #ifndef GD_INL
 #define GD_INL 1               // chunk-0 INTRA/C2R edges read from the inline record (one hop less)
 #endif

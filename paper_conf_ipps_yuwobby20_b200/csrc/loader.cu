@@ -1236,7 +1236,38 @@ gdroid_status load_plain(gdroid_app* a, const gdroid_icfg_desc* d) {
                o_np = take(M * 4), o_mm = take(M * 4), o_ip = take((Dm + 1) * 8), o_is = take(n_insts * 4),
                o_sp = take((Dm + 1) * 8), o_ss = take(n_stat * 4), o_it = take(I * 4), o_tp = take((T + 1) * 8),
                o_tf = take(n_tf * 4), o_hb = take((I + 1) * 8), o_en = take((size_t)d->n_entries * 4);
+  // CELL variant tables: per-method matrix geometry, node index inside its
+  // method, each method's node list and each module's global-row gids in ascending order
+  std::vector<uint32_t> m_rows(M), m_cols(M), m_wpc(M), nidx(N), mcount(M, 0), mnode_ptr(M + 1, 0), mnodes(N);
+  std::vector<uint64_t> m_coff(M);
+  for (uint64_t n = 0; n < N; ++n) nidx[n] = mcount[d->node_method[n]]++;
+  for (uint64_t m = 0; m < M; ++m) mnode_ptr[m + 1] = mnode_ptr[m] + mcount[m];
+  for (uint64_t n = 0; n < N; ++n) mnodes[mnode_ptr[d->node_method[n]] + nidx[n]] = (uint32_t)n;
+  std::vector<uint32_t> mgrow_ptr(Dm + 1, 0), mgrow;
+  for (uint64_t q = 0; q < Dm; ++q) {
+    for (uint64_t k = d->module_static_ptr[q]; k < d->module_static_ptr[q + 1]; ++k)
+      mgrow.push_back((uint32_t)(local_base[M] + d->module_statics[k]));
+    for (uint64_t k = d->module_inst_ptr[q]; k < d->module_inst_ptr[q + 1]; ++k) {
+      const uint32_t o = d->module_insts[k];
+      for (uint64_t f = heap_base[o]; f < heap_base[o + 1]; ++f)
+        mgrow.push_back((uint32_t)(local_base[M] + d->n_statics + f));
+    }
+    mgrow_ptr[q + 1] = (uint32_t)mgrow.size();
+  }
+  uint64_t cell_words = 0;
+  for (uint64_t m = 0; m < M; ++m) {
+    const uint32_t q = d->method_module[m];
+    m_rows[m] = d->method_n_locals[m] + (mgrow_ptr[q + 1] - mgrow_ptr[q]);
+    m_cols[m] = (uint32_t)(d->module_inst_ptr[q + 1] - d->module_inst_ptr[q]);
+    m_wpc[m] = std::max<uint32_t>(1, (mcount[m] + 63) / 64);
+    m_coff[m] = cell_words;
+    cell_words += (uint64_t)m_rows[m] * m_cols[m] * m_wpc[m];
+  }
+  const size_t o_mrows = take(M * 4), o_mcols = take(M * 4), o_mwpc = take(M * 4), o_mcoff = take(M * 8),
+               o_nidx = take(N * 4), o_mnp = take((M + 1) * 4), o_mnodes = take(N * 4),
+               o_mgp = take((Dm + 1) * 4), o_mg = take(std::max<size_t>(mgrow.size(), 1) * 4);
   const size_t in_bytes = off;
+  const size_t o_cells = take(std::max<uint64_t>(cell_words, 1) * 8);
   const size_t o_sets = take(N * sizeof(SetDesc)), o_locks = take(N * 4), o_stamp = take(N * 4),
                o_queue = take(3 * N * 4), o_counts = take(256), o_bar = take(256), o_err = take(256),
                o_top = take(256);
@@ -1265,6 +1296,10 @@ gdroid_status load_plain(gdroid_app* a, const gdroid_icfg_desc* d) {
   put(o_sp, d->module_static_ptr, (Dm + 1) * 8); put(o_ss, d->module_statics, n_stat * 4);
   put(o_it, d->inst_type, I * 4); put(o_tp, d->type_field_ptr, (T + 1) * 8); put(o_tf, d->type_fields, n_tf * 4);
   put(o_hb, heap_base.data(), (I + 1) * 8); put(o_en, d->entries, (size_t)d->n_entries * 4);
+  put(o_mrows, m_rows.data(), M * 4); put(o_mcols, m_cols.data(), M * 4); put(o_mwpc, m_wpc.data(), M * 4);
+  put(o_mcoff, m_coff.data(), M * 8); put(o_nidx, nidx.data(), N * 4); put(o_mnp, mnode_ptr.data(), (M + 1) * 4);
+  put(o_mnodes, mnodes.data(), N * 4); put(o_mgp, mgrow_ptr.data(), (Dm + 1) * 4);
+  put(o_mg, mgrow.data(), mgrow.size() * 4);
   CU(cudaMemcpy(mem, h.data(), in_bytes, cudaMemcpyHostToDevice));
   PlainDev& P = a->P;
   P.row_ptr = (const uint64_t*)(B + o_rp); P.col = (const uint32_t*)(B + o_col); P.ekind = (const uint8_t*)(B + o_ek);
@@ -1283,6 +1318,13 @@ gdroid_status load_plain(gdroid_app* a, const gdroid_icfg_desc* d) {
   P.scratch = (uint64_t*)(B + o_scr); P.maxset = maxset;
   P.heap = (uint64_t*)(B + o_heap); P.heap_cap = heap_bytes / 8;
   P.stats = a->D.stats; P.node_digest = a->D.node_digest; P.app_digest = a->D.app_digest;
+  P.cell = 0; P.n_methods = (uint32_t)M;
+  P.cells = (uint64_t*)(B + o_cells); P.cell_words = cell_words;
+  P.m_rows = (const uint32_t*)(B + o_mrows); P.m_cols = (const uint32_t*)(B + o_mcols);
+  P.m_wpc = (const uint32_t*)(B + o_mwpc); P.m_coff = (const uint64_t*)(B + o_mcoff);
+  P.nidx = (const uint32_t*)(B + o_nidx); P.mnode_ptr = (const uint32_t*)(B + o_mnp);
+  P.mnodes = (const uint32_t*)(B + o_mnodes); P.mgrow_ptr = (const uint32_t*)(B + o_mgp);
+  P.mgrow = (const uint32_t*)(B + o_mg);
   a->plain_blocks = blocks;
   return GDROID_OK;
 }
@@ -1291,9 +1333,14 @@ gdroid_status load_plain(gdroid_app* a, const gdroid_icfg_desc* d) {
 // and stats as the MAT path; alg_bytes = live set bytes, dense_bytes = allocated set bytes
 // (Fig. 10 footprint), atomics = array (re)allocations).
 gdroid_status build_plain(gdroid_app* a, const gdroid_build_opts& o, gdroid_build_stats* stats) {
-  if (!a->d_plain) return set_err(GDROID_E_STATE, "PLAIN variant needs a handle loaded with gdroid_load_icfg_plain");
+  if (!a->d_plain) return set_err(GDROID_E_STATE, "PLAIN / CELL variants need a handle loaded with gdroid_load_icfg_plain");
   PlainDev& P = a->P;
   P.max_rounds = o.max_rounds;
+  P.cell = o.variant == GDROID_V_CELL ? 1u : 0u;
+  if (P.cell) {
+    gdroid_status est = ensure_facts(a);             // the MAT store receives the converted facts
+    if (est) return est;
+  }
   cudaStream_t s = a->stream;
   const uint32_t N = P.n_nodes;
   a->launches = 0;
@@ -1308,11 +1355,20 @@ gdroid_status build_plain(gdroid_app* a, const gdroid_build_opts& o, gdroid_buil
   CU(cudaMemsetAsync(a->D.stats, 0, sizeof(DevStats), s));
   CU(cudaMemsetAsync(a->D.app_digest, 0, 8, s));
   CU(cudaEventRecord(a->ev[1], s));
+  if (P.cell) CU(cudaMemsetAsync(P.cells, 0, P.cell_words * 8, s));
   CU(launch_plain(P, (uint32_t)a->plain_blocks, s));
   a->launches += 2;
   CU(cudaEventRecord(a->ev[2], s));
-  CU(launch_plain_digest(P, s));
-  a->launches++;
+  if (P.cell) {                                       // cells -> node-major, then the MAT digests
+    CU(cudaMemsetAsync(a->D.facts, 0, a->D.n_words * 8, s));
+    CU(launch_cell_to_mat(P, a->D, s));
+    CU(launch_digest(a->D, s));
+    CU(cudaMemsetAsync(&a->D.stats->dense_bytes, 0, 8, s));
+    a->launches += 2;
+  } else {
+    CU(launch_plain_digest(P, s));
+    a->launches++;
+  }
   CU(cudaEventRecord(a->ev[3], s));
   CU(cudaMemcpyAsync(a->h_stats, a->D.stats, sizeof(DevStats), cudaMemcpyDeviceToHost, s));
   uint32_t err = 0;
@@ -1320,9 +1376,10 @@ gdroid_status build_plain(gdroid_app* a, const gdroid_build_opts& o, gdroid_buil
   CU(cudaStreamSynchronize(s));
   a->pending = true;
   a->digests_ok = false;
-  a->last_plain = true;
+  a->last_plain = !P.cell;                            // CELL reads back from the converted MAT store
   gdroid_status st = finish_stats(a, stats);
-  a->last.fact_bytes = a->h_stats->dense_bytes;
+  a->last.fact_bytes = P.cell ? P.cell_words * 8 : a->h_stats->dense_bytes;
+  if (P.cell) { a->facts_valid = true; a->built = true; }
   if (stats) stats->fact_bytes = a->last.fact_bytes;
   if (err) {
     a->built = false;
@@ -1454,7 +1511,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e)));
     D.facts = a->d_facts;
     D.delta = Lo.wide ? a->d_facts + std::max<uint64_t>(Lo.fact_words, 4) : nullptr;
-    size_t s_mask = align256((size_t)N * 8);
+    size_t s_mask = GD_SMASK ? align256((size_t)N * 8) : 256;
     size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t st = s_mask + s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
@@ -1495,7 +1552,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   DeviceGuard guard(a->device);
   Dev& D = a->D;
   D.max_rounds = o.max_rounds;
-  if (o.variant == GDROID_V_PLAIN) return build_plain(a, o, stats);
+  if (o.variant == GDROID_V_PLAIN || o.variant == GDROID_V_CELL) return build_plain(a, o, stats);
   if (o.variant > GDROID_V_GDROID) return set_err(GDROID_E_INVALID, "unknown variant %u", o.variant);
   a->last_plain = false;
   static const uint32_t vflags[4] = {F_GRP | F_CONT, 0u, F_GRP, F_GRP | F_MER};
@@ -1524,7 +1581,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   if (D.delta) CU(cudaMemsetAsync(D.delta, 0, D.n_words * 8, s));   // empty at every fixed point
   if (!keep) {
     CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
-    CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
+    if (GD_SMASK) CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
     a->round_base = 0;
   }
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));

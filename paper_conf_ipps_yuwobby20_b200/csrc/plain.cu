@@ -263,6 +263,64 @@ __device__ bool union_into(const PlainDev& P, uint32_t s, const uint64_t* T, uin
   return true;
 }
 
+// ---- CELL variant: the cell-major per-method matrix store (Fig. 5b)
+// row of slot gid `sl` in method m's matrix (locals first, then the module's global rows)
+__device__ int64_t cell_row(const PlainDev& P, uint32_t m, uint64_t sl) {
+  if (sl >= P.local_base[m] && sl < P.local_base[m + 1]) return (int64_t)(sl - P.local_base[m]);
+  const uint32_t d = P.mmod[m];
+  uint32_t lo = P.mgrow_ptr[d], hi = P.mgrow_ptr[d + 1];
+  const uint32_t base = lo;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (P.mgrow[mid] < sl) lo = mid + 1; else hi = mid;
+  }
+  if (lo < P.mgrow_ptr[d + 1] && P.mgrow[lo] == sl) return (int64_t)(P.local_base[m + 1] - P.local_base[m]) + (lo - base);
+  return -1;
+}
+__device__ int64_t cell_col(const PlainDev& P, uint32_t m, uint32_t o) {
+  const uint32_t d = P.mmod[m];
+  uint64_t lo = P.inst_ptr[d], hi = P.inst_ptr[d + 1];
+  const uint64_t base = lo;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (P.insts[mid] < o) lo = mid + 1; else hi = mid;
+  }
+  return (lo < P.inst_ptr[d + 1] && P.insts[lo] == o) ? (int64_t)(lo - base) : -1;
+}
+
+// IN(n) from the cell store: bit nidx(n) of every cell of its method's matrix, row-major =
+// ascending (slot gid, instance gid).  Read through L2 (cells are OR-ed by other threads).
+__device__ uint64_t cell_gather(const PlainDev& P, uint32_t n, uint64_t* A) {
+  const uint32_t m = P.nmeth[n], d = P.mmod[m];
+  const uint32_t rows = P.m_rows[m], cols = P.m_cols[m], wpc = P.m_wpc[m], i = P.nidx[n];
+  const uint64_t* C = P.cells + P.m_coff[m] + (i >> 6);
+  const uint64_t bit = 1ull << (i & 63);
+  const uint32_t nloc = (uint32_t)(P.local_base[m + 1] - P.local_base[m]);
+  uint64_t k = 0;
+  for (uint32_t r = 0; r < rows; ++r) {
+    const uint64_t sl = r < nloc ? P.local_base[m] + r : P.mgrow[P.mgrow_ptr[d] + (r - nloc)];
+    for (uint32_t c = 0; c < cols; ++c)
+      if (__ldcg(C + ((uint64_t)r * cols + c) * wpc) & bit) A[k++] = pack(sl, P.insts[P.inst_ptr[d] + c]);
+  }
+  return k;
+}
+
+// IN(s) ∪= T on the cell store: one atomicOr of bit nidx(s) per pair; grew = some bit was new.
+__device__ bool cell_union(const PlainDev& P, uint32_t s, const uint64_t* T, uint64_t nt) {
+  const uint32_t m = P.nmeth[s], cols = P.m_cols[m], wpc = P.m_wpc[m], i = P.nidx[s];
+  uint64_t* C = P.cells + P.m_coff[m] + (i >> 6);
+  const uint64_t bit = 1ull << (i & 63);
+  bool grew = false;
+  for (uint64_t j = 0; j < nt; ++j) {
+    const int64_t r = cell_row(P, m, slot_of(T[j])), c = cell_col(P, m, (uint32_t)T[j]);
+    if (r < 0 || c < 0) { atomicExch(P.err, 2u); continue; }           // outside P_m x Q_m (never: π)
+    unsigned long long* w = (unsigned long long*)(C + ((uint64_t)r * cols + (uint64_t)c) * wpc);
+    if (__ldcg((const uint64_t*)w) & bit) continue;                     // (IN only grows)
+    if (!(atomicOr(w, bit) & bit)) grew = true;
+  }
+  return grew;
+}
+
 __device__ __forceinline__ void push(const PlainDev& P, uint32_t s, uint32_t round) {
   if (atomicMax(&P.stamp[s], round + 1) < round + 1) {                      // set insert (dedupe)
     const uint32_t q = (round + 1) % 3;
@@ -316,18 +374,23 @@ __global__ void __launch_bounds__(128) k_plain_fixpoint(PlainDev P) {
     for (uint64_t it = tid; it < total; it += nth) {                         // l.9-11: thread per node
       const uint32_t n = __ldcg(&P.queue[(size_t)cur * P.n_nodes + it]);
       ++visits;
-      lock(&P.locks[n]);                                                     // snapshot of IN(n)
-      const uint64_t off = __ldcg(&P.sets[n].off);
-      const uint32_t sz = __ldcg(&P.sets[n].size);
-      for (uint32_t i = 0; i < sz; ++i) A[i] = __ldcg(P.heap + off + i);
-      unlock(&P.locks[n]);
+      uint64_t sz;
+      if (P.cell) {
+        sz = cell_gather(P, n, A);                                           // IN(n) from the cells
+      } else {
+        lock(&P.locks[n]);                                                   // snapshot of IN(n)
+        const uint64_t off = __ldcg(&P.sets[n].off);
+        sz = __ldcg(&P.sets[n].size);
+        for (uint32_t i = 0; i < sz; ++i) A[i] = __ldcg(P.heap + off + i);
+        unlock(&P.locks[n]);
+      }
       const uint64_t ny = transfer(P, n, A, sz, B, C);                      // l.12 GEN_KILL
       for (uint64_t e = P.row_ptr[n]; e < P.row_ptr[n + 1]; ++e) {          // l.13-17
         const uint32_t s = P.col[e], k = P.ekind[e];
         const uint64_t* T = B;
         uint64_t nt = ny;
         if (k != GE_INTRA) { nt = edge_transform(P, n, s, k, B, ny, C); T = C; }
-        const bool grew = union_into(P, s, T, nt, allocs);
+        const bool grew = P.cell ? cell_union(P, s, T, nt) : union_into(P, s, T, nt, allocs);
         if (grew || __ldcg(&P.stamp[s]) == 0) push(P, s, round);
       }
     }
@@ -377,7 +440,38 @@ __global__ void k_plain_digest(PlainDev P) {
   }
 }
 
+// CELL -> node-major MAT store (readback and digests then use the MAT path's kernels): one
+// warp per method, lanes over its cells; bit i of cell (r, c) -> word (r << logW) + c/64 of
+// IN(node i).  Rows and columns are ordered as the node-major block's (locals, globals in gid
+// order; sorted pool), so only the node changes.
+__global__ void k_cell_to_mat(PlainDev P, Dev D, uint32_t M) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t m = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); m < M; m += nw) {
+    const uint32_t rows = P.m_rows[m], cols = P.m_cols[m], wpc = P.m_wpc[m];
+    const uint64_t ncell = (uint64_t)rows * cols;
+    for (uint64_t q = lane; q < ncell; q += 32) {
+      const uint32_t r = (uint32_t)(q / cols), c = (uint32_t)(q % cols);
+      for (uint32_t w = 0; w < wpc; ++w) {
+        uint64_t x = P.cells[P.m_coff[m] + q * wpc + w];
+        while (x) {
+          const int b = __ffsll((long long)x) - 1;
+          x &= x - 1;
+          const uint32_t node = P.mnodes[P.mnode_ptr[m] + w * 64 + b];
+          const NodeRec R = D.nodes[node];
+          atomicOr((unsigned long long*)(D.facts + R.off + ((uint64_t)r << R.logW) + (c >> 6)), 1ull << (c & 63));
+        }
+      }
+    }
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_cell_to_mat(const PlainDev& P, const Dev& D, cudaStream_t s) {
+  k_cell_to_mat<<<1184, 256, 0, s>>>(P, D, P.n_methods);
+  return cudaGetLastError();
+}
 
 int plain_max_blocks(int device) {
   int sms = 0, occ = 0;

@@ -26,7 +26,7 @@ import time
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
-VARIANTS = ["plain", "mat", "mat_grp", "gdroid", "default"]
+VARIANTS = ["plain", "mat", "mat_grp", "gdroid", "default", "cell"]
 
 
 def sample_ids(n_apps, n_corpus=1000, max_nodes=None):
@@ -45,6 +45,8 @@ def main():
     ap.add_argument("--apps", type=int, default=24)
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--max-nodes", type=int, default=700_000, help="skip larger apps (plain is slow)")
+    ap.add_argument("--cell-max-nodes", type=int, default=150_000,
+                    help="CELL (cell-major matrices, SURVEY §8(f)2) only on apps up to this size (a visit gathers |P_m| x |Q_m| cells)")
     ap.add_argument("--out", default=os.path.join(ROOT, "gpurun_out", "ablation.json"))
     args = ap.parse_args()
 
@@ -63,6 +65,8 @@ def main():
         row = {"app": i, "nodes": g.n_nodes, "edges": int(g.n_edges)}
         ref = None
         for v in VARIANTS:
+            if v == "cell" and g.n_nodes > args.cell_max_nodes:
+                continue
             app.build(variant=v)                               # warm-up
             ts, st = [], None
             for _ in range(args.reps):
@@ -74,14 +78,15 @@ def main():
             row[v] = {"ms": statistics.median(ts), "rounds": st["rounds"], "visits": st["node_visits"],
                       "fact_bytes": st["fact_bytes"], "digest": str(dig)}
         for v in VARIANTS:
-            assert row[v]["digest"] == str(ref), f"app {i}: {v} digest differs from the default path"
+            if v in row:
+                assert row[v]["digest"] == str(ref), f"app {i}: {v} digest differs from the default path"
         app.free()
         rows.append(row)
-        print(f"app {i:4d} nodes {g.n_nodes:8d}  " + "  ".join(f"{v} {row[v]['ms']:9.2f}" for v in VARIANTS)
+        print(f"app {i:4d} nodes {g.n_nodes:8d}  " + "  ".join(f"{v} {row[v]['ms']:9.2f}" for v in VARIANTS if v in row)
               + f"  ({time.time() - t0:.1f}s)", flush=True)
 
     def ratio(a, b):
-        return [r[a]["ms"] / r[b]["ms"] for r in rows]
+        return [r[a]["ms"] / r[b]["ms"] for r in rows if a in r and b in r]
 
     def summ(x):
         x = sorted(x)
@@ -99,6 +104,8 @@ def main():
         "default_vs_plain": summ(ratio("plain", "default")),
         "default_vs_gdroid": summ(ratio("gdroid", "default")),
         "fig10_set_bytes_over_mat_bytes": summ(mem),
+        "f2_mat_vs_cell": summ(ratio("cell", "mat")),
+        "f2_cell_bytes_over_mat_bytes": summ([r["cell"]["fact_bytes"] / r["mat"]["fact_bytes"] for r in rows if "cell" in r]),
         "paper": {"mat_vs_plain_avg": 26.7, "grp_vs_mat_note": "<1.5x for 76.3% of apps, <1x for 15.5%",
                   "mer_vs_mat_grp_avg": 1.94, "gdroid_vs_plain_avg": 71.3, "mat_memory": "-75% on average",
                   "hardware": "NVIDIA Tesla P40 (PAPER.md:1090-1100)"},

@@ -66,14 +66,14 @@ def _check(app, k, g, ref):
 
 @pytest.mark.parametrize("name,variant", [("small", "default"), ("median", "default"), ("worst", "default"),
                                           ("small", "mat"), ("median", "mat_grp"), ("median", "gdroid"),
-                                          ("small", "plain")])
+                                          ("small", "plain"), ("small", "cell")])
 def test_preset_full_size(name, variant):
     fx = _fixture()
     if name not in fx:
         pytest.skip(f"{name} not in fixture")
     ref = fx[name]
     g = G.preset(name)
-    app = gd.load(g, plain=(variant == "plain"))
+    app = gd.load(g, plain=(variant in ("plain", "cell")))
     app.build(variant=variant)
     per, dig = app.node_digests()
     assert str(dig) == ref["app_digest"]

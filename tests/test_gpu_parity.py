@@ -260,3 +260,22 @@ def test_hybrid_schedule_limits_and_async():
     app.build(blocks=37)
     assert str(int(app.app_digests()[0])) == fx["median"]["app_digest"]
     app.free()
+
+
+@pytest.mark.parametrize("chunk", range(2))
+def test_cell_major_variant_random(chunk):
+    """CELL: the paper's cell-major per-method matrices (Fig. 5b)
+    as the fact store of the thread-per-node schedule, on 60 random tiny ICFGs (narrow and wide
+    pools, arity up to 5) and the hand goldens — pair for pair against the oracle."""
+    gs = [random_tiny(s, wide_pad=(80 if s % 4 == 0 else 0)) for s in range(13000 + chunk * 30, 13030 + chunk * 30)]
+    if chunk == 0:
+        gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0]]
+    for g in gs:
+        app = gd.load(g, plain=True)
+        st = app.build(variant="cell")
+        r = oracle.build_idfg(g)
+        _assert_same(app, 0, g, r, f"cell/{g.name}")
+        per, dig = app.node_digests()
+        assert dig == r.app_digest and np.array_equal(per, r.node_digest)
+        assert st["fact_bytes"] > 0
+        app.free()
