@@ -138,9 +138,14 @@ typedef struct {
  *            instance pool, cell = an n_m-bit mask over the method's statements), run by the
  *            PLAIN schedule (thread per node: IN(n) gathered from bit n of every cell, unions
  *            = one atomicOr per pair); the facts are converted to the node-major store for
- *            readback.  Needs a gdroid_load_icfg_plain handle; fact_bytes = the cell store. */
+ *            readback.  Needs a gdroid_load_icfg_plain handle; fact_bytes = the cell store.
+ *   SBDA     the paper's two-level decomposition (§III-A2, Fig. 3; Alg. 2
+ *            l.6 mid <- blockIdx.x): per pass, every method with queued nodes is claimed by
+ *            one CTA, which runs that method's worklist to local quiescence in shared memory
+ *            (__syncthreads between local rounds); CALL / RET successors start the next pass.
+ *            Same least fixed point (DESIGN.md §5.6 and reading R8); rounds = passes.        */
 typedef enum { GDROID_V_DEFAULT = 0, GDROID_V_MAT = 1, GDROID_V_MAT_GRP = 2, GDROID_V_GDROID = 3,
-               GDROID_V_PLAIN = 4, GDROID_V_CELL = 5 } gdroid_variant;
+               GDROID_V_PLAIN = 4, GDROID_V_CELL = 5, GDROID_V_SBDA = 6 } gdroid_variant;
 
 /* Device-counted statistics of the last build (DESIGN.md §5 byte models). */
 typedef struct {

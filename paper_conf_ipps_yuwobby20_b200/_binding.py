@@ -49,7 +49,7 @@ class BuildStats(C.Structure):
         return d
 
 
-VARIANTS = {"default": 0, "mat": 1, "mat_grp": 2, "gdroid": 3, "plain": 4, "cell": 5}   # gdroid_variant
+VARIANTS = {"default": 0, "mat": 1, "mat_grp": 2, "gdroid": 3, "plain": 4, "cell": 5, "sbda": 6}   # gdroid_variant
 
 
 def variant_id(v) -> int:

@@ -199,6 +199,12 @@ struct Dev {
   uint32_t n_seed_nodes, n_seed_pairs;
   uint32_t push_entries;        // 1: k_seed queues the component entries (fresh builds)
   uint32_t round0;              // first round of this build / launch (1 for a fresh build)
+  // SBDA schedule (variant GDROID_V_SBDA), set up at its first build:
+  const uint32_t* meth_node_ptr;  // [n_meths+1] CSR of each method's nodes
+  const uint32_t* meth_nodes;
+  uint32_t* claim;              // [n_meths] last pass a CTA claimed the method
+  unsigned long long* lstamp;   // [N] last local round a node was queued in (pass << 32 | counter)
+  uint32_t n_meths;
   uint32_t hyb;                 // 1: hybrid launch sequence: start at round bar[3], return if it is 0
   uint32_t sw_lo, sw_hi;        // hybrid: leave at the start of a round with < sw_lo / >= sw_hi items
                                 // (bar[3] = that round), 0 = off
@@ -267,6 +273,9 @@ cudaError_t launch_rebase(const Dev& D, NodeRec* nodes, uint32_t* nodemeth, uint
 cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,
                          const uint8_t* ekind, const uint32_t* exoff, cudaStream_t s);
 cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s);
+cudaError_t launch_sbda(const Dev& D, uint32_t blocks, cudaStream_t s);
+cudaError_t launch_meth_csr(const Dev& D, uint32_t* ptr, uint32_t* nodes, uint32_t* cursor, cudaStream_t s);
+int sbda_max_blocks(int device, uint32_t wide);
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_digest(const Dev& D, cudaStream_t s);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s,

@@ -83,7 +83,14 @@ struct CtaStage {              // per-CTA staged worklist appends of the current
   uint32_t nodes;
   uint32_t gbase[NCLS];
   uint32_t buf[NCLS][SCAP];
+  // SBDA schedule (k_sbda): the CTA's method-local worklists in shared memory
+  uint32_t* lq;                // [2][LQCAP] entries (node << 5 | chunk), LQ_SKIP = empty slot
+  uint32_t lcnt[2];
+  uint32_t lsel;               // local queue being processed
+  unsigned long long lid;      // local round id (pass << 32 | counter): dedupe key in D.lstamp
 };
+constexpr uint32_t LQCAP = 1024;
+constexpr uint32_t LQ_SKIP = 0xffffffffu;
 
 // fire-and-forget 64-bit OR at L2 (RED; no return value, no scoreboard wait)
 __device__ __forceinline__ void red_or(uint64_t* p, uint64_t v) {
@@ -128,6 +135,7 @@ __device__ __forceinline__ void stage_init(CtaStage& st) {
 // does not queue it: the warp reads IN(dst) after its own ORs, and a later grower of dst sees a
 // stamp below round+1 and queues dst as usual, so no growth is lost.  cont[dst] == round keeps
 // a second warp from continuing into the same node in the same round (it queues it instead).
+template <bool SB = false>
 __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
                                              uint32_t dst, uint32_t info, bool grew, uint32_t round,
                                              uint32_t nxt, uint32_t* cont = nullptr, bool cont_dense = false,
@@ -137,6 +145,28 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
   // grew, or first reach (A5).  pre_stamp: stamp[dst] loaded early by the caller (a stale value
   // is safe: stamps only grow, and the atomicMax below decides the push)
   if (active) want = grew || ((pre_stamp != NO_CONT ? pre_stamp : D.stamp[dst]) == 0);
+  if constexpr (SB) {
+    // SBDA: an INTRA / C2R successor belongs to the method this CTA is solving,
+    // so it joins the CTA's next local round (deduplicated per local round through D.lstamp);
+    // CALL / RET successors go to the next pass through the global worklist below.
+    const uint32_t ek = info & 3u;
+    if (want && (ek == GE_INTRA || ek == GE_C2R)) {
+      atomicMax(&D.stamp[dst], round);                     // reached (first-reach history)
+      const unsigned long long lid = st.lid;
+      if (atomicMax((unsigned long long*)&D.lstamp[dst], lid) < lid) {
+        const uint32_t nch = ((info >> 5) & 31u) + 1, nl = st.lsel ^ 1u;
+        const uint32_t base = atomicAdd(&st.lcnt[nl], nch);
+        if (base + nch <= LQCAP) {
+          for (uint32_t q = 0; q < nch; ++q) st.lq[nl * LQCAP + base + q] = (dst << 5) | q;
+          want = false;
+        } else {                                            // local queue full: next pass
+          for (uint32_t q = base; q < LQCAP; ++q) st.lq[nl * LQCAP + q] = LQ_SKIP;
+        }
+      } else {
+        want = false;                                      // already in the next local round
+      }
+    }
+  }
   if (cont && *cont == NO_CONT && (D.flags & F_CONT)) {
     const unsigned cand = __ballot_sync(FULL, want && (cont_dense || (info & INFO_WIDE)) && ((info >> 5) & 31u) == 0);
     if (cand) {
@@ -310,7 +340,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
 // the same least fixed point (C4) with work proportional to the new facts.  Δ bits are
 // consumed with RED.AND of exactly the bits read; bits arriving later stay for the next visit
 // (their writer also queued the node).
-template <bool CNT, int MW>
+template <bool CNT, int MW, bool SB = false>
 __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0, uint32_t e1,
                              bool first, uint32_t round, uint32_t nxt, int lane, WarpScratchT<true>& ws, Acc& acc,
                              uint32_t alg_l0, uint32_t* cont, bool cont_dense) {
@@ -524,7 +554,7 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
     const uint32_t gm = eb - e0 < 1024u ? ws.gbits[(eb - e0) >> 5] : ~0u;   // beyond: push (safe)
     const uint32_t my_info = lane < (int)ne ? D.edges[eb + lane].info : 0u;
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gm >> lane) & 1u, round, nxt, cont, cont_dense);
+    flush_pushes<SB>(D, st, lane, lane < (int)ne, my_dst, my_info, (gm >> lane) & 1u, round, nxt, cont, cont_dense);
   }
   if constexpr (CNT) {                     // byte models (dead code, removed, when !CNT)
     // touched words of the semi-naive visit: Δ(src) words read and cleared, T_e(OUT_Δ) words
@@ -563,7 +593,7 @@ __device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r)
 // path, with every read that the chain allows issued in the first memory hop: IN(src), the
 // destinations' round stamps and (FLOAD/FSTORE) the field-row table; the rows the transfer
 // function reads are taken from the IN(src) registers by shuffles instead of reloads.
-template <bool CNT, bool CD>
+template <bool CNT, bool CD, bool SB = false>
 __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
                                                    uint32_t round, uint32_t nxt, int lane, Acc& acc,
                                                    bool cont_ok) {
@@ -667,7 +697,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     if (__any_sync(FULL, g)) gmask |= 1u << i;
   }
   uint32_t cont_v = NO_CONT;                               // GD_CONT_DENSE: depth-first successor
-  flush_pushes(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt,
+  flush_pushes<SB>(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt,
                (CD && cont_ok) ? &cont_v : nullptr, true, my_stamp);
   if constexpr (CNT) {
     const uint32_t alg_l0 = (uint32_t)sizeof(NodeRec) + (uint32_t)sizeof(InlEdge) * ne + 4u;
@@ -679,7 +709,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
 }
 
 // ---------------------------------------------------------------------------------- one item
-template <bool WIDE, bool CNT, int MW, bool CD>
+template <bool WIDE, bool CNT, int MW, bool CD, bool SB = false>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
@@ -699,13 +729,13 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   if constexpr (WIDE) {
     if (R.logW >= 1) {                                      // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
-      process_wide<CNT, MW>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
+      process_wide<CNT, MW, SB>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
                    allow_cont ? &cont_v : nullptr, CD && light);
       return cont_v;
     }
   }
   if (GD_INL && !WIDE && !GD_SMASK && first && R.n_inl) {   // (wide batches: measured slower)
-    return process_inline<CNT, CD>(D, st, R, me, round, nxt, lane, acc, allow_cont && light);
+    return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light);
   }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
@@ -946,7 +976,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     }
     const unsigned gall = __reduce_or_sync(FULL, gmask);
     const uint32_t my_dst = lane < (int)ne ? D.edges[eb + lane].dst : 0u;
-    flush_pushes(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt,
+    flush_pushes<SB>(D, st, lane, lane < (int)ne, my_dst, my_info, (gall >> lane) & 1u, round, nxt,
                  (CD && allow_cont && light) ? &cont_v : nullptr, true);
   }
   if constexpr (CNT) {
@@ -1145,6 +1175,160 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_round(Dev D, uint32_t roun
     D.stats->limit_hit = 1;
   if (total) stage_publish(D, st, (round + 1) % 3);
   flush_acc(D, acc);
+}
+
+// ---------------------------------------------------------------------------------- SBDA
+// The paper's two-level decomposition (§III-A2, Fig. 3; Alg. 2 l.6 "mid <-
+// blockIdx.x"): one CTA per method, its threads running the method's worklist.  On B200 a
+// pass claims every method with queued nodes (the global worklist, one entry per node) for one
+// CTA; the CTA solves that method to local quiescence in shared-memory worklists with
+// __syncthreads between local rounds (no grid barrier), INTRA/C2R successors staying local;
+// CALL/RET successors — the interprocedural hops a method summary would stand for — go to the
+// global worklist of the next pass.  Passes end at an empty worklist.  Same least fixed point
+// (any fair chaotic iteration, DESIGN.md §3 C4 / reading R8); visits = local items processed.
+template <bool WIDE, bool CNT, int MW>
+__global__ void __launch_bounds__(THREADS, GD_MINB) k_sbda(Dev D) {
+  __shared__ WarpScratchT<WIDE> ws_all[WARPS];
+  __shared__ Acc acc_all[WARPS];
+  __shared__ CtaStage st;
+  __shared__ uint32_t lq[2 * LQCAP];
+  __shared__ uint32_t s_m, s_go;
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  Acc& acc = acc_all[wib];
+  if (lane == 0) acc = Acc{0, 0, 0, 0};
+  stage_init(st);
+  if (threadIdx.x == 0) st.lq = lq;
+  __syncthreads();
+  uint32_t counter = 0;
+  for (uint32_t pass = D.round0;; ++pass) {
+    const uint32_t cur = pass % 3, nxt = (pass + 1) % 3, clr = (pass + 2) % 3;
+    if (D.bar[2]) break;
+    uint32_t cnt[NCLS], total = 0;
+#pragma unroll
+    for (int c = 0; c < NCLS; ++c) { cnt[c] = D.counts[cur * CNT_STRIDE + c]; total += cnt[c]; }
+    if (total == 0) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) D.bar[2] = 1;
+      break;
+    }
+    if (D.max_rounds && pass > D.max_rounds) {
+      if (blockIdx.x == 0 && threadIdx.x == 0) D.stats->limit_hit = 1;
+      break;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+#pragma unroll
+      for (int c = 0; c < CNT_STRIDE; ++c) D.counts[clr * CNT_STRIDE + c] = 0;
+      D.bar[4 + nxt] = 0;                                   // claim cursor of the next pass
+      atomicAdd(&D.stats->rounds, 1ull);
+      const uint32_t nodes = D.counts[cur * CNT_STRIDE + CNT_NODES];
+      atomicAdd(&D.stats->hist[nodes <= 32 ? 0 : (nodes <= 64 ? 1 : 2)], 1ull);
+    }
+    const uint32_t* Q = D.queue + (size_t)cur * D.n_chunks;
+    const uint32_t b1 = cnt[0], b2 = b1 + cnt[1], b3 = b2 + cnt[2], b4 = b3 + cnt[3];
+    for (;;) {
+      if (threadIdx.x == 0) {                               // claim the next queued node's method
+        const uint32_t i = atomicAdd(&D.bar[4 + cur], 1u);
+        s_go = i < total;
+        s_m = 0xffffffffu;
+        if (i < total) {
+          const uint32_t c = (i >= b1) + (i >= b2) + (i >= b3) + (i >= b4);
+          const uint32_t base = c == 0 ? 0u : (c == 1 ? b1 : (c == 2 ? b2 : (c == 3 ? b3 : b4)));
+          const uint32_t n = Q[D.seg[c] + (i - base)] >> 5;
+          const uint32_t m = D.node_method[n];
+          if (atomicExch(&D.claim[m], pass) != pass) s_m = m;
+        }
+        st.lsel = 0;
+        st.lcnt[0] = st.lcnt[1] = 0;
+        st.lid = ((unsigned long long)pass << 32) | ++counter;
+      }
+      __syncthreads();
+      if (!s_go) break;
+      const uint32_t m = s_m;
+      if (m != 0xffffffffu) {
+        // local worklist 0: the method's nodes queued for this pass (all their chunks)
+        const uint32_t p0 = D.meth_node_ptr[m], p1 = D.meth_node_ptr[m + 1];
+        for (uint32_t t = p0 + threadIdx.x; t < p1; t += THREADS) {
+          const uint32_t n = D.meth_nodes[t];
+          if (D.stamp[n] != pass) continue;
+          const NodeRec R = D.nodes[n];
+          const uint32_t nch = n_chunks_of(R.e1 - R.e0, R.cls, R.logW);
+          const uint32_t base = atomicAdd(&st.lcnt[0], nch);
+          if (base + nch <= LQCAP) {
+            for (uint32_t q = 0; q < nch; ++q) lq[base + q] = (n << 5) | q;
+          } else {                                          // local queue full: the next pass
+            for (uint32_t q = base; q < LQCAP; ++q) lq[q] = LQ_SKIP;
+            if (atomicMax(&D.stamp[n], pass + 1) < pass + 1) {
+              const uint32_t cls = (D.flags & F_GRP) ? R.cls : 0u;
+              const uint32_t g = atomicAdd(&D.counts[nxt * CNT_STRIDE + cls], nch);
+              for (uint32_t q = 0; q < nch; ++q) D.queue[(size_t)nxt * D.n_chunks + D.seg[cls] + g + q] = (n << 5) | q;
+              atomicAdd(&D.counts[nxt * CNT_STRIDE + CNT_NODES], 1u);
+            }
+          }
+        }
+        __syncthreads();
+        for (;;) {                                          // local rounds (Alg. 2 l.7-18 in one block)
+          const uint32_t sel = st.lsel;
+          const uint32_t ni = min(st.lcnt[sel], LQCAP);
+          if (ni == 0) break;
+          for (uint32_t it = wib; it < ni; it += WARPS) {
+            const uint32_t e = lq[sel * LQCAP + it];
+            if (e == LQ_SKIP) continue;
+            process_item<WIDE, CNT, MW, false, true>(D, st, e >> 5, e & 31u, pass, nxt, lane, ws_all[wib], acc, false);
+            if (lane == 0) acc.cont += 1;                   // a visit (stats->visits)
+          }
+          __syncthreads();
+          if (threadIdx.x == 0) {
+            st.lcnt[sel] = 0;
+            st.lsel = sel ^ 1u;
+            st.lid = ((unsigned long long)pass << 32) | ++counter;
+          }
+          __syncthreads();
+        }
+      }
+      __syncthreads();
+    }
+    stage_publish(D, st, nxt);
+    grid_sync(D.bar, gridDim.x);
+  }
+  flush_acc(D, acc);
+}
+
+// method -> nodes CSR for the SBDA schedule (counts, one-block scan, fill)
+__global__ void k_meth_count(Dev D, uint32_t* cnt) {
+  for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < D.n_nodes; n += gridDim.x * blockDim.x)
+    atomicAdd(&cnt[D.node_method[n] + 1], 1u);
+}
+__global__ void k_meth_scan(uint32_t* ptr, uint32_t M) {   // inclusive scan of ptr[1..M], one block
+  __shared__ uint32_t carry;
+  if (threadIdx.x == 0) carry = 0;
+  __syncthreads();
+  for (uint32_t b = 0; b < M; b += blockDim.x) {
+    const uint32_t i = b + threadIdx.x + 1;
+    uint32_t v = i <= M ? ptr[i] : 0u;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) { const uint32_t t = __shfl_up_sync(FULL, v, o); if (lane >= o) v += t; }
+    __shared__ uint32_t ws[32];
+    if (lane == 31) ws[w] = v;
+    __syncthreads();
+    if (w == 0) {
+      uint32_t x = lane < (int)(blockDim.x >> 5) ? ws[lane] : 0u;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) { const uint32_t t = __shfl_up_sync(FULL, x, o); if (lane >= o) x += t; }
+      ws[lane] = x;
+    }
+    __syncthreads();
+    v += (w ? ws[w - 1] : 0u) + carry;
+    if (i <= M) ptr[i] = v;
+    __syncthreads();
+    if (threadIdx.x == blockDim.x - 1) carry = v;
+    __syncthreads();
+  }
+}
+__global__ void k_meth_fill(Dev D, const uint32_t* ptr, uint32_t* cursor, uint32_t* nodes) {
+  for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < D.n_nodes; n += gridDim.x * blockDim.x) {
+    const uint32_t m = D.node_method[n];
+    nodes[ptr[m] + atomicAdd(&cursor[m], 1u)] = n;
+  }
 }
 
 // (a1) Rebase the staged app-local node tables by their app's bases (NodeRec::app).
@@ -1409,6 +1593,41 @@ cudaError_t launch_fixpoint(const Dev& D, uint32_t blocks, cudaStream_t s) {
   void* args[] = {&d};
   const void* f = D.count ? fixpoint_fn<true>(D.wide, D.hiocc) : fixpoint_fn<false>(D.wide, D.hiocc);
   return cudaLaunchCooperativeKernel(f, dim3(blocks), dim3(THREADS), args, 0, s);
+}
+
+template <bool CNT>
+static const void* sbda_fn(uint32_t wide) {
+  switch (wide) {
+    case 0: return (const void*)k_sbda<false, CNT, 1>;
+    case 1: return (const void*)k_sbda<true, CNT, 2>;
+    case 2: return (const void*)k_sbda<true, CNT, 4>;
+    default: return (const void*)k_sbda<true, CNT, 8>;
+  }
+}
+
+int sbda_max_blocks(int device, uint32_t wide) {
+  int sms = 0, occ = 0, occ2 = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, sbda_fn<true>(wide), THREADS, 0);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, sbda_fn<false>(wide), THREADS, 0);
+  occ = occ2 < occ ? occ2 : occ;
+  return sms * (occ > 0 ? occ : 1);
+}
+
+cudaError_t launch_sbda(const Dev& D, uint32_t blocks, cudaStream_t s) {
+  Dev d = D;
+  void* args[] = {&d};
+  return cudaLaunchCooperativeKernel(D.count ? sbda_fn<true>(D.wide) : sbda_fn<false>(D.wide), dim3(blocks),
+                                     dim3(THREADS), args, 0, s);
+}
+
+cudaError_t launch_meth_csr(const Dev& D, uint32_t* ptr, uint32_t* nodes, uint32_t* cursor, cudaStream_t s) {
+  cudaMemsetAsync(ptr, 0, (size_t)(D.n_meths + 1) * 4, s);
+  cudaMemsetAsync(cursor, 0, (size_t)D.n_meths * 4, s);
+  k_meth_count<<<1184, 256, 0, s>>>(D, ptr);
+  k_meth_scan<<<1, 1024, 0, s>>>(ptr, D.n_meths);
+  k_meth_fill<<<1184, 256, 0, s>>>(D, ptr, cursor, nodes);
+  return cudaGetLastError();
 }
 
 template <bool CNT>

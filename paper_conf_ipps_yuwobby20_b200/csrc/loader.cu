@@ -808,7 +808,7 @@ struct Layout {
   size_t total = 0;              // device bytes of the tables
   size_t upload = 0;             // staged (host-built) prefix of them
   std::vector<uint32_t> app_base;
-  uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0;
+  uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0, n_meths = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
   uint32_t wide = 0;            // max logW over the modules
 };
@@ -921,7 +921,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   uint64_t nc = 0;
   for (int c = 0; c < NCLS; ++c) nc += Lo.cls_count[c];
   if (nc >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
-  Lo.N = T.node; Lo.NC = nc; Lo.n_entries = T.ent; Lo.fact_words = T.fact;
+  Lo.N = T.node; Lo.NC = nc; Lo.n_entries = T.ent; Lo.fact_words = T.fact; Lo.n_meths = T.meth;
   Lo.app_base.resize(n_apps + 1);
   for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
   const size_t bytes[NPART] = {
@@ -1096,6 +1096,9 @@ struct gdroid_app {
   void* h_seed = nullptr;             // pinned staging of the seeds
   void* d_seed = nullptr;
   size_t seed_cap = 0;
+  // SBDA schedule state (allocated at the first SBDA build)
+  void* d_sbda = nullptr;
+  int sbda_blocks = 0;
   uint64_t counts_build = ~0ull;      // build_serial whose per-node counts are in d_scratch
   bool release_pending = false;
   int max_blocks = 0;
@@ -1122,6 +1125,7 @@ void free_app(gdroid_app* a) {
   if (a->D.trace) cudaFree(a->D.trace);
   if (a->pending || a->h_seed) cudaStreamSynchronize(a->stream);   // copies target host slots
   if (a->d_seed) cudaFreeAsync(a->d_seed, a->stream);
+  if (a->d_sbda) cudaFreeAsync(a->d_sbda, a->stream);
   if (a->h_seed) cudaFreeHost(a->h_seed);
   stats_slots().put(a->h_stats);
   for (auto& e : a->ev)
@@ -1487,6 +1491,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.seg[NCLS] = acc;
   D.n_words = Lo.fact_words;
   D.wide = Lo.wide;
+  D.n_meths = (uint32_t)Lo.n_meths;
   {
     // (a1) per-app bases added to the staged app-local node tables, then the edge records and
     // inline chunk-0 edges derived from col / edge_kind / projection offsets and the NodeRecs
@@ -1553,10 +1558,27 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   Dev& D = a->D;
   D.max_rounds = o.max_rounds;
   if (o.variant == GDROID_V_PLAIN || o.variant == GDROID_V_CELL) return build_plain(a, o, stats);
-  if (o.variant > GDROID_V_GDROID) return set_err(GDROID_E_INVALID, "unknown variant %u", o.variant);
+  if (o.variant > GDROID_V_SBDA || o.variant == GDROID_V_CELL)
+    return set_err(GDROID_E_INVALID, "unknown variant %u", o.variant);
   a->last_plain = false;
+  const bool sbda = o.variant == GDROID_V_SBDA;
   static const uint32_t vflags[4] = {F_GRP | F_CONT, 0u, F_GRP, F_GRP | F_MER};
-  D.flags = vflags[o.variant];
+  D.flags = sbda ? F_GRP : vflags[o.variant];
+  if (sbda && !a->d_sbda) {                          // method -> nodes CSR, claims, local stamps
+    const size_t M = D.n_meths, N = D.n_nodes;
+    const size_t bytes = align256((M + 1) * 4) + align256(N * 4) + align256(M * 4) * 2 + align256(N * 8);
+    CU(cudaMallocAsync(&a->d_sbda, bytes, a->stream));
+    char* S = (char*)a->d_sbda;
+    uint32_t* ptr = (uint32_t*)S; S += align256((M + 1) * 4);
+    uint32_t* nodes = (uint32_t*)S; S += align256(N * 4);
+    uint32_t* cursor = (uint32_t*)S; S += align256(M * 4);
+    D.claim = (uint32_t*)S; S += align256(M * 4);
+    D.lstamp = (unsigned long long*)S;
+    D.meth_node_ptr = ptr;
+    D.meth_nodes = nodes;
+    CU(launch_meth_csr(D, ptr, nodes, cursor, a->stream));
+    a->sbda_blocks = sbda_max_blocks(a->device, D.wide);
+  }
   D.count = o.no_byte_model ? 0u : 1u;
   {                                                   // GRP off: one segment holds every item
     uint32_t acc = 0;
@@ -1612,7 +1634,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   D.n_seed_nodes = D.n_seed_pairs = 0;
   CU(cudaEventRecord(a->ev[1], s));
   D.sw_lo = D.sw_hi = 0;
-  if (o.loop_mode == 0 && D.hiocc && GD_HYBRID && (D.flags & F_CONT)) {
+  if (!sbda && o.loop_mode == 0 && D.hiocc && GD_HYBRID && (D.flags & F_CONT)) {
     // Hybrid (large narrow batches, default variant): light rounds run in the 3-CTA/SM
     // instantiation with narrow continuation, heavy rounds (>= 4 waves of items) in the 4-CTA/SM
     // one; a launch leaves at the first round of the other kind (bar[3] = that round) and the
@@ -1637,6 +1659,12 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
     }
     D.hyb = 0u;
     D.sw_lo = D.sw_hi = 0;
+  } else if (sbda) {
+    CU(cudaMemsetAsync(D.claim, 0, (size_t)D.n_meths * 4, s));
+    CU(cudaMemsetAsync(D.lstamp, 0, (size_t)N * 8, s));
+    const uint32_t bs = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->sbda_blocks) : (uint32_t)a->sbda_blocks;
+    CU(launch_sbda(D, bs, s));
+    a->launches++;
   } else if (o.loop_mode == 0) {
     CU(launch_fixpoint(D, blocks, s));
     a->launches++;

@@ -66,7 +66,8 @@ def _check(app, k, g, ref):
 
 @pytest.mark.parametrize("name,variant", [("small", "default"), ("median", "default"), ("worst", "default"),
                                           ("small", "mat"), ("median", "mat_grp"), ("median", "gdroid"),
-                                          ("small", "plain"), ("small", "cell")])
+                                          ("small", "plain"), ("small", "cell"), ("small", "sbda"),
+                                          ("median", "sbda"), ("worst", "sbda")])
 def test_preset_full_size(name, variant):
     fx = _fixture()
     if name not in fx:

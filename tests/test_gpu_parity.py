@@ -279,3 +279,22 @@ def test_cell_major_variant_random(chunk):
         assert dig == r.app_digest and np.array_equal(per, r.node_digest)
         assert st["fact_bytes"] > 0
         app.free()
+
+
+@pytest.mark.parametrize("blocks", [0, 2])
+def test_sbda_schedule(blocks):
+    """SBDA (SURVEY §8(f)3 as a schedule, DESIGN.md §5.6 / reading R8): one CTA per method per
+    pass with shared-memory local worklists; narrow + wide random tiny ICFGs (arity up to 5,
+    recursion, projection) and the goldens in one batch, pair for pair against the oracle."""
+    gs = [random_tiny(s, max_stmts=7, wide_pad=(90 if s % 3 == 0 else 0)) for s in range(14000, 14120)]
+    gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0]]
+    app = gd.load(gs)
+    st = app.build(variant="sbda", blocks=blocks)
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        _assert_same(app, k, g, r, f"sbda/{g.name}")
+        assert int(digs[k]) == r.app_digest
+    assert st["rounds"] > 0 and st["node_visits"] > 0
+    app.build(variant="sbda", byte_model=False)        # rebuild: claims / local stamps reset
+    assert np.array_equal(app.app_digests(), digs)
