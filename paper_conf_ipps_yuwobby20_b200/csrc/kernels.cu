@@ -700,7 +700,9 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
   flush_pushes<SB>(D, st, lane, lane < (int)ne, me.dst, me.info, (gmask >> lane) & 1u, round, nxt,
                (CD && cont_ok) ? &cont_v : nullptr, true, my_stamp);
   if constexpr (CNT) {
-    const uint32_t alg_l0 = (uint32_t)sizeof(NodeRec) + (uint32_t)sizeof(InlEdge) * ne + 4u;
+    // SURVEY §8(d) per-visit constants: 16 B statement record + 8 B row_ptr pair + 5 B per edge
+    // (col + kind) + 8 B queue in/out (not this implementation's 64 B NodeRec / 16 B inline edges)
+    const uint32_t alg_l0 = 16u + 8u + 5u * ne + 8u;
     acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (lane == 0 ? alg_l0 : 0u));
     acc_add(acc.atom, red);
     if (lane == 0) acc.dense += 8ull * B + 16ull * B * ne + alg_l0;
@@ -721,7 +723,9 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
   const bool first = ci == 0;
   const uint32_t L = R.L, B = R.B;
-  uint32_t alg_l0 = (first ? (uint32_t)sizeof(NodeRec) : 0u) + (uint32_t)sizeof(Edge) * (e1 - e0) + 4u;
+  // SURVEY §8(d) constants: statement record + row_ptr once per node visit (chunk 0), 5 B per
+  // edge, 8 B queue entry in/out per item
+  uint32_t alg_l0 = (first ? 16u + 8u : 0u) + 5u * (e1 - e0) + 8u;
   if (e0 >= e1) {                                           // no successor: nothing to propagate
     if (CNT && lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
     return NO_CONT;
@@ -1450,39 +1454,78 @@ __global__ void k_apply_seeds(Dev D) {
 // (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp's nodes are
 // nw apart, so consecutive ones almost always belong to the same app: the app sum is carried in
 // a register and added once per app change (not one same-address atomic per node).
+// Digest of one node's block held as y[k] = word lane + 32k (k < DKW), plus any words beyond.
+constexpr int DKW = 4;
+__device__ __forceinline__ unsigned long long digest_words(const Dev& D, const NodeRec& R, uint64_t hn,
+                                                           const uint64_t (&y)[DKW], int lane) {
+  const uint32_t logW = R.logW, L = R.L, B = R.B, jm = (1u << logW) - 1;
+  unsigned long long s = 0;
+  auto one = [&](uint32_t w, uint64_t x) {
+    const uint32_t r = w >> logW, j = w & jm;
+    const uint64_t slot = r < L ? (uint64_t)(R.local_base + r) : (uint64_t)D.grow_gid[R.grow_off + r - L];
+    while (x) {
+      const int b = __ffsll((long long)x) - 1;
+      x &= x - 1;
+      const uint64_t o = D.col_gid[R.col_off + j * 64 + b];
+      s += mix64(hn ^ ((slot << 32) | o));
+    }
+  };
+#pragma unroll
+  for (int k = 0; k < DKW; ++k)
+    if (y[k]) one(lane + 32 * k, y[k]);
+  const uint64_t* X = D.facts + R.off;
+  for (uint32_t w = lane + 32 * DKW; w < B; w += 32) {     // blocks beyond 128 words (wide)
+    const uint64_t x = X[w];
+    if (x) one(w, x);
+  }
+  return s;
+}
+
+// (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp takes two
+// nodes at a time: both NodeRecs, then the first 128 words of both blocks, are loaded before any
+// bit is hashed (memory-level parallelism; the store is read once, coalesced).  A warp's nodes
+// are nw apart, so consecutive ones almost always belong to the same app: the app sum is
+// carried in a register and added once per app change.
 __global__ void __launch_bounds__(256) k_digest(Dev D) {
   const int lane = threadIdx.x & 31;
   const uint32_t nw = gridDim.x * (blockDim.x >> 5);
   unsigned long long app_sum = 0;
   uint32_t app_cur = 0xffffffffu;
-  for (uint32_t n = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < D.n_nodes; n += nw) {
+  const uint32_t g0 = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+  for (uint32_t n = g0; n < D.n_nodes; n += 2 * nw) {
+    const uint32_t n2 = n + nw;
+    const bool has2 = n2 < D.n_nodes;
     const NodeRec R = D.nodes[n];
-    const uint32_t local_base = R.local_base;
-    const uint32_t logW = R.logW, L = R.L, B = R.B;
-    const uint64_t* X = D.facts + R.off;
+    NodeRec R2 = R;
+    if (has2) R2 = D.nodes[n2];
     const uint64_t hn = mix64((uint64_t)(n - D.app_node_base[R.app]));
-    unsigned long long s = 0;
-    for (uint32_t w = lane; w < B; w += 32) {
-      uint64_t x = X[w];
-      if (!x) continue;
-      const uint32_t r = w >> logW, j = w & ((1u << logW) - 1);
-      const uint64_t slot = r < L ? (uint64_t)(local_base + r) : (uint64_t)D.grow_gid[R.grow_off + r - L];
-      while (x) {
-        const int b = __ffsll((long long)x) - 1;
-        x &= x - 1;
-        const uint64_t o = D.col_gid[R.col_off + j * 64 + b];
-        s += mix64(hn ^ ((slot << 32) | o));
-      }
+    const uint64_t hn2 = has2 ? mix64((uint64_t)(n2 - D.app_node_base[R2.app])) : 0ull;
+    uint64_t y[DKW], y2[DKW];
+#pragma unroll
+    for (int k = 0; k < DKW; ++k) {
+      const uint32_t w = lane + 32 * k;
+      y[k] = w < R.B ? D.facts[R.off + w] : 0ull;
+      y2[k] = (has2 && w < R2.B) ? D.facts[R2.off + w] : 0ull;
     }
-    s = warp_sum64(s);
+    const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane));
+    const unsigned long long s2 = has2 ? warp_sum64(digest_words(D, R2, hn2, y2, lane)) : 0ull;
     if (lane == 0) {
       D.node_digest[n] = s;
+      if (has2) D.node_digest[n2] = s2;
       if (R.app != app_cur) {
         if (app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
         app_cur = R.app;
         app_sum = 0;
       }
       app_sum += s;
+      if (has2) {
+        if (R2.app != app_cur) {
+          if (app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
+          app_cur = R2.app;
+          app_sum = 0;
+        }
+        app_sum += s2;
+      }
     }
   }
   if (lane == 0 && app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
