@@ -296,10 +296,19 @@ def run_ours(args):
     nthreads = max(1, host_threads() // max(1, per_host))
     os.environ.setdefault("GDROID_HOST_THREADS", str(nthreads))
     assert torch.cuda.is_available(), "bench needs a GPU"
+    # GDROID_BENCH_SHARE_GPU=1 (test hook): every rank on cuda:0 with gloo collectives, to run the
+    # multi-rank path on a one-GPU box; the driver's runs use one GPU per rank and NCCL
+    share = os.environ.get("GDROID_BENCH_SHARE_GPU") == "1"
+    if share:
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
+    cdev = None if share else dev                         # where collective tensors live
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -342,8 +351,8 @@ def run_ours(args):
     rec = corpus.pack_record(apps=len(my_ids), visits=visits, alg_bytes=alg, build_ns=int(my_ms * 1e6),
                              wall_ns=int(my_ms * 1e6), max_app_ns=int(max(batch_ms) * 1e6),
                              digest_sum=sum(res.digests.values()), errors=0)
-    recs = corpus.unpack_records(corpus.gather_records(rec, dev if world > 1 else None))
-    dig_all, dig_mask = corpus.gather_digests(plan.n_apps, res.digests, dev if world > 1 else None)
+    recs = corpus.unpack_records(corpus.gather_records(rec, cdev if world > 1 else None))
+    dig_all, dig_mask = corpus.gather_digests(plan.n_apps, res.digests, cdev if world > 1 else None)
     shard.free()
 
     # e2e through the public API from host arrays: load (host tables + pinned H2D) of batch i+1
@@ -368,7 +377,7 @@ def run_ours(args):
                 h2d += br.h2d_bytes
         torch.cuda.synchronize()
         e2e_ms = (time.perf_counter() - t0) * 1e3 / args.e2e_steps
-        t = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([e2e_ms], dtype=torch.float64, device=cdev if cdev is not None else "cpu")
         if world > 1:
             g = [torch.zeros_like(t) for _ in range(world)]
             dist.all_gather(g, t)
@@ -451,7 +460,7 @@ def run_ours(args):
                                           "(tests/golden/oracle_digests.json records the oracle's time)"}
     elif not args.no_cpu_baseline:
         wall, osec, ovis, odig = oracle_pool(sample_apps, P)
-        ok = sum(1 for i, d in zip(ids, odig) if i in res.digests and d == res.digests[i])
+        ok = sum(1 for i, d in zip(ids, odig) if d == int(dig_all[i]))   # vs the gathered GPU digests
         line["cpu_baseline"] = {
             "value": len(sample_apps) / wall, "unit": "apps/s", "cores": P, "kind": "oracle",
             "cpu_model": cpu_model(),

@@ -49,6 +49,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_BAR_NS
 #define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
 #endif
+#ifndef GD_CONT_WIDE
+#define GD_CONT_WIDE 1         // wide items continue depth-first into wide successors
+#endif
 #ifndef GD_CONT_DENSE
 #define GD_CONT_DENSE 1        // continue into narrow (one word per row) destinations too (light rounds)
 #endif
@@ -352,6 +355,8 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
   const uint64_t* OCC = X + occ_offset(B);
   const uint32_t nocc = occ_words(rows);
   const uint32_t kind = R.kind;
+  if (lane < (int)min(e1 - e0, 32u))                       // edge records into L1 (read in pass 2)
+    asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.edges + e0 + lane)));
   // ---- transfer setup on IN(src): generated row t (mode 1 replace / 2 or-in) or FSTORE rows
   //      (mode 3).  The full GEN is emitted on every visit (a superset of its new part).
   int mode = 0, t = -1;
@@ -459,8 +464,9 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
   };
   // ---- pass 1: keep the candidate rows whose OUT_Δ is non-empty (compacted in place; a row
   //      that gains Δ bits after this scan keeps them for the node's next visit)
-  uint32_t kept = 0;
-  for (uint32_t p0 = 0; p0 < cnt; p0 += 32) {
+  //      (at most 32 candidates: no compaction, pass 2 reads every candidate once)
+  uint32_t kept = cnt <= 32 ? cnt : 0u;
+  for (uint32_t p0 = 0; cnt > 32 && p0 < cnt; p0 += 32) {
     const uint32_t p = p0 + lane;
     uint64_t y[MW];
     const uint32_t r = p < cnt ? ws.rowlist[p] : 0u;
@@ -734,7 +740,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     if (R.logW >= 1) {                                      // wide block: row-sparse path
       uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
       process_wide<CNT, MW, SB>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
-                   allow_cont ? &cont_v : nullptr, CD && light);
+                   (GD_CONT_WIDE && allow_cont) ? &cont_v : nullptr, CD && light);
       return cont_v;
     }
   }

@@ -139,7 +139,7 @@ def _corpus_check(ids, node_budget=4_000_000):
     plan = corpus.plan_corpus(sizes, wide, 1, node_budget=node_budget, app_ids=ids)
     checked = 0
     for b in plan.batches[0]:
-        apps = {i: G.corpus_app(i) for i in b}
+        apps = corpus.make_apps(b, G.corpus_app, threads=min(16, len(os.sched_getaffinity(0))))
         sh = corpus.DeviceShard([b], apps)
         sh.step()
         sh.finish()
