@@ -13,6 +13,10 @@ constexpr int NCLS = 5;            // GRP classes + 2 interpr
 enum Cls : uint8_t { C_ONETIME = 0, C_SINGLE = 1, C_DOUBLE = 2, C_CALL = 3, C_EXIT = 4 };
 constexpr int CNT_STRIDE = 8;      // counts[rot * CNT_STRIDE + cls]; slot CNT_NODES = nodes queued
 constexpr int CNT_NODES = 5;
+// D.bar words: [0] arrivals and [1] generation of the grid barrier, [3] hybrid hand-over round,
+// [4..6] SBDA claim cursors; the worklist-empty flag that every warp reads after the barrier
+// sits in its own 128-byte line, away from the barrier's atomics and pollers.
+constexpr int BAR_DONE = 32;
 #ifndef GD_HIOCC_NODES
 #define GD_HIOCC_NODES (1u << 17)
 #endif

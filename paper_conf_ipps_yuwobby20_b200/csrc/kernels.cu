@@ -147,7 +147,11 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
   bool want = false;
   // grew, or first reach (A5).  pre_stamp: stamp[dst] loaded early by the caller (a stale value
   // is safe: stamps only grow, and the atomicMax below decides the push)
-  if (active) want = grew || ((pre_stamp != NO_CONT ? pre_stamp : D.stamp[dst]) == 0);
+  uint32_t sv = 0;
+  if (active) {
+    sv = pre_stamp != NO_CONT ? pre_stamp : D.stamp[dst];
+    want = grew || sv == 0;
+  }
   if constexpr (SB) {
     // SBDA: an INTRA / C2R successor belongs to the method this CTA is solving,
     // so it joins the CTA's next local round (deduplicated per local round through D.lstamp);
@@ -184,7 +188,9 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
     }
   }
   if (active) {
-    if (want) {
+    // sv == round + 1: already queued for the next round (stamps never exceed round + 1 during
+    // round `round`, and a stale value is never larger than the true one) — no atomic needed
+    if (want && sv != round + 1) {
       const uint32_t old = atomicMax(&D.stamp[dst], round + 1);  // test-and-set: de-duplicates (MER)
       push = old < round + 1;
     }
@@ -1036,12 +1042,12 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
   uint32_t cnt[NCLS];
   uint32_t total = 0;
-  if (D.bar[2]) return 0;                 // an earlier round found the worklist empty
+  if (D.bar[BAR_DONE]) return 0;          // an earlier round found the worklist empty
 #pragma unroll
   for (int c = 0; c < NCLS; ++c) { cnt[c] = D.counts[cur * CNT_STRIDE + c]; total += cnt[c]; }
   if (total == 0) {
     if (blockIdx.x == 0 && threadIdx.x == 0) {
-      D.bar[2] = 1;
+      D.bar[BAR_DONE] = 1;
       if (round <= D.trace_cap) {
         unsigned long long ns;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ns));
@@ -1212,12 +1218,12 @@ __global__ void __launch_bounds__(THREADS, GD_MINB) k_sbda(Dev D) {
   uint32_t counter = 0;
   for (uint32_t pass = D.round0;; ++pass) {
     const uint32_t cur = pass % 3, nxt = (pass + 1) % 3, clr = (pass + 2) % 3;
-    if (D.bar[2]) break;
+    if (D.bar[BAR_DONE]) break;
     uint32_t cnt[NCLS], total = 0;
 #pragma unroll
     for (int c = 0; c < NCLS; ++c) { cnt[c] = D.counts[cur * CNT_STRIDE + c]; total += cnt[c]; }
     if (total == 0) {
-      if (blockIdx.x == 0 && threadIdx.x == 0) D.bar[2] = 1;
+      if (blockIdx.x == 0 && threadIdx.x == 0) D.bar[BAR_DONE] = 1;
       break;
     }
     if (D.max_rounds && pass > D.max_rounds) {

@@ -1681,10 +1681,10 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
         a->launches++;
       }
       round += K;
-      cudaMemcpyAsync(h_counts, D.bar, 16, cudaMemcpyDeviceToHost, s);
+      cudaMemcpyAsync(h_counts, D.bar + BAR_DONE, 4, cudaMemcpyDeviceToHost, s);
       cudaError_t e = cudaStreamSynchronize(s);
       if (e != cudaSuccess) { cudaFreeHost(h_counts); return set_err(GDROID_E_CUDA, "round loop: %s", cudaGetErrorString(e)); }
-      if (h_counts[2]) break;                                      // a round found an empty worklist
+      if (h_counts[0]) break;                                      // a round found an empty worklist
       if (D.max_rounds && round > D.max_rounds + 1) break;
     }
     cudaFreeHost(h_counts);
