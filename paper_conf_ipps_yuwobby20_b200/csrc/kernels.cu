@@ -49,6 +49,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_BAR_NS
 #define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
 #endif
+#ifndef GD_PAIR
+#define GD_PAIR 1              // heavy rounds: two inline items per warp (half-warp each)
+#endif
 #ifndef GD_CONT_WIDE
 #define GD_CONT_WIDE 1         // wide items continue depth-first into wide successors
 #endif
@@ -578,6 +581,10 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
 }
 
 // ---------------------------------------------------------------------------------- inline items
+__device__ __forceinline__ uint64_t hshfl_xor64(uint64_t v, int o) {   // xor within the half-warp
+  const uint32_t lo = __shfl_xor_sync(FULL, (uint32_t)v, o, 16), hi = __shfl_xor_sync(FULL, (uint32_t)(v >> 32), o, 16);
+  return ((uint64_t)hi << 32) | lo;
+}
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   const uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src), hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src);
   return ((uint64_t)hi << 32) | lo;
@@ -720,6 +727,151 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     if (lane == 0) acc.dense += 8ull * B + 16ull * B * ne + alg_l0;
   }
   return cont_v;
+}
+
+// ---------------------------------------------------------------------------------- paired items
+// Heavy rounds (the 4-CTA/SM instantiation): a warp takes two inline items at once, one per
+// half-warp (16 lanes x 8 words = the 128-word inline limit), so every warp keeps two dependent
+// load -> transfer -> union -> push chains in flight.  Same transfer and union as
+// process_inline, with width-16 shuffles; IN(dst) words are loaded only where OUT is non-zero
+// (no pre-read: two full pre-reads per half would not fit the register budget).
+constexpr int HKW = 8;
+__device__ __forceinline__ uint64_t hshfl64(uint64_t v, int src) {      // within the half-warp
+  const uint32_t lo = __shfl_sync(FULL, (uint32_t)v, src, 16), hi = __shfl_sync(FULL, (uint32_t)(v >> 32), src, 16);
+  return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t half_or64(uint64_t v) {
+#pragma unroll
+  for (int o = 8; o; o >>= 1) v |= hshfl_xor64(v, o);
+  return v;
+}
+__device__ __forceinline__ uint32_t half_or32(uint32_t v) {
+#pragma unroll
+  for (int o = 8; o; o >>= 1) v |= __shfl_xor_sync(FULL, v, o, 16);
+  return v;
+}
+// word r of the half's block held as y[k] = word hl + 16k: r uniform in the half / per lane
+__device__ __forceinline__ uint64_t huword_of(const uint64_t (&y)[HKW], uint32_t r) {
+  uint64_t s = y[0];
+#pragma unroll
+  for (int k = 1; k < HKW; ++k) if ((r >> 4) == (uint32_t)k) s = y[k];
+  return hshfl64(s, (int)(r & 15u));
+}
+__device__ __forceinline__ uint64_t hword_of(const uint64_t (&y)[HKW], uint32_t r) {
+  uint64_t s = 0;
+#pragma unroll
+  for (int k = 0; k < HKW; ++k) {
+    const uint64_t v = hshfl64(y[k], (int)(r & 15u));
+    if ((r >> 4) == (uint32_t)k) s = v;
+  }
+  return s;
+}
+
+template <bool CNT>
+__device__ __forceinline__ void process_inline2(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
+                                                uint32_t round, uint32_t nxt, int lane, Acc& acc) {
+  const int hl = lane & 15;
+  const unsigned hmask = 0xffffu << (lane & 16);
+  const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
+  const uint64_t* X = D.facts + R.off;
+  uint64_t y[HKW];
+#pragma unroll
+  for (int k = 0; k < HKW; ++k) {
+    const uint32_t w = hl + 16 * k;
+    y[k] = w < B ? X[w] : 0ull;
+  }
+  const uint32_t my_stamp = hl < (int)ne ? D.stamp[me.dst] : 1u;
+  const bool dbl = kind == GK_FLOAD || kind == GK_ALOAD || kind == GK_FSTORE || kind == GK_ASTORE;
+  int hr[4] = {-1, -1, -1, -1};                             // heap rows of this lane's columns
+  if (dbl) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t c = hl + 16 * q;
+      hr[q] = (c < R.n_cols) ? D.frow[R.r3 + c] : -1;
+    }
+  }
+  int mode = 0, t = -1;
+  uint64_t genv = 0;
+  uint32_t fmask = 0, hwords = 0;
+  if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
+    mode = 1; t = R.r0;
+    if (kind != GK_PRIM) genv = 1ull << (R.r3 & 63);
+  } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
+    mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
+    genv = huword_of(y, (uint32_t)R.r1);
+  } else if (kind == GK_FLOAD || kind == GK_ALOAD) {
+    mode = 1; t = R.r0;
+    const uint64_t wrow = huword_of(y, (uint32_t)R.r1);
+    uint64_t a = 0;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t c = hl + 16 * q;
+      const bool take = hr[q] >= 0 && ((wrow >> c) & 1ull);
+      const uint64_t v = hword_of(y, take ? L + (uint32_t)hr[q] : 0u);
+      if (take) { a |= v; hwords += 1; }
+    }
+    genv = half_or64(a);
+  } else if (kind == GK_FSTORE || kind == GK_ASTORE) {
+    mode = 3;
+    const uint64_t vrow = huword_of(y, (uint32_t)R.r0);
+    genv = huword_of(y, (uint32_t)R.r1);
+#pragma unroll
+    for (int k = 0; k < HKW; ++k) {
+      uint32_t m = 0;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t c = hl + 16 * q;
+        if (hr[q] >= 0 && ((vrow >> c) & 1ull)) {
+          const uint32_t w = L + (uint32_t)hr[q];
+          if ((w >> 4) == (uint32_t)k) m |= 1u << (w & 15u);
+        }
+      }
+      m = half_or32(m);
+      if ((m >> hl) & 1u) fmask |= 1u << k;
+    }
+  }
+  uint32_t nzx = 0, nz = 0, red = 0;
+#pragma unroll
+  for (int k = 0; k < HKW; ++k) {
+    const uint32_t w = hl + 16 * k;
+    if (CNT) nzx += (y[k] != 0);
+    if (mode == 1) { if ((int)w == t) y[k] = genv; }
+    else if (mode == 2) { if ((int)w == t) y[k] |= genv; }
+    else if (mode == 3) { if ((fmask >> k) & 1u) y[k] |= genv; }
+  }
+  unsigned gmask = 0;
+#pragma unroll
+  for (uint32_t i = 0; i < 4; ++i) {                        // inline edges (<= 4; per-half count)
+    const bool act = i < ne;
+    const uint64_t off = hshfl64(me.off, (int)i);
+    const uint32_t info = __shfl_sync(FULL, me.info, (int)i, 16);
+    const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;
+    uint64_t* Z = D.facts + off;
+    uint64_t cur[HKW];
+#pragma unroll
+    for (int k = 0; k < HKW; ++k) {
+      const uint32_t w = hl + 16 * k;
+      cur[k] = (act && y[k] && (int)w != kill) ? Z[w] : ~0ull;
+    }
+    bool g = false;
+#pragma unroll
+    for (int k = 0; k < HKW; ++k) {
+      const uint32_t w = hl + 16 * k;
+      const uint64_t z = (!act || (int)w == kill) ? 0ull : y[k];
+      nz += (z != 0);
+      if (z & ~cur[k]) { red_or(Z + w, z); ++red; g = true; }
+    }
+    if (__ballot_sync(FULL, g) & hmask) gmask |= 1u << i;
+  }
+  flush_pushes(D, st, lane, hl < (int)ne, me.dst, me.info, (gmask >> hl) & 1u, round, nxt, nullptr, true, my_stamp);
+  if constexpr (CNT) {
+    const uint32_t alg_l0 = 16u + 8u + 5u * ne + 8u;       // SURVEY §8(d) constants, per item
+    acc_add(acc.alg, 16u * nz + 8u * nzx + 8u * hwords + (hl == 0 ? alg_l0 : 0u));
+    acc_add(acc.atom, red);
+    const unsigned long long d = 8ull * B + 16ull * B * ne + alg_l0;
+    const unsigned long long d2 = __shfl_sync(FULL, d, 16);
+    if (lane == 0) acc.dense += d + d2;
+  }
 }
 
 // ---------------------------------------------------------------------------------- one item
@@ -1036,7 +1188,7 @@ __device__ __forceinline__ void flush_acc(const Dev& D, const Acc& acc) {
 
 // Process every item of round `round` with warps gw, gw+nw, ...; returns total items (0 when
 // the worklist is empty: the fixed point of Alg. 1 l.10 is reached).
-template <bool WIDE, bool CNT, int MW, bool CD>
+template <bool WIDE, bool CNT, int MW, bool CD, bool PAIR = false>
 __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32_t round, uint32_t gw,
                                               uint32_t nw, int lane, WarpScratchT<WIDE>& ws, Acc& acc) {
   const uint32_t cur = round % 3, nxt = (round + 1) % 3, clr = (round + 2) % 3;
@@ -1093,6 +1245,30 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   // MER (Fig. 7): process the head list — whole waves of nw items — and
   // merge the tail into the next worklist (the round stamp removes repetitions).
   const uint32_t head = ((D.flags & F_MER) && total > nw) ? (total / nw) * nw : total;
+  if constexpr (PAIR) {
+    // heavy rounds (4-CTA/SM instantiation, no continuation, no MER): two items per warp; a pair
+    // of inline items runs on the two half-warps, any other pair item by item on the full warp
+    if (!(D.flags & F_MER)) {
+      for (uint32_t item = gw; item < total; item += 2 * nw) {
+        const uint32_t item2 = item + nw;
+        const bool has2 = item2 < total;
+        const uint32_t ea = entry_of(item), eb = has2 ? entry_of(item2) : ea;
+        const uint32_t my_e = (lane >= 16 && has2) ? eb : ea;
+        const uint32_t my_n = my_e >> 5;
+        const NodeRec R = D.nodes[my_n];
+        InlEdge me{0u, 0u, 0ull};
+        if ((lane & 15) < 4) me = D.inl[4 * my_n + (lane & 15)];
+        const bool elig = (my_e & 31u) == 0 && R.n_inl != 0;
+        if (has2 && __all_sync(FULL, elig)) {
+          process_inline2<CNT>(D, st, R, me, round, nxt, lane, acc);
+        } else {
+          process_item<WIDE, CNT, MW, CD>(D, st, ea >> 5, ea & 31u, round, nxt, lane, ws, acc, false);
+          if (has2) process_item<WIDE, CNT, MW, CD>(D, st, eb >> 5, eb & 31u, round, nxt, lane, ws, acc, false);
+        }
+      }
+      return total;
+    }
+  }
   uint32_t item = gw;
   uint32_t entry = item < total ? entry_of(item) : 0u;
   while (item < total) {
@@ -1153,8 +1329,8 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   }
   __syncthreads();
   for (uint32_t round = round0;; ++round) {
-    const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB>(D, st, round, gw, nw, lane,
-                                                                                 ws_all[wib], acc);
+    const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB,
+                                     GD_PAIR && !WIDE && MINB == GD_MINB_HI>(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == ROUND_SWITCH) break;                 // bar[3] = this round (run_round)
     if (total == 0) {                                 // fixed point: later launches return at once
       if (D.hyb && blockIdx.x == 0 && threadIdx.x == 0) D.bar[3] = 0;
