@@ -50,7 +50,8 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
 #endif
 #ifndef GD_PAIR
-#define GD_PAIR 1              // heavy rounds: two inline items per warp (half-warp each)
+#define GD_PAIR 0              // heavy rounds: two inline items per warp (half-warp each); measured
+                               // 36 % slower on corpus200 (spills, no IN(dst) pre-read): off
 #endif
 #ifndef GD_CONT_WIDE
 #define GD_CONT_WIDE 1         // wide items continue depth-first into wide successors
@@ -781,53 +782,62 @@ __device__ __forceinline__ void process_inline2(const Dev& D, CtaStage& st, cons
     y[k] = w < B ? X[w] : 0ull;
   }
   const uint32_t my_stamp = hl < (int)ne ? D.stamp[me.dst] : 1u;
-  const bool dbl = kind == GK_FLOAD || kind == GK_ALOAD || kind == GK_FSTORE || kind == GK_ASTORE;
+  const bool is_fl = kind == GK_FLOAD || kind == GK_ALOAD, is_fs = kind == GK_FSTORE || kind == GK_ASTORE;
+  const bool is_cp = kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE;
   int hr[4] = {-1, -1, -1, -1};                             // heap rows of this lane's columns
-  if (dbl) {
+  if (is_fl || is_fs) {
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       const uint32_t c = hl + 16 * q;
       hr[q] = (c < R.n_cols) ? D.frow[R.r3 + c] : -1;
     }
   }
+  // The two halves run different node kinds: every shuffle below is executed by all 32 lanes
+  // (branches on warp-uniform __any_sync), each half using only its own results.
+  const uint64_t row1 = huword_of(y, (is_cp || is_fl || is_fs) ? (uint32_t)R.r1 : 0u);   // rhs / w
+  uint64_t row0 = 0;
+  if (__any_sync(FULL, is_fs)) row0 = huword_of(y, is_fs ? (uint32_t)R.r0 : 0u);        // FSTORE base v
   int mode = 0, t = -1;
   uint64_t genv = 0;
   uint32_t fmask = 0, hwords = 0;
   if (kind == GK_PRIM || kind == GK_CONST || kind == GK_NEW) {
     mode = 1; t = R.r0;
     if (kind != GK_PRIM) genv = 1ull << (R.r3 & 63);
-  } else if (kind == GK_COPY || kind == GK_SLOAD || kind == GK_RETV || kind == GK_SSTORE) {
+  } else if (is_cp) {
     mode = kind == GK_SSTORE ? 2 : 1; t = R.r0;
-    genv = huword_of(y, (uint32_t)R.r1);
-  } else if (kind == GK_FLOAD || kind == GK_ALOAD) {
+    genv = row1;
+  } else if (is_fl) {
     mode = 1; t = R.r0;
-    const uint64_t wrow = huword_of(y, (uint32_t)R.r1);
+  } else if (is_fs) {
+    mode = 3;
+    genv = row1;                                            // row w, OR-ed into rows (o1, f)
+  }
+  if (__any_sync(FULL, is_fl)) {                            // v = w.f: OR of rows (o1,f), o1 ∈ w
     uint64_t a = 0;
 #pragma unroll
     for (int q = 0; q < 4; ++q) {
       const uint32_t c = hl + 16 * q;
-      const bool take = hr[q] >= 0 && ((wrow >> c) & 1ull);
+      const bool take = is_fl && hr[q] >= 0 && ((row1 >> c) & 1ull);   // NULL has no row
       const uint64_t v = hword_of(y, take ? L + (uint32_t)hr[q] : 0u);
       if (take) { a |= v; hwords += 1; }
     }
-    genv = half_or64(a);
-  } else if (kind == GK_FSTORE || kind == GK_ASTORE) {
-    mode = 3;
-    const uint64_t vrow = huword_of(y, (uint32_t)R.r0);
-    genv = huword_of(y, (uint32_t)R.r1);
+    a = half_or64(a);
+    if (is_fl) genv = a;
+  }
+  if (__any_sync(FULL, is_fs)) {                            // v.f = w: target words of rows (o1, f)
 #pragma unroll
     for (int k = 0; k < HKW; ++k) {
       uint32_t m = 0;
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         const uint32_t c = hl + 16 * q;
-        if (hr[q] >= 0 && ((vrow >> c) & 1ull)) {
+        if (is_fs && hr[q] >= 0 && ((row0 >> c) & 1ull)) {
           const uint32_t w = L + (uint32_t)hr[q];
           if ((w >> 4) == (uint32_t)k) m |= 1u << (w & 15u);
         }
       }
       m = half_or32(m);
-      if ((m >> hl) & 1u) fmask |= 1u << k;
+      if (is_fs && ((m >> hl) & 1u)) fmask |= 1u << k;
     }
   }
   uint32_t nzx = 0, nz = 0, red = 0;

@@ -298,3 +298,21 @@ def test_sbda_schedule(blocks):
     assert st["rounds"] > 0 and st["node_visits"] > 0
     app.build(variant="sbda", byte_model=False)        # rebuild: claims / local stamps reset
     assert np.array_equal(app.app_digests(), digs)
+
+
+def test_heavy_round_instantiation_random_batch():
+    """A narrow batch big enough for the hybrid schedule's heavy rounds (>= 2^17 nodes; the
+    4-CTA/SM instantiation with paired half-warp inline items): 12,000 random
+    tiny ICFGs (every node kind, arity up to 5, recursion, projection) — every app digest and
+    the complete pair lists of 150 of them against the oracle."""
+    gs = [random_tiny(s, max_stmts=7) for s in range(100000, 112000)]
+    assert sum(g.n_nodes for g in gs) >= (1 << 17)
+    app = gd.load(gs)
+    st = app.build()
+    assert st["kernel_launches"] >= 3                # the hybrid sequence ran
+    digs = app.app_digests()
+    for k, g in enumerate(gs):
+        r = oracle.build_idfg(g)
+        assert int(digs[k]) == r.app_digest, g.name
+        if k % 80 == 0:
+            _assert_same(app, k, g, r, g.name)
