@@ -58,6 +58,8 @@ def parse(argv=None):
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--e2e-steps", type=int, default=1)
     ap.add_argument("--e2e-readback", default="facts", choices=["facts", "digests"])
+    ap.add_argument("--e2e-reserve-sms", type=int, default=0,
+                    help="SMs the e2e builds leave free for the previous batch's readback kernels")
     ap.add_argument("--gen-threads", type=int, default=0)
     return ap.parse_args(argv)
 
@@ -361,14 +363,14 @@ def run_ours(args):
     if args.e2e_steps > 0:
         bufs = corpus.ReadbackBuffers()
         corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback,
-                             bufs=bufs)                  # untimed warm-up: sizes the pinned buffers
+                             bufs=bufs, reserve_sms=args.e2e_reserve_sms)   # untimed warm-up: sizes the pinned buffers
         barrier()
         torch.cuda.synchronize()
         d2h = h2d = 0
         t0 = time.perf_counter()
         for _ in range(args.e2e_steps):
             out = corpus.run_pipelined(my_batches, lambda i: apps[i], device=local, readback=args.e2e_readback,
-                                       bufs=bufs)
+                                       bufs=bufs, reserve_sms=args.e2e_reserve_sms)
             for br in out:
                 for k, i in enumerate(br.app_ids):
                     if int(br.digests[k]) != res.digests[i]:

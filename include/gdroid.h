@@ -120,6 +120,9 @@ typedef struct {
                             monotone iteration: the out-of-core sub-graph loop (§III-A1,
                             PAPER.md:524-580) runs each sub-graph this way until no seed
                             changes.                                                         */
+  uint32_t reserve_sms;  /* leave this many SMs' worth of CTAs out of the persistent grid, so
+                            kernels on other streams (e.g. the fact readback of the previous
+                            batch) run beside the fixed point; 0 = full grid */
 } gdroid_build_opts;
 
 /* Variants (Fig. 8-12), recast on B200:

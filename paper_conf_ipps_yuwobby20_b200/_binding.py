@@ -34,7 +34,7 @@ class IcfgDesc(C.Structure):
 class BuildOpts(C.Structure):
     _fields_ = [("async_", C.c_uint32), ("max_rounds", C.c_uint32), ("blocks", C.c_uint32),
                 ("loop_mode", C.c_uint32), ("variant", C.c_uint32), ("no_byte_model", C.c_uint32),
-                ("release_facts", C.c_uint32), ("keep_facts", C.c_uint32)]
+                ("release_facts", C.c_uint32), ("keep_facts", C.c_uint32), ("reserve_sms", C.c_uint32)]
 
 
 class BuildStats(C.Structure):
@@ -172,9 +172,9 @@ class App:
 
     def build(self, max_rounds: int = 0, blocks: int = 0, loop_mode: int = 0,
               asynchronous: bool = False, variant=0, byte_model: bool = True,
-              release_facts: bool = False, keep_facts: bool = False) -> Optional[dict]:
+              release_facts: bool = False, keep_facts: bool = False, reserve_sms: int = 0) -> Optional[dict]:
         o = BuildOpts(1 if asynchronous else 0, max_rounds, blocks, loop_mode, variant_id(variant),
-                      0 if byte_model else 1, 1 if release_facts else 0, 1 if keep_facts else 0)
+                      0 if byte_model else 1, 1 if release_facts else 0, 1 if keep_facts else 0, reserve_sms)
         s = BuildStats()
         _check(lib().gdroid_build_idfg(self._h, C.byref(o), C.byref(s)))
         if asynchronous:

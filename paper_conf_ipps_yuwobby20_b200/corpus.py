@@ -306,7 +306,7 @@ class ReadbackBuffers:
 
 def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], device: int = 0,
                   readback: str = "facts", on_facts: Optional[Callable] = None,
-                  bufs: Optional[ReadbackBuffers] = None) -> List[BatchResult]:
+                  bufs: Optional[ReadbackBuffers] = None, reserve_sms: int = 0) -> List[BatchResult]:
     """End to end through the public API: a loader thread generates batch i+1 and uploads it
     (gdroid_load_batch on its own stream: the paper's dual buffering) while
     batch i builds; batch i's facts come back (gdroid_read_batch_facts into pinned buffers:
@@ -364,7 +364,9 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
                 raise item
             ids, app, load_ms, nn, ib = item
             t0 = time.perf_counter()
-            app.build(asynchronous=True)
+            # the fixed point leaves reserve_sms SMs free, so the readback kernels of batch i
+            # (other stream) run beside it instead of waiting for the persistent grid
+            app.build(asynchronous=True, reserve_sms=reserve_sms if readback == "facts" else 0)
             if prev is not None:                          # read back i while i+1 builds
                 finish(prev)
                 prev = None

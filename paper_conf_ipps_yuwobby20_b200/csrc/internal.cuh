@@ -188,6 +188,7 @@ struct Dev {
   DevStats* stats;
   uint32_t* bar;                // grid barrier {count, generation}
   uint64_t* node_digest;        // [N]
+  uint32_t* node_popc;          // [N] facts per node, written by k_digest (readback sizes)
   unsigned long long* app_digest; // [n_apps]
   uint64_t n_words;             // fact store size in words
   uint32_t n_nodes;
@@ -282,6 +283,9 @@ cudaError_t launch_meth_csr(const Dev& D, uint32_t* ptr, uint32_t* nodes, uint32
 int sbda_max_blocks(int device, uint32_t wide);
 cudaError_t launch_round(const Dev& D, uint32_t round, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_digest(const Dev& D, cudaStream_t s);
+// exclusive prefix of counts[0..n) (u32) into ptr[0..n] (u64) on the device; tmp >= 2 * nblk u64
+cudaError_t launch_scan_counts(const uint32_t* counts, uint32_t n, uint64_t* ptr, uint64_t* tmp, cudaStream_t s);
+size_t scan_tmp_words(uint32_t n);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s,
                         const uint32_t* list = nullptr);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,

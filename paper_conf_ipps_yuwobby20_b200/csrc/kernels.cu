@@ -1707,9 +1707,17 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
     }
     const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane));
     const unsigned long long s2 = has2 ? warp_sum64(digest_words(D, R2, hn2, y2, lane)) : 0ull;
+    uint32_t pc = 0, pc2 = 0;                               // facts per node (readback sizes)
+#pragma unroll
+    for (int k = 0; k < DKW; ++k) { pc += __popcll(y[k]); pc2 += __popcll(y2[k]); }
+    for (uint32_t w = lane + 32 * DKW; w < R.B; w += 32) pc += __popcll(D.facts[R.off + w]);
+    if (has2) for (uint32_t w = lane + 32 * DKW; w < R2.B; w += 32) pc2 += __popcll(D.facts[R2.off + w]);
+    pc = __reduce_add_sync(FULL, pc);
+    pc2 = __reduce_add_sync(FULL, pc2);
     if (lane == 0) {
       D.node_digest[n] = s;
-      if (has2) D.node_digest[n2] = s2;
+      D.node_popc[n] = pc;
+      if (has2) { D.node_digest[n2] = s2; D.node_popc[n2] = pc2; }
       if (R.app != app_cur) {
         if (app_sum) atomicAdd(&D.app_digest[app_cur], app_sum);
         app_cur = R.app;
@@ -1780,7 +1788,71 @@ __global__ void k_expand(Dev D, uint32_t n0, uint32_t n1, const uint64_t* ptr, u
   }
 }
 
+// Exclusive prefix of u32 counts into u64 offsets: per-block scan of SCAN_ITEMS elements (block
+// totals to tmp), one-block scan of the totals, then each block adds its offset.
+constexpr uint32_t SCAN_T = 1024, SCAN_PER = 8, SCAN_ITEMS = SCAN_T * SCAN_PER;
+__device__ __forceinline__ unsigned long long block_exclusive_scan(unsigned long long v, unsigned long long* total) {
+  __shared__ unsigned long long ws[32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  unsigned long long x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) { const unsigned long long t = __shfl_up_sync(FULL, x, o); if (lane >= o) x += t; }
+  if (lane == 31) ws[w] = x;
+  __syncthreads();
+  if (w == 0) {
+    unsigned long long z = lane < (int)(blockDim.x >> 5) ? ws[lane] : 0ull;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) { const unsigned long long t = __shfl_up_sync(FULL, z, o); if (lane >= o) z += t; }
+    ws[lane] = z;
+  }
+  __syncthreads();
+  const unsigned long long incl = x + (w ? ws[w - 1] : 0ull);
+  *total = ws[(blockDim.x >> 5) - 1];
+  __syncthreads();
+  return incl - v;
+}
+__global__ void __launch_bounds__(SCAN_T) k_scan_blocks(const uint32_t* c, uint32_t n, uint64_t* ptr, uint64_t* tot) {
+  const uint64_t b0 = (uint64_t)blockIdx.x * SCAN_ITEMS + (uint64_t)threadIdx.x * SCAN_PER;
+  uint32_t v[SCAN_PER];
+  unsigned long long sum = 0;
+#pragma unroll
+  for (int i = 0; i < (int)SCAN_PER; ++i) { v[i] = b0 + i < n ? c[b0 + i] : 0u; sum += v[i]; }
+  unsigned long long total;
+  unsigned long long run = block_exclusive_scan(sum, &total);
+#pragma unroll
+  for (int i = 0; i < (int)SCAN_PER; ++i) { if (b0 + i < n) ptr[b0 + i] = run; run += v[i]; }
+  if (threadIdx.x == 0) tot[blockIdx.x] = total;
+}
+__global__ void __launch_bounds__(SCAN_T) k_scan_totals(uint64_t* tot, uint32_t nb, uint64_t* ptr, uint32_t n) {
+  unsigned long long carry = 0;
+  for (uint32_t b = 0; b < nb; b += SCAN_T) {
+    const uint32_t i = b + threadIdx.x;
+    const unsigned long long v = i < nb ? tot[i] : 0ull;
+    unsigned long long total;
+    const unsigned long long ex = block_exclusive_scan(v, &total);
+    if (i < nb) tot[i] = carry + ex;
+    carry += total;
+  }
+  if (threadIdx.x == 0) ptr[n] = carry;
+}
+__global__ void __launch_bounds__(SCAN_T) k_scan_add(uint64_t* ptr, uint32_t n, const uint64_t* tot) {
+  const uint64_t b0 = (uint64_t)blockIdx.x * SCAN_ITEMS;
+  const unsigned long long add = tot[blockIdx.x];
+  for (uint32_t i = threadIdx.x; i < SCAN_ITEMS; i += SCAN_T)
+    if (b0 + i < n) ptr[b0 + i] += add;
+}
+
 }  // namespace
+
+size_t scan_tmp_words(uint32_t n) { return (size_t)((n + SCAN_ITEMS - 1) / SCAN_ITEMS) + 1; }
+
+cudaError_t launch_scan_counts(const uint32_t* counts, uint32_t n, uint64_t* ptr, uint64_t* tmp, cudaStream_t s) {
+  const uint32_t nb = (n + SCAN_ITEMS - 1) / SCAN_ITEMS;
+  if (nb) k_scan_blocks<<<nb, SCAN_T, 0, s>>>(counts, n, ptr, tmp);
+  k_scan_totals<<<1, SCAN_T, 0, s>>>(tmp, nb, ptr, n);
+  if (nb) k_scan_add<<<nb, SCAN_T, 0, s>>>(ptr, n, tmp);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_rebase(const Dev& D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* rowptr, uint32_t* argptr,
                           const AppBase* bases, cudaStream_t s) {

@@ -1103,6 +1103,7 @@ struct gdroid_app {
   bool release_pending = false;
   int max_blocks = 0;
   int max_blocks_lo = 0;              // hybrid (large narrow batches): grid of the 3-CTA/SM instantiation
+  int n_sms = 0;
   // PLAIN variant (plain.cu): set-based state, present when loaded with gdroid_load_icfg_plain
   PlainDev P{};
   void* d_plain = nullptr;            // uploaded inputs + sets, locks, stamps, queues, scratch, heap
@@ -1519,7 +1520,8 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     size_t s_mask = GD_SMASK ? align256((size_t)N * 8) : 256;
     size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
-    size_t st = s_mask + s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad;
+    size_t s_pc = align256((size_t)N * 4);
+    size_t st = s_mask + s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad + s_pc;
     e = cudaMallocAsync(&a->d_state, st, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "device state (%zu B): %s", st, cudaGetErrorString(e)));
     char* S = (char*)a->d_state;
@@ -1531,6 +1533,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     D.stats = (DevStats*)S; S += s_stats;
     D.bar = (uint32_t*)S; S += s_bar;
     D.node_digest = (uint64_t*)S; S += s_nd;
+    D.node_popc = (uint32_t*)S; S += s_pc;
     D.app_digest = (unsigned long long*)S;
     a->h_stats = stats_slots().get();
     if (!a->h_stats) return fail(set_err(GDROID_E_OOM, "pinned stats slot"));
@@ -1540,6 +1543,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.hiocc = (D.wide == 0 && N >= HIOCC_NODES) ? 1u : 0u;
   a->max_blocks = fixpoint_max_blocks(device, D.wide, D.hiocc);
   a->max_blocks_lo = fixpoint_max_blocks(device, D.wide, 0u);
+  cudaDeviceGetAttribute(&a->n_sms, cudaDevAttrMultiProcessorCount, device);
   PHASE("device state + k_rebase/k_edges");
   *out = a;
   return GDROID_OK;
@@ -1590,6 +1594,13 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   cudaStream_t s = a->stream;
   const uint32_t N = D.n_nodes;
   uint32_t blocks = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks) : (uint32_t)a->max_blocks;
+  // reserve_sms: shrink the persistent grids by that share of the SMs (occupancy is per SM)
+  auto reserve = [&](uint32_t b) -> uint32_t {
+    if (!o.reserve_sms || a->n_sms <= (int)o.reserve_sms) return b;
+    const uint64_t r = (uint64_t)b * (uint64_t)(a->n_sms - (int)o.reserve_sms) / (uint64_t)a->n_sms;
+    return r ? (uint32_t)r : 1u;
+  };
+  blocks = reserve(blocks);
   a->launches = 0;
   gdroid_status est = ensure_facts(a);               // released by an earlier build: re-allocate
   if (est) return est;
@@ -1642,7 +1653,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
     // The hand-over is device-side: every launch of the alternating sequence is enqueued up
     // front (no host round trip); a launch starts at the round in bar[3] (k_seed sets 1) and
     // returns at once when bar[3] = 0 (an earlier launch reached the fixed point or the limit).
-    uint32_t blocks_lo = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks_lo) : (uint32_t)a->max_blocks_lo;
+    uint32_t blocks_lo = reserve(o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->max_blocks_lo) : (uint32_t)a->max_blocks_lo);
     const uint32_t nw_lo = blocks_lo * (THREADS / 32);
     bool heavy = false;
     D.hyb = 1u;
@@ -1662,7 +1673,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   } else if (sbda) {
     CU(cudaMemsetAsync(D.claim, 0, (size_t)D.n_meths * 4, s));
     CU(cudaMemsetAsync(D.lstamp, 0, (size_t)N * 8, s));
-    const uint32_t bs = o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->sbda_blocks) : (uint32_t)a->sbda_blocks;
+    const uint32_t bs = reserve(o.blocks ? std::min<uint32_t>(o.blocks, (uint32_t)a->sbda_blocks) : (uint32_t)a->sbda_blocks);
     CU(launch_sbda(D, bs, s));
     a->launches++;
   } else if (o.loop_mode == 0) {
@@ -1731,11 +1742,37 @@ gdroid_status gdroid_read_batch_facts(const gdroid_app* ca, uint64_t* ptr, uint6
   DeviceGuard guard(a->device);
   const uint32_t n = a->app_base[a->n_apps];
   const bool cached = pairs && a->counts_build == a->build_serial;
+  if (!a->last_plain) {
+    // MAT store: per-node counts from k_digest, offsets scanned on the device (no host prefix,
+    // no H2D of ptr); the fetch reuses the device offsets of the size query
+    const size_t tw = scan_tmp_words(n);
+    if (!cached) {
+      gdroid_status st = ensure_scratch(a, (size_t)(n + 1 + tw) * 8);
+      if (st) return st;
+      CU(launch_scan_counts(a->D.node_popc, n, a->d_scratch, a->d_scratch + n + 1, a->stream));
+      CU(cudaMemcpyAsync(ptr, a->d_scratch, (size_t)(n + 1) * 8, cudaMemcpyDeviceToHost, a->stream));
+      CU(cudaStreamSynchronize(a->stream));
+      a->counts_build = a->build_serial;
+    }
+    const uint64_t total = ptr[n];
+    if (!pairs) return GDROID_OK;
+    if (cap < total) return set_err(GDROID_E_SMALLBUF, "need %llu pairs, cap %llu", (unsigned long long)total, (unsigned long long)cap);
+    gdroid_status st = ensure_scratch(a, (size_t)(n + 1 + tw) * 8 + (size_t)total * 8 + 8);
+    if (st) return st;
+    uint64_t* d_ptr = a->d_scratch;
+    uint64_t* d_pairs = a->d_scratch + (n + 1 + tw);
+    // the scratch may have been re-allocated (or used by another readback) since the size
+    // query: rebuild the device offsets (a scan of the k_digest counts, ~1 ms per 16M nodes)
+    CU(launch_scan_counts(a->D.node_popc, n, d_ptr, d_ptr + n + 1, a->stream));
+    CU(launch_expand(a->D, 0, n, d_ptr, d_pairs, a->stream));
+    CU(cudaMemcpyAsync(pairs, d_pairs, (size_t)total * 8, cudaMemcpyDeviceToHost, a->stream));
+    CU(cudaStreamSynchronize(a->stream));
+    return GDROID_OK;
+  }
   if (!cached) {
     gdroid_status st = ensure_scratch(a, (size_t)(n + 1) * 8);
     if (st) return st;
-    CU(a->last_plain ? launch_plain_sizes(a->P, 0, n, a->d_scratch, a->stream)
-                     : launch_popc(a->D, 0, n, a->d_scratch, a->stream));
+    CU(launch_plain_sizes(a->P, 0, n, a->d_scratch, a->stream));
     CU(cudaMemcpyAsync(ptr + 1, a->d_scratch, (size_t)n * 8, cudaMemcpyDeviceToHost, a->stream));
     CU(cudaStreamSynchronize(a->stream));
     ptr[0] = 0;
