@@ -1655,7 +1655,7 @@ __global__ void k_apply_seeds(Dev D) {
 // Digest of one node's block held as y[k] = word lane + 32k (k < DKW), plus any words beyond.
 constexpr int DKW = 4;
 __device__ __forceinline__ unsigned long long digest_words(const Dev& D, const NodeRec& R, uint64_t hn,
-                                                           const uint64_t (&y)[DKW], int lane) {
+                                                           const uint64_t (&y)[DKW], int lane, uint32_t& pc) {
   const uint32_t logW = R.logW, L = R.L, B = R.B, jm = (1u << logW) - 1;
   unsigned long long s = 0;
   auto one = [&](uint32_t w, uint64_t x) {
@@ -1672,8 +1672,11 @@ __device__ __forceinline__ unsigned long long digest_words(const Dev& D, const N
   for (int k = 0; k < DKW; ++k)
     if (y[k]) one(lane + 32 * k, y[k]);
   const uint64_t* X = D.facts + R.off;
+#pragma unroll
+  for (int k = 0; k < DKW; ++k) pc += __popcll(y[k]);
   for (uint32_t w = lane + 32 * DKW; w < B; w += 32) {     // blocks beyond 128 words (wide)
     const uint64_t x = X[w];
+    pc += __popcll(x);
     if (x) one(w, x);
   }
   return s;
@@ -1705,13 +1708,9 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
       y[k] = w < R.B ? D.facts[R.off + w] : 0ull;
       y2[k] = (has2 && w < R2.B) ? D.facts[R2.off + w] : 0ull;
     }
-    const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane));
-    const unsigned long long s2 = has2 ? warp_sum64(digest_words(D, R2, hn2, y2, lane)) : 0ull;
     uint32_t pc = 0, pc2 = 0;                               // facts per node (readback sizes)
-#pragma unroll
-    for (int k = 0; k < DKW; ++k) { pc += __popcll(y[k]); pc2 += __popcll(y2[k]); }
-    for (uint32_t w = lane + 32 * DKW; w < R.B; w += 32) pc += __popcll(D.facts[R.off + w]);
-    if (has2) for (uint32_t w = lane + 32 * DKW; w < R2.B; w += 32) pc2 += __popcll(D.facts[R2.off + w]);
+    const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane, pc));
+    const unsigned long long s2 = has2 ? warp_sum64(digest_words(D, R2, hn2, y2, lane, pc2)) : 0ull;
     pc = __reduce_add_sync(FULL, pc);
     pc2 = __reduce_add_sync(FULL, pc2);
     if (lane == 0) {
