@@ -233,6 +233,14 @@ gdroid_status gdroid_read_all_facts(const gdroid_app* app, uint32_t k, uint64_t*
  * (Alg. 3 l.17 h_fact <- d_fact_mat). */
 gdroid_status gdroid_read_batch_facts(const gdroid_app* app, uint64_t* ptr, uint64_t* pairs,
                                       uint64_t cap);
+/* Asynchronous form of gdroid_read_batch_facts: scans the offsets on the device
+ * (one 8-byte synchronous copy of the pair count into *total), expands the pairs on the device
+ * and enqueues the copies of ptr[N_batch+1] and of the pairs into the caller's PINNED buffers
+ * without waiting, so they overlap the next work enqueued (the next batch's fixed point).
+ * Complete with gdroid_stream_sync; the buffers must stay valid until then.  *total > cap:
+ * GDROID_E_SMALLBUF, nothing copied.  `blocks` is reserved (0). */
+gdroid_status gdroid_read_batch_facts_async(gdroid_app* app, uint64_t* ptr, uint64_t* pairs,
+                                            uint64_t cap, uint64_t* total, uint32_t blocks);
 /* Per-node digests d(n) = sum over IN(n) of mix64(mix64(n) ^ pair),
  * computed on the device at the end of the build; per_node may be NULL. */
 gdroid_status gdroid_node_digests(const gdroid_app* app, uint64_t* per_node, uint64_t* app_digest);

@@ -93,6 +93,7 @@ def lib():
         L.gdroid_read_facts_in.argtypes = [P, C.c_uint32, C.c_uint32, P, C.c_uint64, P]
         L.gdroid_read_all_facts.argtypes = [P, C.c_uint32, P, P, C.c_uint64]
         L.gdroid_read_batch_facts.argtypes = [P, P, P, C.c_uint64]
+        L.gdroid_read_batch_facts_async.argtypes = [P, P, P, C.c_uint64, P, C.c_uint32]
         L.gdroid_node_digests.argtypes = [P, P, P]
         L.gdroid_node_digests_in.argtypes = [P, C.c_uint32, P, P]
         L.gdroid_app_digests.argtypes = [P, P]
@@ -112,6 +113,7 @@ def lib():
                   "gdroid_stage_seeds", "gdroid_read_reached", "gdroid_read_nodes_facts", "gdroid_export_facts", "gdroid_import_facts",
                   "gdroid_stream_sync",
                   "gdroid_read_facts", "gdroid_read_facts_in", "gdroid_read_all_facts", "gdroid_read_batch_facts",
+                  "gdroid_read_batch_facts_async",
                   "gdroid_node_digests", "gdroid_node_digests_in", "gdroid_app_digests"):
             getattr(L, f).restype = C.c_int
         _lib = L
@@ -265,6 +267,17 @@ class App:
         pairs = pairs_buf.get(tot) if pairs_buf is not None else np.zeros(max(tot, 1), dtype=np.uint64)[:tot]
         _check(L.gdroid_read_batch_facts(self._h, _ptr(ptr), _ptr(pairs) if tot else None, tot))
         return ptr, pairs[:tot]
+
+    def read_batch_facts_async(self, ptr: np.ndarray, pairs: np.ndarray, total: np.ndarray, blocks: int = 0):
+        """gdroid_read_batch_facts_async: enqueue the whole-batch readback into PINNED buffers
+        (ptr of n+1, pairs of any capacity, total of 1); complete with stream_sync()."""
+        n = sum(self.n_nodes)
+        assert ptr.dtype == np.uint64 and ptr.size >= n + 1 and total.size >= 1
+        rc = lib().gdroid_read_batch_facts_async(self._h, _ptr(ptr), _ptr(pairs), pairs.size, _ptr(total), blocks)
+        if rc == -7:
+            return False                                   # pairs buffer too small (nothing copied)
+        _check(rc)
+        return True
 
     def node_digests(self, k: int = 0) -> Tuple[np.ndarray, int]:
         per = np.zeros(self.n_nodes[k], dtype=np.uint64)

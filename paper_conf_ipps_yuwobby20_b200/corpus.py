@@ -301,7 +301,8 @@ class PinnedBuf:
 
 class ReadbackBuffers:
     def __init__(self):
-        self.ptr, self.pairs = PinnedBuf(), PinnedBuf()
+        self.ptr, self.pairs, self.total = PinnedBuf(), PinnedBuf(), PinnedBuf()
+        self.cap = 0                                  # pairs capacity the async readback may use
 
 
 def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], device: int = 0,
@@ -309,15 +310,18 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
                   bufs: Optional[ReadbackBuffers] = None, reserve_sms: int = 0) -> List[BatchResult]:
     """End to end through the public API: a loader thread generates batch i+1 and uploads it
     (gdroid_load_batch on its own stream: the paper's dual buffering) while
-    batch i builds; batch i's facts come back (gdroid_read_batch_facts into pinned buffers:
-    Alg. 3 l.17 h_fact <- d_fact) while batch i+1 builds on the other stream.
-    readback='digests' reads only the app digests.  A loader failure is re-raised here."""
+    batch i builds.  As soon as batch i's fixed point is done its facts are expanded on the device
+    and their copy to pinned host memory is enqueued (gdroid_read_batch_facts_async — Alg. 3
+    l.17 h_fact <- d_fact); batch i+1's fixed point then runs while the copy engine
+    moves batch i's facts.  readback='digests' reads only the app digests.  A loader failure is
+    re-raised here."""
     import torch
     from . import _binding as gd
     q: "Queue" = Queue(maxsize=1)
     streams = [torch.cuda.Stream(device=device), torch.cuda.Stream(device=device)]
     stop = threading.Event()
     bufs = bufs or ReadbackBuffers()
+    facts = readback == "facts"
 
     def loader():
         try:
@@ -336,12 +340,29 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
 
     out: List[BatchResult] = []
 
+    pending = {"async": False}
+
+    def start_readback(cur):
+        ids, app, st, t0, load_ms, nn = cur[:6]
+        pending["async"] = False
+        if facts and bufs.cap:
+            n = sum(nn)
+            pending["async"] = app.read_batch_facts_async(bufs.ptr.get(n + 1), bufs.pairs.get(bufs.cap),
+                                                          bufs.total.get(1))
+
     def finish(prev):
         ids, app, st, t0, load_ms, nn, ib = prev
         dig = app.app_digests()
         d2h = 8 * len(ids)
-        if readback == "facts":
-            ptr, pairs = app.read_batch_facts(bufs.ptr, bufs.pairs)
+        if facts:
+            n = sum(nn)
+            app.stream_sync()                              # the async readback (if any) is done
+            tot = int(bufs.total.get(1)[0]) if pending["async"] else -1
+            if 0 <= tot <= bufs.cap:
+                ptr, pairs = bufs.ptr.get(n + 1), bufs.pairs.get(bufs.cap)[:tot]
+            else:                                          # first pass / too small: synchronous, grow
+                ptr, pairs = app.read_batch_facts(bufs.ptr, bufs.pairs)
+                bufs.cap = max(bufs.cap, int(1.25 * len(pairs)) + (1 << 20))
             d2h += ptr.nbytes + pairs.nbytes
             if on_facts is not None:
                 base = 0
@@ -364,20 +385,20 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
                 raise item
             ids, app, load_ms, nn, ib = item
             t0 = time.perf_counter()
-            # the fixed point leaves reserve_sms SMs free, so the readback kernels of batch i
-            # (other stream) run beside it instead of waiting for the persistent grid
-            app.build(asynchronous=True, reserve_sms=reserve_sms if readback == "facts" else 0)
-            if prev is not None:                          # read back i while i+1 builds
+            app.build(asynchronous=True, reserve_sms=reserve_sms if facts else 0)
+            if prev is not None:                          # batch i-1's readback ran beside it
                 finish(prev)
                 prev = None
             st = app.sync()
             prev = (ids, app, st, t0, load_ms, nn, ib)
+            start_readback(prev)
         if prev is not None:
             finish(prev)
             prev = None
     finally:
         stop.set()
         if prev is not None:
+            prev[1].stream_sync()
             prev[1].free()
         while th.is_alive() or not q.empty():             # drain so the loader can finish
             try:

@@ -289,7 +289,8 @@ size_t scan_tmp_words(uint32_t n);
 cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, cudaStream_t s,
                         const uint32_t* list = nullptr);
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr,
-                          uint64_t* pairs, cudaStream_t s, const uint32_t* list = nullptr);
+                          uint64_t* pairs, cudaStream_t s, const uint32_t* list = nullptr,
+                          uint32_t max_blocks = 0);
 int fixpoint_max_blocks(int device, uint32_t wide, uint32_t hiocc);
 
 }  // namespace gd

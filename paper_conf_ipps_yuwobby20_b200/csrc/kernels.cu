@@ -1975,8 +1975,10 @@ cudaError_t launch_popc(const Dev& D, uint32_t n0, uint32_t n1, uint64_t* out, c
 }
 
 cudaError_t launch_expand(const Dev& D, uint32_t n0, uint32_t n1, const uint64_t* ptr, uint64_t* pairs,
-                          cudaStream_t s, const uint32_t* list) {
-  k_expand<<<grid_for(n1 - n0), 256, 0, s>>>(D, n0, n1, ptr, pairs, list);
+                          cudaStream_t s, const uint32_t* list, uint32_t max_blocks) {
+  uint32_t g = grid_for(n1 - n0);
+  if (max_blocks && g > max_blocks) g = max_blocks;
+  k_expand<<<g, 256, 0, s>>>(D, n0, n1, ptr, pairs, list);
   return cudaGetLastError();
 }
 

@@ -1909,6 +1909,43 @@ gdroid_status gdroid_stream_sync(gdroid_app* a) {
 
 uint64_t gdroid_fact_bytes(const gdroid_app* a) { return a ? a->D.n_words * 8 : 0; }
 
+// Asynchronous whole-batch readback: offsets scanned on the device (one small
+// synchronous copy of the pair count), pairs expanded on the device, then ptr (n+1 words) and
+// the pairs copied to the caller's PINNED buffers by the copy engine without waiting — the copy
+// overlaps whatever the caller enqueues next (the next batch's fixed point).  Complete with
+// gdroid_stream_sync.  *total gets the pair count; GDROID_E_SMALLBUF (nothing copied) if it
+// exceeds cap.
+gdroid_status gdroid_read_batch_facts_async(gdroid_app* a, uint64_t* ptr, uint64_t* pairs, uint64_t cap,
+                                            uint64_t* total, uint32_t blocks) {
+  (void)blocks;
+  if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
+  if (!a->built || a->last_plain) return set_err(GDROID_E_STATE, "async readback needs a completed MAT build with facts");
+  if (!ptr || !pairs || !total) return set_err(GDROID_E_INVALID, "ptr / pairs / total is NULL");
+  DeviceGuard guard(a->device);
+  const uint32_t n = a->app_base[a->n_apps];
+  const size_t tw = scan_tmp_words(n);
+  gdroid_status st = ensure_scratch(a, (size_t)(n + 1 + tw) * 8);
+  if (st) return st;
+  CU(launch_scan_counts(a->D.node_popc, n, a->d_scratch, a->d_scratch + n + 1, a->stream));
+  CU(cudaMemcpyAsync(total, a->d_scratch + n, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  const uint64_t tot = *total;
+  if (tot > cap) return set_err(GDROID_E_SMALLBUF, "need %llu pairs, cap %llu", (unsigned long long)tot, (unsigned long long)cap);
+  const size_t need = (size_t)(n + 1 + tw) * 8 + (size_t)tot * 8 + 8;
+  if (a->scratch_bytes < need) {                     // grown: the offsets move with the scratch
+    st = ensure_scratch(a, need);
+    if (st) return st;
+    CU(launch_scan_counts(a->D.node_popc, n, a->d_scratch, a->d_scratch + n + 1, a->stream));
+  }
+  uint64_t* d_ptr = a->d_scratch;
+  uint64_t* d_pairs = a->d_scratch + (n + 1 + tw);
+  CU(launch_expand(a->D, 0, n, d_ptr, d_pairs, a->stream));
+  CU(cudaMemcpyAsync(ptr, d_ptr, (size_t)(n + 1) * 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaMemcpyAsync(pairs, d_pairs, (size_t)tot * 8, cudaMemcpyDeviceToHost, a->stream));
+  a->counts_build = ~0ull;                            // scratch now holds pairs after the offsets
+  return GDROID_OK;
+}
+
 gdroid_status gdroid_release_facts(gdroid_app* a) {
   if (!a) return set_err(GDROID_E_INVALID, "app is NULL");
   if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
