@@ -24,6 +24,9 @@ namespace {
 #ifndef GD_MINB
 #define GD_MINB 3              // resident CTAs per SM the fixed-point kernels are compiled for
 #endif
+#ifndef GD_MINB_WIDE
+#define GD_MINB_WIDE GD_MINB   // ... for wide batches (4: measured flat, profiles/r02_ab_knobs.log)
+#endif
 #ifndef GD_MINB_HI
 #define GD_MINB_HI 4           // ... for large narrow batches (Dev::hiocc)
 #endif
@@ -1885,9 +1888,9 @@ static const void* fixpoint_fn(uint32_t wide, uint32_t hiocc) {
   switch (wide) {
     case 0: return hiocc ? (const void*)k_fixpoint<false, CNT, 1, GD_MINB_HI>
                          : (const void*)k_fixpoint<false, CNT, 1, GD_MINB>;
-    case 1: return (const void*)k_fixpoint<true, CNT, 2, GD_MINB>;
-    case 2: return (const void*)k_fixpoint<true, CNT, 4, GD_MINB>;
-    default: return (const void*)k_fixpoint<true, CNT, 8, GD_MINB>;
+    case 1: return (const void*)k_fixpoint<true, CNT, 2, GD_MINB_WIDE>;
+    case 2: return (const void*)k_fixpoint<true, CNT, 4, GD_MINB_WIDE>;
+    default: return (const void*)k_fixpoint<true, CNT, 8, GD_MINB_WIDE>;
   }
 }
 
