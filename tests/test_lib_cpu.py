@@ -75,3 +75,30 @@ def test_loader_rejects_invalid():
     g2 = tiny2()[0]
     mi2 = g2.module_insts.copy(); mi2[0] = 1
     assert _load_status(_mut(g2, module_insts=mi2)) in (-1, -2)
+
+
+def test_loader_size_limits():
+    """GDROID_E_LIMIT (include/gdroid.h): > 512 instances in one module pool, a wide block of
+    > 1024 rows, an out-degree > 32768 — all rejected by host validation before the device."""
+    from synth import IcfgBuilder
+
+    def app(n_inst=1, n_stat=0, fanout=1):
+        b = IcfgBuilder(n_fields=1)
+        t = b.add_type([0])
+        for _ in range(n_stat):
+            b.add_static()
+        insts = [b.add_instance(t) for _ in range(n_inst)]
+        d = b.add_module()
+        m = b.add_method(d, 0, 2)
+        n = b.nop(m)
+        for _ in range(fanout):
+            b.edge(b.entry(m), n)
+        b.edge(n, b.exit(m))
+        b.set_module(d, insts=insts, statics=list(range(n_stat)))
+        b.add_entry(m)
+        return b.build()
+
+    assert _load_status(app(n_inst=513)) == -8             # pool > 512 instances
+    assert _load_status(app(n_inst=100, n_stat=1100)) == -8 # wide block (> 64 instances) of > 1024 rows
+    assert _load_status(app(fanout=32769)) == -8            # out-degree > 32768
+    assert _load_status(app(n_inst=100, n_stat=10, fanout=3)) not in (-1, -2, -8)   # within limits
