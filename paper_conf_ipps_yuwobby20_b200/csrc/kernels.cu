@@ -1675,9 +1675,30 @@ __device__ __forceinline__ unsigned long long digest_words(const Dev& D, const N
   for (int k = 0; k < DKW; ++k)
     if (y[k]) one(lane + 32 * k, y[k]);
   const uint64_t* X = D.facts + R.off;
+  if (logW >= 1) {                                         // wide block: occupied rows only
+    const uint32_t rows = B >> logW, nocc = occ_words(rows), W = 1u << logW;
+    const uint64_t* X = D.facts + R.off;
+    const uint64_t* OCC = X + occ_offset(B);
+    for (uint32_t i = 0; i < nocc; ++i) {
+      const uint64_t ow = OCC[i];
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const uint32_t j = (uint32_t)lane + 32u * h;
+        if (!((ow >> j) & 1ull)) continue;
+        const uint32_t r = i * 64 + j;
+        for (uint32_t q = 0; q < W; ++q) {
+          const uint32_t w = (r << logW) + q;
+          const uint64_t x = X[w];
+          pc += __popcll(x);
+          if (x) one(w, x);
+        }
+      }
+    }
+    return s;
+  }
 #pragma unroll
   for (int k = 0; k < DKW; ++k) pc += __popcll(y[k]);
-  for (uint32_t w = lane + 32 * DKW; w < B; w += 32) {     // blocks beyond 128 words (wide)
+  for (uint32_t w = lane + 32 * DKW; w < B; w += 32) {     // blocks beyond 128 words (narrow)
     const uint64_t x = X[w];
     pc += __popcll(x);
     if (x) one(w, x);
@@ -1706,10 +1727,10 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
     const uint64_t hn2 = has2 ? mix64((uint64_t)(n2 - D.app_node_base[R2.app])) : 0ull;
     uint64_t y[DKW], y2[DKW];
 #pragma unroll
-    for (int k = 0; k < DKW; ++k) {
+    for (int k = 0; k < DKW; ++k) {                         // (wide blocks read occupied rows instead)
       const uint32_t w = lane + 32 * k;
-      y[k] = w < R.B ? D.facts[R.off + w] : 0ull;
-      y2[k] = (has2 && w < R2.B) ? D.facts[R2.off + w] : 0ull;
+      y[k] = (R.logW == 0 && w < R.B) ? D.facts[R.off + w] : 0ull;
+      y2[k] = (has2 && R2.logW == 0 && w < R2.B) ? D.facts[R2.off + w] : 0ull;
     }
     uint32_t pc = 0, pc2 = 0;                               // facts per node (readback sizes)
     const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane, pc));

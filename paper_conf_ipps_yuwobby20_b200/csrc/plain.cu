@@ -460,6 +460,8 @@ __global__ void k_cell_to_mat(PlainDev P, Dev D, uint32_t M) {
           const uint32_t node = P.mnodes[P.mnode_ptr[m] + w * 64 + b];
           const NodeRec R = D.nodes[node];
           atomicOr((unsigned long long*)(D.facts + R.off + ((uint64_t)r << R.logW) + (c >> 6)), 1ull << (c & 63));
+          if (R.logW >= 1)                                  // wide block: row-occupancy bit (digest)
+            atomicOr((unsigned long long*)(D.facts + R.off + ((R.B + 3u) & ~3u) + (r >> 6)), 1ull << (r & 63));
         }
       }
     }
