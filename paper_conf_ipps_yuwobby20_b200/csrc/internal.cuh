@@ -25,10 +25,13 @@ constexpr uint32_t HIOCC_NODES = GD_HIOCC_NODES;   // batches this large are ite
 #define GD_THREADS 256
 #endif
 constexpr int THREADS = GD_THREADS; // fixed-point kernel block size
-#ifndef GD_SMASK
-#define GD_SMASK 0             // narrow blocks: read only word groups flagged in D.smask (measured
-                               // slower, round 1); 0: D.smask is not allocated
+#ifndef GD_NMASK
+#define GD_NMASK 0             // narrow blocks: word-occupancy masks in D.smask (2 words per node
+                               // cover words 0..127); readers load only non-zero words of IN(src).
+                               // Correct (all GPU tests pass) but +6 % on corpus200, +4 % on median
+                               // (profiles/r02_ab_nmask.log): off, D.smask not allocated
 #endif
+constexpr uint32_t NMW = 2;    // mask words per node
 constexpr int WARPS = THREADS / 32;
 
 // One ICFG node (64 B).  Row indices r* are relative to the node's fact block (method-local
@@ -64,15 +67,6 @@ static_assert(sizeof(NodeRec) == 64, "NodeRec must be 64 bytes");
 // flagged rows (a fact written after the reader's bitmap load is re-processed next round,
 // because its writer also queued the node).
 __host__ __device__ __forceinline__ uint32_t occ_offset(uint32_t B) { return (B + 3u) & ~3u; }
-// Narrow blocks (one word per row) carry a 64-bit group-occupancy mask in D.smask: bit i covers
-// words [i << s, (i + 1) << s) with s = mshift_of(B) (s = 2: one 32-byte sector for B <= 256).
-// Readers load only flagged groups; every writer that turns a zero word non-zero sets the bit
-// (same visibility argument as the wide row-occupancy bitmaps).
-__host__ __device__ __forceinline__ uint32_t mshift_of(uint32_t B) {
-  uint32_t l = 0;
-  while ((1u << l) < B) ++l;          // ceil(log2 B)
-  return l > 8 ? l - 6 : 2u;
-}
 __host__ __device__ __forceinline__ uint32_t occ_words(uint32_t rows) { return (rows + 63u) >> 6; }
 
 // Work items.  A node's out-edges are split into chunks of ebs(deg) edges (at most 32 chunks
@@ -179,7 +173,7 @@ struct Dev {
   uint64_t* facts;
   uint64_t* delta;              // wide batches: Δ store, same layout as facts (bits that reached
                                 // IN(n) since n's last visit); nullptr if narrow
-  uint64_t* smask;              // [N] narrow blocks: bit i = word group i (mshift_of(B)) may be non-zero
+  uint64_t* smask;              // [NMW N] narrow word-occupancy masks (GD_NMASK): bit w = word w may be non-zero
   uint32_t* stamp;              // [N] last round a node was queued for (0 = never)
   uint32_t* cont;               // [N] last round a warp continued into the node (0 = never)
   uint32_t* queue;              // [3][n_chunks] rotating class-segmented worklists of
@@ -273,6 +267,7 @@ cudaError_t launch_plain_gather(const PlainDev& P, uint32_t n0, uint32_t n1, con
 
 // kernels.cu launch wrappers (return cudaError_t of the launch)
 cudaError_t launch_seed(const Dev& D, cudaStream_t s);
+cudaError_t launch_nmask_rebuild(const Dev& D, cudaStream_t s);
 cudaError_t launch_rebase(const Dev& D, NodeRec* nodes, uint32_t* nodemeth, uint32_t* rowptr, uint32_t* argptr,
                           const AppBase* bases, cudaStream_t s);
 cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes, const uint32_t* ecol,

@@ -107,6 +107,17 @@ __device__ __forceinline__ void red_or(uint64_t* p, uint64_t v) {
   asm volatile("red.relaxed.gpu.global.or.b64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
 }
 
+// Narrow word-occupancy masks (GD_NMASK): bit w of the node's 2 mask words = word w of IN(n) may
+// be non-zero (words >= 128 are never masked).  A writer that turns a word non-zero sets the bit
+// (one RED, at most once per word per build in practice); a reader that misses a bit still in
+// flight is re-run next round, because that writer also queued the node.
+__device__ __forceinline__ void nmask_note(uint64_t* m, uint32_t w) {
+  if (GD_NMASK && w < 64u * NMW) red_or(m + (w >> 6), 1ull << (w & 63));
+}
+__device__ __forceinline__ bool nmask_has(uint64_t m0, uint64_t m1, uint32_t w) {
+  return !GD_NMASK || w >= 64u * NMW || (((w < 64 ? m0 : m1) >> (w & 63)) & 1ull);
+}
+
 // fire-and-forget 64-bit AND at L2 (clears the Δ bits a visit consumed)
 __device__ __forceinline__ void red_and(uint64_t* p, uint64_t v) {
   asm volatile("red.relaxed.gpu.global.and.b64 [%0], %1;" :: "l"(p), "l"(v) : "memory");
@@ -276,7 +287,7 @@ __device__ __forceinline__ void stage_publish(const Dev& D, CtaStage& st, uint32
 // Words of row `kill` are dropped (C2R).  Returns the number of non-zero words in the low
 // 16 bits and the number of REDs issued in the high bits.
 __device__ __forceinline__ uint32_t or_chunk(uint64_t* Z, const uint64_t (&y)[KW], uint32_t c0,
-                                             int lane, int kill, uint32_t logW, uint64_t& mbits, uint32_t msh) {
+                                             int lane, int kill, uint32_t logW, uint64_t* zm) {
   uint64_t cur[KW];
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
@@ -293,19 +304,12 @@ __device__ __forceinline__ uint32_t or_chunk(uint64_t* Z, const uint64_t (&y)[KW
     if (z & ~cur[k]) {
       red_or(Z + w, z);
       ++red;
-      if (GD_SMASK && cur[k] == 0) mbits |= 1ull << (w >> msh);   // zero word becomes non-zero
+      if (cur[k] == 0) nmask_note(zm, w);                         // zero word becomes non-zero
     }
   }
   return nz | (red << 16);
 }
 
-// Publish the warp's new group-occupancy bits of narrow block `dst` (one RED per warp).
-__device__ __forceinline__ void set_mask(const Dev& D, uint32_t dst, uint64_t mbits, int lane) {
-  if (!GD_SMASK) return;
-  if (!__any_sync(FULL, mbits != 0)) return;
-  const uint64_t m = warp_or64(mbits);
-  if (lane == 0) red_or(D.smask + dst, m);
-}
 
 // ---------------------------------------------------------------------------------- wide blocks
 // Row-sparse processing of a node whose block is wide (W >= 2 words per row): only the rows
@@ -344,7 +348,7 @@ __device__ __forceinline__ void emit_row_words(uint64_t* Z, uint32_t Bt, uint32_
     }
   }
   if (logWt >= 1 && was_zero) red_or(Z + occ_offset(Bt) + (rt >> 6), 1ull << (rt & 63));   // occupancy
-  if (GD_SMASK && logWt == 0 && was_zero && wrote) red_or(mask_t, 1ull << (rt >> mshift_of(Bt)));
+  if (logWt == 0 && was_zero && wrote) nmask_note(mask_t, rt);   // narrow target: word-occupancy
 }
 
 // Semi-naive (Δ) visit of a wide block.  IN(src) supplies the transfer
@@ -552,12 +556,12 @@ __device__ void process_wide(const Dev& D, CtaStage& st, const NodeRec& R, uint3
             }
           }
           if (!call_local) {
-            emit_row_words(Z, Bt, logWt, (uint32_t)rt, out, nz, red, g, D.smask + ep->dst, Zd);
+            emit_row_words(Z, Bt, logWt, (uint32_t)rt, out, nz, red, g, D.smask + (uint64_t)NMW * ep->dst, Zd);
           } else {
             const uint32_t a0 = npar > 3 ? D.arg_ptr[n] : 0u;
             for (uint32_t jj = 0; jj < npar; ++jj) {        // param_jj <- arg_jj whenever arg_jj = rr
               const int a = npar > 3 ? D.args[a0 + jj] : (jj == 0 ? R.r1 : (jj == 1 ? R.r2 : R.r3));
-              if (a == (int)rr) emit_row_words(Z, Bt, logWt, jj, out, nz, red, g, D.smask + ep->dst, Zd);
+              if (a == (int)rr) emit_row_words(Z, Bt, logWt, jj, out, nz, red, g, D.smask + (uint64_t)NMW * ep->dst, Zd);
             }
           }
         }
@@ -619,18 +623,21 @@ __device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r)
 template <bool CNT, bool CD, bool SB = false>
 __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
                                                    uint32_t round, uint32_t nxt, int lane, Acc& acc,
-                                                   bool cont_ok) {
+                                                   bool cont_ok, uint64_t mk0, uint64_t mk1) {
   const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
   const uint64_t* X = D.facts + R.off;             // coherent loads (no __restrict__: see process_wide)
   uint64_t y[KW], p0[KW], p1[KW];
   const uint64_t off0 = shfl64(me.off, 0), off1 = shfl64(me.off, 1);
+  uint32_t hasm = 0;                                        // bit k: word lane + 32k may be non-zero
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
     const uint32_t w = lane + 32 * k;
-    y[k] = w < B ? X[w] : 0ull;
+    const bool h = w < B && nmask_has(mk0, mk1, w);
+    hasm |= (uint32_t)h << k;
+    y[k] = h ? X[w] : 0ull;
     if (GD_PRE) {                                           // IN(dst) of edges 0 and 1, same hop
-      p0[k] = w < B ? D.facts[off0 + w] : 0ull;
-      if (GD_PRE2) p1[k] = (ne > 1 && w < B) ? D.facts[off1 + w] : 0ull;
+      p0[k] = h ? D.facts[off0 + w] : 0ull;                 // (only words IN(src) may carry)
+      if (GD_PRE2) p1[k] = (ne > 1 && h) ? D.facts[off1 + w] : 0ull;
     }
   }
   const uint32_t my_stamp = lane < (int)ne ? D.stamp[me.dst] : 1u;
@@ -700,13 +707,15 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     const uint32_t info = __shfl_sync(FULL, me.info, (int)i);
     const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;  // C2R drops lhs(c)
     uint64_t* Z = D.facts + off;
+    uint64_t* zm = D.smask + (uint64_t)NMW * __shfl_sync(FULL, me.dst, (int)i);
     uint64_t cur[KW];
 #pragma unroll
     for (int k = 0; k < KW; ++k) {
       const uint32_t w = lane + 32 * k;
       const bool keep = y[k] && (int)w != kill;
-      if (GD_PRE && i == 0) cur[k] = keep ? p0[k] : ~0ull;
-      else if (GD_PRE && GD_PRE2 && i == 1) cur[k] = keep ? p1[k] : ~0ull;
+      const bool pre = (hasm >> k) & 1u;                    // pre-read done for this word
+      if (GD_PRE && i == 0) cur[k] = keep ? (pre ? p0[k] : Z[w]) : ~0ull;
+      else if (GD_PRE && GD_PRE2 && i == 1) cur[k] = keep ? (pre ? p1[k] : Z[w]) : ~0ull;
       else cur[k] = keep ? Z[w] : ~0ull;
     }
     bool g = false;
@@ -715,7 +724,10 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
       const uint32_t w = lane + 32 * k;
       const uint64_t z = (int)w == kill ? 0ull : y[k];
       nz += (z != 0);
-      if (z & ~cur[k]) { red_or(Z + w, z); ++red; g = true; }
+      if (z & ~cur[k]) {
+        red_or(Z + w, z); ++red; g = true;
+        if (cur[k] == 0) nmask_note(zm, w);                 // zero word becomes non-zero
+      }
     }
     if (__any_sync(FULL, g)) gmask |= 1u << i;
   }
@@ -860,6 +872,7 @@ __device__ __forceinline__ void process_inline2(const Dev& D, CtaStage& st, cons
     const uint32_t info = __shfl_sync(FULL, me.info, (int)i, 16);
     const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;
     uint64_t* Z = D.facts + off;
+    uint64_t* zm = D.smask + (uint64_t)NMW * __shfl_sync(FULL, me.dst, (int)i, 16);
     uint64_t cur[HKW];
 #pragma unroll
     for (int k = 0; k < HKW; ++k) {
@@ -872,7 +885,10 @@ __device__ __forceinline__ void process_inline2(const Dev& D, CtaStage& st, cons
       const uint32_t w = hl + 16 * k;
       const uint64_t z = (!act || (int)w == kill) ? 0ull : y[k];
       nz += (z != 0);
-      if (z & ~cur[k]) { red_or(Z + w, z); ++red; g = true; }
+      if (z & ~cur[k]) {
+        red_or(Z + w, z); ++red; g = true;
+        if (cur[k] == 0) nmask_note(zm, w);
+      }
     }
     if (__ballot_sync(FULL, g) & hmask) gmask |= 1u << i;
   }
@@ -892,7 +908,8 @@ template <bool WIDE, bool CNT, int MW, bool CD, bool SB = false>
 __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
                                  uint32_t nxt, int lane, WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont,
                                  bool light = false) {
-  const uint64_t mk = GD_SMASK ? __ldcg(D.smask + n) : ~0ull;   // (issued with the NodeRec load)
+  const uint64_t mk0 = GD_NMASK ? D.smask[(uint64_t)NMW * n] : ~0ull;       // (issued with the NodeRec load)
+  const uint64_t mk1 = GD_NMASK ? D.smask[(uint64_t)NMW * n + 1] : ~0ull;
   const NodeRec R = D.nodes[n];
   InlEdge me{0u, 0u, 0ull};                                 // inline chunk-0 edge of this lane (same hop)
   if (GD_INL && !WIDE && lane < 4) me = D.inl[4 * n + lane];
@@ -915,8 +932,8 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
       return cont_v;
     }
   }
-  if (GD_INL && !WIDE && !GD_SMASK && first && R.n_inl) {   // (wide batches: measured slower)
-    return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light);
+  if (GD_INL && !WIDE && first && R.n_inl) {               // (wide batches: measured slower)
+    return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
   }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
@@ -926,8 +943,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
 
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
   //      the rows the transfer function reads
-  const uint32_t msh = mshift_of(B);
-  auto has = [&](uint32_t w) -> bool { return !GD_SMASK || ((mk >> (w >> msh)) & 1ull); };
+  auto has = [&](uint32_t w) -> bool { return nmask_has(mk0, mk1, w); };
   uint64_t y[KW];
 #pragma unroll
   for (int k = 0; k < KW; ++k) {
@@ -1021,9 +1037,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
           const uint32_t info = ep->info;
           const uint64_t off = ep->off;
           const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;     // C2R drops lhs(c)
-          uint64_t mb = 0;
-          const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW, mb, msh);
-          set_mask(D, ep->dst, mb, lane);
+          const uint32_t r = or_chunk(D.facts + off, y, c0, lane, kill, logW, D.smask + (uint64_t)NMW * ep->dst);
           nz += r & 0xffffu;
           red += r >> 16;
           if (r >> 16) gmask |= 1u << i;
@@ -1069,9 +1083,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
             const uint32_t ws = ((uint32_t)src << logW) + j;
             z[k] = (src >= 0 && has(ws)) ? X[ws] : 0ull;                  // CALL/EXIT: identity
           }
-          uint64_t mb = 0;
-          const uint32_t r = or_chunk(Z, z, c0, lane, -1, logW, mb, mshift_of(Bt));
-          set_mask(D, ep->dst, mb, lane);
+          const uint32_t r = or_chunk(Z, z, c0, lane, -1, logW, D.smask + (uint64_t)NMW * ep->dst);
           nz += r & 0xffffu;
           red += r >> 16;
           if (r >> 16) g = true;
@@ -1099,8 +1111,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
           }
           __syncwarp();
           if (!WIDE || (W == 1 && logWt == 0)) {            // one word per row on both sides
-            uint64_t v[KW], cur[KW], mb = 0;
-            const uint32_t mst = mshift_of(Bt);
+            uint64_t v[KW], cur[KW];
 #pragma unroll
             for (int k = 0; k < KW; ++k) v[k] = (src[k] >= 0 && has((uint32_t)src[k])) ? X[src[k]] : 0ull;
 #pragma unroll
@@ -1122,10 +1133,9 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                 red_or(Z + r0 + lane + 32 * k, v[k]);
                 ++red;
                 g = true;
-                if (GD_SMASK && cur[k] == 0) mb |= 1ull << ((r0 + lane + 32 * k) >> mst);
+                if (cur[k] == 0) nmask_note(D.smask + (uint64_t)NMW * ep->dst, r0 + lane + 32 * k);
               }
             }
-            set_mask(D, ep->dst, mb, lane);
           } else if constexpr (WIDE) {
 #pragma unroll
             for (int k = 0; k < KW; ++k) {
@@ -1146,7 +1156,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
                     if (q == (cd >> 6)) out[q] |= 1ull << (cd & 63);
                 }
               }
-              emit_row_words(Z, Bt, logWt, r, out, nz, red, g, D.smask + ep->dst, D.delta + off);   // occupancy, Δ
+              emit_row_words(Z, Bt, logWt, r, out, nz, red, g, D.smask + (uint64_t)NMW * ep->dst, D.delta + off);   // occupancy, Δ
             }
           }
         }
@@ -1649,6 +1659,25 @@ __global__ void k_apply_seeds(Dev D) {
   if (R.logW >= 1) {
     atomicOr((unsigned long long*)(D.delta + R.off + w), bit);
     atomicOr((unsigned long long*)(D.facts + R.off + occ_offset(R.B) + (row >> 6)), 1ull << (row & 63));
+  } else if (GD_NMASK && w < 64u * NMW) {
+    atomicOr((unsigned long long*)(D.smask + (uint64_t)NMW * node + (w >> 6)), 1ull << (w & 63));
+  }
+}
+
+// Narrow word-occupancy masks from the facts themselves (after gdroid_import_facts).
+__global__ void k_nmask_rebuild(Dev D) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t nw = gridDim.x * (blockDim.x >> 5);
+  for (uint32_t n = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); n < D.n_nodes; n += nw) {
+    const NodeRec R = D.nodes[n];
+    if (R.logW != 0) continue;
+#pragma unroll
+    for (uint32_t q = 0; q < NMW; ++q) {
+      const uint32_t w0 = q * 64 + lane, w1 = w0 + 32;
+      const bool a = w0 < R.B && D.facts[R.off + w0] != 0, b = w1 < R.B && D.facts[R.off + w1] != 0;
+      const uint64_t m = (uint64_t)__ballot_sync(FULL, a) | ((uint64_t)__ballot_sync(FULL, b) << 32);
+      if (lane == 0) D.smask[(uint64_t)NMW * n + q] = m;
+    }
   }
 }
 
@@ -1890,6 +1919,11 @@ cudaError_t launch_edges(const Dev& D, Edge* edges, InlEdge* inl, NodeRec* nodes
   uint32_t blocks = (D.n_nodes + 255) / 256;
   blocks = blocks == 0 ? 1u : (blocks > 148 * 8 ? 148 * 8 : blocks);
   k_edges<<<blocks, 256, 0, s>>>(D, edges, inl, nodes, ecol, ekind, exoff);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_nmask_rebuild(const Dev& D, cudaStream_t s) {
+  k_nmask_rebuild<<<1184, 256, 0, s>>>(D);
   return cudaGetLastError();
 }
 

@@ -1089,6 +1089,7 @@ struct gdroid_app {
   uint64_t build_serial = 0;          // completed builds (readback count cache key)
   // incremental builds / out-of-core sub-graphs
   bool state_valid = false;           // stamps hold a completed build's history
+  bool mask_stale = false;            // facts imported: narrow occupancy masks must be rebuilt
   bool facts_valid = false;           // the fact store holds facts (build or import), not garbage
   uint32_t round_base = 0;            // rounds used by earlier builds of this handle
   std::vector<uint32_t> seed_nodes;   // staged for the next keep_facts build
@@ -1517,7 +1518,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e)));
     D.facts = a->d_facts;
     D.delta = Lo.wide ? a->d_facts + std::max<uint64_t>(Lo.fact_words, 4) : nullptr;
-    size_t s_mask = GD_SMASK ? align256((size_t)N * 8) : 256;
+    size_t s_mask = GD_NMASK ? align256((size_t)N * 8 * NMW) : 256;
     size_t s_stamp = align256((size_t)N * 8), s_queue = align256((size_t)3 * NC * 4), s_counts = align256(3 * CNT_STRIDE * 4);
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t s_pc = align256((size_t)N * 4);
@@ -1612,11 +1613,16 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   // (a2) zero the fact matrices and the worklist state
   if (!(o.keep_facts && a->facts_valid)) CU(cudaMemsetAsync(D.facts, 0, D.n_words * 8, s));
   if (D.delta) CU(cudaMemsetAsync(D.delta, 0, D.n_words * 8, s));   // empty at every fixed point
+  const bool facts_kept = o.keep_facts && a->facts_valid;
   if (!keep) {
     CU(cudaMemsetAsync(D.stamp, 0, (size_t)N * 8, s));   // stamp + cont
-    if (GD_SMASK) CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8, s));
+    if (GD_NMASK) CU(cudaMemsetAsync(D.smask, 0, (size_t)N * 8 * NMW, s));
     a->round_base = 0;
   }
+  // narrow word masks must describe the kept facts: rebuilt from them after an import (a fresh
+  // handle's masks were just zeroed, the facts were not)
+  if (GD_NMASK && facts_kept && (a->mask_stale || !keep)) CU(launch_nmask_rebuild(D, s));
+  a->mask_stale = false;
   CU(cudaMemsetAsync(D.counts, 0, 3 * CNT_STRIDE * 4, s));
   CU(cudaMemsetAsync(D.stats, 0, sizeof(DevStats), s));
   CU(cudaMemsetAsync(D.bar, 0, 256, s));                 // barrier + round descriptor words
@@ -1896,6 +1902,7 @@ gdroid_status gdroid_import_facts(gdroid_app* a, const void* host, uint64_t byte
   if (st) return st;
   CU(cudaMemcpyAsync(a->d_facts, host, bytes, cudaMemcpyHostToDevice, a->stream));
   a->facts_valid = true;
+  a->mask_stale = true;                               // narrow masks are rebuilt by the next keep build
   a->built = false;                                   // facts no longer those of a build
   return GDROID_OK;
 }

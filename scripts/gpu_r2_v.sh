@@ -1,0 +1,10 @@
+# narrow word-occupancy masks (GD_NMASK): parity + A/B
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -1
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -2
+for F in "" "-DGD_NMASK=0"; do
+  GDROID_NVCC_FLAGS="$F" python -c "import __graft_entry__ as g; g.build()" || exit 1
+  timeout 900 python bench.py --n-apps 200 --steps 2 --warmup 1 --no-per-config --no-cpu-baseline --e2e-steps 0 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('[$F] corpus200', round(d['ms_per_step'],1), 'fix', round(d['fixpoint_ms_per_step_rank0'],1), 'wide', round(d['batch_ms_rank0']['wide'],1), d['parity']['mismatches'])"
+  timeout 600 python bench.py --workload median --steps 5 --warmup 2 --no-cpu-baseline --e2e-steps 0 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('[$F] median', round(d['ms_per_step'],3), d['rounds_rank0'])"
+  timeout 600 python bench.py --workload small --steps 5 --warmup 2 --no-cpu-baseline --e2e-steps 0 2>&1 | tail -1 | python -c "import json,sys; d=json.loads(sys.stdin.read()); print('[$F] small', round(d['ms_per_step'],3), d['rounds_rank0'])"
+done
+python -c "import __graft_entry__ as g; g.build()"
