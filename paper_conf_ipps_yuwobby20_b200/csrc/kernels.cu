@@ -52,6 +52,10 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_BAR_NS
 #define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
 #endif
+#ifndef GD_PF
+#define GD_PF 0                // two-stage prefetch pipeline across the items of a warp (run_round):
+                               // +9 % on corpus200 (profiles/r02_ab_prefetch.log), off
+#endif
 #ifndef GD_PAIR
 #define GD_PAIR 0              // heavy rounds: two inline items per warp (half-warp each); measured
                                // 36 % slower on corpus200 (spills, no IN(dst) pre-read): off
@@ -1309,7 +1313,26 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     }
     const uint32_t nitem = item + nw;
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
-    if (nitem < total && lane < 2) {                                   // NodeRec, inline edges into L1
+    if constexpr (GD_PF) {
+      // two-stage software pipeline: the records of item i+2 into L1, and — from item i+1's
+      // records, prefetched one iteration ago — the lines of its IN(src) and of the first two
+      // IN(dst) blocks into L2, all before item i's own chain starts
+      const uint32_t n2item = nitem + nw;
+      if (n2item < total && lane < 2) {
+        const uint32_t nn2 = entry_of(n2item) >> 5;
+        asm volatile("prefetch.global.L1 [%0];" :: "l"(lane == 0 ? (const char*)(D.nodes + nn2) : (const char*)(D.inl + 4 * nn2)));
+      }
+      if (nitem < total && lane < 24 && (nentry & 31u) == 0) {
+        const uint32_t nn = nentry >> 5;
+        const uint32_t Bn = D.nodes[nn].B, line = lane & 7u;
+        if (D.nodes[nn].logW == 0 && line * 16u < Bn) {
+          const uint32_t which = lane >> 3;                  // 0: IN(src), 1-2: IN(dst) of inline edges
+          const uint64_t o = which == 0 ? D.nodes[nn].off
+                                        : (which <= D.nodes[nn].n_inl ? D.inl[4 * nn + which - 1].off : ~0ull);
+          if (o != ~0ull) asm volatile("prefetch.global.L2 [%0];" :: "l"((const char*)(D.facts + o + line * 16u)));
+        }
+      }
+    } else if (nitem < total && lane < 2) {                            // NodeRec, inline edges into L1
       const uint32_t nn = nentry >> 5;
       asm volatile("prefetch.global.L1 [%0];" :: "l"(lane == 0 ? (const char*)(D.nodes + nn) : (const char*)(D.inl + 4 * nn)));
     }
