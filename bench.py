@@ -190,7 +190,7 @@ def ncu_traffic(workload):
 
 
 # ------------------------------------------------------------------ CPU oracle legs
-def oracle_sample_ids(plan, make_app_cost, budget_nodes):
+def oracle_sample_ids(plan, budget_nodes):
     """A size-stratified sample of the workload's narrow apps (evenly spaced in size order)
     whose node count is about budget_nodes.  Worst-shaped apps (~800 s of one core each) are
     excluded from the timed sample and reported separately."""
@@ -226,7 +226,7 @@ def run_reference(args):
     plan, make_app, desc, scaling = workload(args, 1)
     P = host_threads()
     per_step_nodes = ORACLE_NODES_PER_CORE_S * P * 4.0   # ~4 s of P threads per step
-    ids = oracle_sample_ids(plan, None, per_step_nodes * (args.steps + args.warmup))
+    ids = oracle_sample_ids(plan, per_step_nodes * (args.steps + args.warmup))
     if not ids:                                          # a preset workload: its one app
         ids = plan.shards[0]
     apps = [make_app(i) for i in ids]
@@ -452,7 +452,7 @@ def run_ours(args):
         import oracle
         oracle.build()
         P = host_threads()
-        ids = oracle_sample_ids(plan, None, ORACLE_NODES_PER_CORE_S * P * args.cpu_seconds)
+        ids = oracle_sample_ids(plan, ORACLE_NODES_PER_CORE_S * P * args.cpu_seconds)
         sample_apps = [apps[i] if i in apps else make_app(i) for i in ids]
         if not sample_apps and not plan.wide[my_ids[0]]:
             ids, sample_apps = [my_ids[0]], [apps[my_ids[0]]]

@@ -52,6 +52,9 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #ifndef GD_BAR_NS
 #define GD_BAR_NS 20           // grid barrier: __nanosleep between polls of the generation word
 #endif
+#ifndef GD_CD_HI
+#define GD_CD_HI 0             // narrow continuation compiled into the 4-CTA/SM (heavy-round) build too
+#endif
 #ifndef GD_PF
 #define GD_PF 0                // two-stage prefetch pipeline across the items of a warp (run_round):
                                // +9 % on corpus200 (profiles/r02_ab_prefetch.log), off
@@ -1375,7 +1378,7 @@ __global__ void __launch_bounds__(THREADS, MINB) k_fixpoint(Dev D) {
   }
   __syncthreads();
   for (uint32_t round = round0;; ++round) {
-    const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && MINB == GD_MINB,
+    const uint32_t total = run_round<WIDE, CNT, MW, GD_CONT_DENSE && !WIDE && (MINB == GD_MINB || GD_CD_HI),
                                      GD_PAIR && !WIDE && MINB == GD_MINB_HI>(D, st, round, gw, nw, lane, ws_all[wib], acc);
     if (total == ROUND_SWITCH) break;                 // bar[3] = this round (run_round)
     if (total == 0) {                                 // fixed point: later launches return at once
