@@ -84,3 +84,26 @@ def test_pipelined_loader_error_surfaces():
     bad.module_insts[:] = 0                          # pools lose their sites: V1 fails (E_POOL)
     with pytest.raises(gd.GdroidError):
         corpus.run_pipelined([[0], [1]], lambda i: random_tiny(5) if i == 0 else bad)
+
+
+def test_async_batch_readback_and_reserve_sms():
+    """gdroid_read_batch_facts_async into pinned buffers equals the synchronous readback; a
+    too-small pairs buffer is reported (nothing copied); a build with reserve_sms (smaller
+    persistent grid) reaches the same fixed point."""
+    gs = [random_tiny(s, wide_pad=(90 if s % 3 == 0 else 0)) for s in range(500, 560)]
+    app = gd.load(gs)
+    app.build()
+    digs = app.app_digests().copy()
+    ptr, pairs = app.read_batch_facts()
+    bufs = corpus.ReadbackBuffers()
+    n = sum(app.n_nodes)
+    assert app.read_batch_facts_async(bufs.ptr.get(n + 1), bufs.pairs.get(max(1, len(pairs) - 1)),
+                                      bufs.total.get(1)) is False
+    assert app.read_batch_facts_async(bufs.ptr.get(n + 1), bufs.pairs.get(len(pairs) + 8), bufs.total.get(1))
+    app.stream_sync()
+    assert int(bufs.total.get(1)[0]) == len(pairs)
+    assert np.array_equal(bufs.ptr.get(n + 1), ptr)
+    assert np.array_equal(bufs.pairs.get(len(pairs)), pairs)
+    app.build(reserve_sms=16)
+    assert np.array_equal(app.app_digests(), digs)
+    app.free()
