@@ -117,6 +117,43 @@ def tiny2():
     return g, L, slots, insts
 
 
+def tiny_args(wide_pad: int = 0):
+    """A call with 5 parameters and one local passed three times (``r = m1(a, a, b, a, -)``),
+    the shape whose wide-pool form lost parameters 4+ in round 1 (param_j <-
+    arg_j for every j).  The callee stores through its first parameter, so a heap fact comes
+    back through RET.  ``wide_pad`` > 0 pads the pool with field-less instances below and above
+    the real ones (|Q| > 64: the wide-block path).  Expected sets: tiny_args.expected (by hand;
+    the padding changes nothing)."""
+    b = IcfgBuilder(n_fields=2)
+    F = 1
+    T = b.add_type([F]); T0 = b.add_type([])
+    pad_lo = [b.add_instance(T0) for _ in range(wide_pad // 2)]
+    o1 = b.add_instance(T); o2 = b.add_instance(T)
+    pad_hi = [b.add_instance(T0) for _ in range(wide_pad - wide_pad // 2)]
+    d = b.add_module(insts=pad_lo + [o1, o2] + pad_hi)
+    m0 = b.add_method(d, 0, 4)    # a b r RET0
+    m1 = b.add_method(d, 5, 7)    # p0 p1 p2 p3 p4 t RET1
+    a, bb, r = (b.L(m0, i) for i in range(3))
+    p0, p2, p3 = b.L(m1, 0), b.L(m1, 2), b.L(m1, 3)
+    t = b.L(m1, 5)
+    L = {"e0": b.entry(m0), "x0": b.exit(m0), "e1": b.entry(m1), "x1": b.exit(m1)}
+    L["n1"] = b.new(m0, a, o1)
+    L["n2"] = b.new(m0, bb, o2)
+    L["n3"], L["n4"] = b.call(m0, r, [a, a, bb, a, -1], [m1])
+    L["k0"] = b.fstore(m1, p0, F, p2)
+    L["k1"] = b.copy(m1, t, p3)
+    L["k2"] = b.retv(m1, t)
+    b.chain(L["e0"], L["n1"], L["n2"], L["n3"])
+    b.chain(L["n4"], L["x0"])
+    b.chain(L["e1"], L["k0"], L["k1"], L["k2"], L["x1"])
+    b.add_entry(m0)
+    g = b.build(name=f"tiny_args{'_wide' if wide_pad else ''}")
+    slots = {"a": 0, "b": 1, "r": 2, "R0": 3, "p0": 4, "p1": 5, "p2": 6, "p3": 7, "p4": 8,
+             "t": 9, "R1": 10, "o1.f": 11, "o2.f": 12}
+    insts = {"N": 0, "o1": o1, "o2": o2}
+    return g, L, slots, insts
+
+
 def fig2():
     b = IcfgBuilder(n_fields=1)
     T = b.add_type([])

@@ -10,7 +10,7 @@ import pytest
 
 import oracle
 import paper_conf_ipps_yuwobby20_b200 as gd
-from programs import fig2, load_expected, tiny, tiny2
+from programs import fig2, load_expected, tiny, tiny2, tiny_args
 from synth import random_tiny
 from synth.reductions import random_inline_pair, random_rd, random_ssa_loop
 
@@ -27,12 +27,14 @@ def _assert_same(app, k, g, r, label=""):
         raise AssertionError(f"{label}: CSR layout differs")
 
 
-@pytest.mark.parametrize("which", ["tiny", "tiny_m2", "tiny2", "fig2"])
+@pytest.mark.parametrize("which", ["tiny", "tiny_m2", "tiny2", "fig2", "tiny_args", "tiny_args_wide"])
 def test_golden_programs(which):
     if which == "fig2":
         g = fig2()[0]
     elif which == "tiny2":
         g, L, slots, insts = tiny2()
+    elif which.startswith("tiny_args"):      # 5-param call, one local passed 3 times (narrow / |Q|>64)
+        g, L, slots, insts = tiny_args(wide_pad=(100 if which.endswith("wide") else 0))
     else:
         g, L, slots, insts = tiny(m2_entry=(which == "tiny_m2"))
     app = gd.load(g)
@@ -43,7 +45,7 @@ def test_golden_programs(which):
     assert dig == r.app_digest and np.array_equal(per, r.node_digest)
     assert st["rounds"] > 0 and st["node_visits"] > 0
     if which != "fig2":      # and against the hand-computed fixture directly
-        exp = load_expected(which)
+        exp = load_expected("tiny_args" if which.startswith("tiny_args") else which)
         inv_s = {v: k for k, v in slots.items()}
         inv_i = {v: k for k, v in insts.items()}
         for lab, n in L.items():
@@ -269,7 +271,7 @@ def test_cell_major_variant_random(chunk):
     pools, arity up to 5) and the hand goldens — pair for pair against the oracle."""
     gs = [random_tiny(s, wide_pad=(80 if s % 4 == 0 else 0)) for s in range(13000 + chunk * 30, 13030 + chunk * 30)]
     if chunk == 0:
-        gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0]]
+        gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0], tiny_args()[0], tiny_args(100)[0]]
     for g in gs:
         app = gd.load(g, plain=True)
         st = app.build(variant="cell")
@@ -287,7 +289,7 @@ def test_sbda_schedule(blocks):
     pass with shared-memory local worklists; narrow + wide random tiny ICFGs (arity up to 5,
     recursion, projection) and the goldens in one batch, pair for pair against the oracle."""
     gs = [random_tiny(s, max_stmts=7, wide_pad=(90 if s % 3 == 0 else 0)) for s in range(14000, 14120)]
-    gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0]]
+    gs += [tiny(m2_entry=True)[0], tiny2()[0], fig2()[0], tiny_args()[0], tiny_args(100)[0]]
     app = gd.load(gs)
     st = app.build(variant="sbda", blocks=blocks)
     digs = app.app_digests()

@@ -10,7 +10,7 @@ import pytest
 import oracle
 from kleene import Sym, kleene, reach, to_sym
 from reductions import andersen, reaching_definitions
-from programs import fig2, load_expected, tiny, tiny2
+from programs import tiny_args, fig2, load_expected, tiny, tiny2
 from synth import random_tiny
 from synth.reductions import random_inline_pair, random_rd, random_ssa_loop
 
@@ -38,6 +38,18 @@ def test_golden_tiny2_projection():
     """Hand-computed projection example (two modules, partial pools; C1/C3, A9)."""
     g, L, slots, insts = tiny2()
     exp = load_expected("tiny2")
+    assert set(exp) == set(L)
+    r = oracle.build_idfg(g)
+    for lab, n in L.items():
+        assert _named(g, slots, insts, r, n) == exp[lab], lab
+
+
+@pytest.mark.parametrize("pad", [0, 100])
+def test_golden_tiny_args(pad):
+    """Hand-computed IN sets of a 5-parameter call with one local passed three times (C3 maps
+    it to every such parameter), narrow and wide pools (padding never flows)."""
+    g, L, slots, insts = tiny_args(wide_pad=pad)
+    exp = load_expected("tiny_args")
     assert set(exp) == set(L)
     r = oracle.build_idfg(g)
     for lab, n in L.items():
