@@ -170,11 +170,16 @@ gdroid_status gdroid_load_icfg(const gdroid_icfg_desc* desc, int device, void* c
                                gdroid_app** out);
 /* Load n_apps independent apps into ONE handle; they share every device round
  * (IDFG-instance batching).  Node ids, slot gids and digests stay
- * per app.  Host side: the apps are validated and laid out in parallel on a worker
- * pool of min(hardware threads, $GDROID_HOST_THREADS) threads; the call returns once
- * the tables are on the device (stream-ordered kernels k_rebase / k_edges finish the
- * layout before any later work on cuda_stream).  The descriptor arrays are only read
- * during the call. */
+ * per app.  Device layout (the default): the host validates and lays
+ * out only the per-type / per-method / per-module tables (apps in parallel on a worker
+ * pool of min(hardware threads, $GDROID_HOST_THREADS) threads), copies the raw
+ * descriptor arrays into a pinned staging buffer and uploads them; kernels resolve the
+ * operands, validate every node and edge (V1-V6), and build the node / edge records and
+ * the field-row and projection tables.  The call waits for those kernels (two short
+ * round trips), so every validation error is returned by this call: the host validator
+ * then re-runs for the exact status and message.  $GDROID_HOST_LAYOUT=1 (and hosts
+ * without a device) lay out every table on the host instead (same bytes).  The
+ * descriptor arrays are only read during the call. */
 gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, int device,
                                 void* cuda_stream, gdroid_app** out);
 /* Load ONE app for every variant including GDROID_V_PLAIN: the MAT handle of
@@ -257,6 +262,14 @@ gdroid_status gdroid_debug_read_trace(const gdroid_app* app, uint64_t* out, uint
 /* Diagnostics: per-phase cycle counters of the last build (only filled by a library compiled
  * with -DGD_PHASES): setup, edges, pushes, round end (publish + grid barrier), items. */
 gdroid_status gdroid_debug_phases(const gdroid_app* app, uint64_t* out8);
+/* Diagnostics: copy one of the handle's device tables to host memory, to compare
+ * the device layout (layout.cu, the default) with the host layout ($GDROID_HOST_LAYOUT=1) byte for
+ * byte.  which: 0 NodeRec[N] (64 B), 1 Edge[E] (32 B), 2 InlEdge[4N] (16 B), 3 field-row table
+ * (i32), 4 projection tables (i32), 5 argument rows (i32), 6 row_ptr u32[N+1], 7 arg_ptr
+ * u32[N+1], 8 node-method u32[N].  host == NULL: *bytes = the size only; cap < size:
+ * GDROID_E_SMALLBUF. */
+gdroid_status gdroid_debug_tables(const gdroid_app* app, uint32_t which, void* host, uint64_t cap,
+                                  uint64_t* bytes);
 void          gdroid_free(gdroid_app* app);
 const char*   gdroid_last_error(void);   /* thread-local; valid until the next call */
 uint32_t      gdroid_abi_version(void);

@@ -105,6 +105,8 @@ def lib():
         L.gdroid_debug_read_trace.restype = C.c_int
         L.gdroid_debug_phases.argtypes = [P, P]
         L.gdroid_debug_phases.restype = C.c_int
+        L.gdroid_debug_tables.argtypes = [P, C.c_uint32, P, C.c_uint64, P]
+        L.gdroid_debug_tables.restype = C.c_int
         L.gdroid_free.argtypes = [P]
         L.gdroid_free.restype = None
         L.gdroid_last_error.restype = C.c_char_p
@@ -306,6 +308,14 @@ class App:
         out = np.zeros(8, dtype=np.uint64)
         _check(lib().gdroid_debug_phases(self._h, _ptr(out)))
         return out
+
+    def table(self, which: int) -> np.ndarray:
+        """Raw bytes of one device table (gdroid_debug_tables; diagnostics)."""
+        n = C.c_uint64(0)
+        _check(lib().gdroid_debug_tables(self._h, which, None, 0, C.byref(n)))
+        buf = np.zeros(max(n.value, 1), dtype=np.uint8)
+        _check(lib().gdroid_debug_tables(self._h, which, _ptr(buf), buf.size, C.byref(n)))
+        return buf[:n.value]
 
     def free(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -8,7 +8,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgdroid.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("loader.cu", "kernels.cu", "plain.cu")]
+SOURCES = [os.path.join(CSRC, f) for f in ("loader.cu", "kernels.cu", "plain.cu", "layout.cu")]
 DEPS = SOURCES + [os.path.join(CSRC, "internal.cuh"), os.path.join(ROOT, "include", "gdroid.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",

@@ -257,6 +257,66 @@ struct PlainDev {
   const uint32_t* mgrow;
 };
 
+// ---- device layout of a batch (layout.cu): the per-node / per-edge part of (a1)
+// run as kernels over the uploaded descriptor arrays.  The host validates and lays out only the
+// per-type / per-method / per-module tables; node records, operand rows, fact offsets, field-row
+// and projection tables, edge records and V1-V6 of every node and edge are computed here.
+__host__ __device__ __forceinline__ uint32_t kind_cls(uint32_t k) {
+  switch (k) {
+    case GK_COPY: case GK_SLOAD: case GK_SSTORE: case GK_RETV: return C_SINGLE;      // (ii)
+    case GK_FLOAD: case GK_FSTORE: case GK_ALOAD: case GK_ASTORE: return C_DOUBLE;   // (iii)
+    case GK_CALL: return C_CALL;
+    case GK_EXIT: return C_EXIT;
+    default: return C_ONETIME;                                                      // (i)
+  }
+}
+
+// Per-app bases of a batch.  Raw per-node arrays are concatenated app after app (node ids, method
+// ids, slot gids and node_ops stay app-local in them); row_ptr / call_arg_ptr slices hold n+1
+// entries each, so app k's start at node_base + k.
+struct __align__(16) DLApp {
+  uint64_t key_base;     // dense (module, field) table of the app: key_base + d * n_fields + f
+  uint64_t pair_base;    // dense (module, module) table: pair_base + sm * n_mods + dm
+  uint64_t n_edges;      // E of the app
+  uint32_t node_base, n_nodes, edge_base, arg_base, n_args;
+  uint32_t meth_base, n_meths, mod_base, n_mods;
+  uint32_t n_fields, n_inst;
+  uint32_t stat_lo, stat_hi; // app-local slot gids of the statics: [L_total, L_total + G)
+  uint32_t ptr_base;     // = node_base + k (row_ptr / call_arg_ptr slices)
+  uint32_t pad[2];
+};
+
+// Error word of the layout kernels: min over (app << 44 | node << 4 | code), code = -status.
+constexpr unsigned long long DL_NO_ERR = ~0ull;
+
+struct DLDev {
+  // uploaded descriptor arrays (app-local values)
+  const uint8_t* kind; const uint32_t* meth; const int32_t* ops;
+  const uint64_t* rp; const uint64_t* ap; const uint32_t* col; const uint8_t* ekind;
+  const int32_t* cargs; const uint32_t* mentry;
+  const DLApp* apps; uint32_t n_apps;
+  uint32_t N;
+  uint64_t K, P;                // entries of the dense key / pair tables of the batch
+  // scratch
+  uint32_t* words;              // [N] padded block words (scan input)
+  uint64_t* foff;               // [N+1] fact offsets (exclusive scan)
+  uint32_t* ksz; uint64_t* koff;  // [K] field-row table size (n_cols) of used keys, 0 else; offsets [K+1]
+  uint32_t* psz; uint64_t* poff;  // [P] projection table size of used module pairs, 0 else; [P+1]
+  uint32_t* cls;                // [NCLS] work items per class
+  unsigned long long* err;      // DL_NO_ERR or the first error
+  // uploaded per-method / per-module tables (batch-global indices)
+  const MethRec* meths; const ModRec* mods;
+  const uint32_t* col_gid; const int32_t* col_type; const uint32_t* col_hbase;
+  const uint32_t* grow_gid; const uint32_t* tf_ptr; const uint32_t* tf;
+  // outputs
+  NodeRec* nodes; uint32_t* nodemeth; uint32_t* rowptr; uint32_t* argptr; int32_t* args;
+  Edge* edges; InlEdge* inl; int32_t* frow; int32_t* xmap;
+};
+// phase 1: validate nodes / edges, block sizes, used keys and module pairs, class counts, scans
+cudaError_t launch_dl_sizes(const DLDev& L, uint64_t* scan_tmp, cudaStream_t s);
+// phase 2 (after the host allocated frow / xmap from the totals): records, tables, edges
+cudaError_t launch_dl_records(const DLDev& L, cudaStream_t s);
+
 int plain_max_blocks(int device);
 cudaError_t launch_plain(const PlainDev& P, uint32_t blocks, cudaStream_t s);
 cudaError_t launch_plain_digest(const PlainDev& P, cudaStream_t s);

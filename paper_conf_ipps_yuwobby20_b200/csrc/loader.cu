@@ -277,7 +277,10 @@ void scan_marks(const std::vector<uint8_t>& mark, F f) {
     if (mark[i]) f(i);
 }
 
-gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
+// dl = true (device layout, layout.cu): only the per-type / per-method / per-module part and the
+// O(1) CSR bounds run here; the per-node and per-edge passes (CSR checks, node pass, projection
+// tables, edge pass) are the layout kernels' work.
+gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k, bool dl = false) {
   if (!d) return set_err(GDROID_E_INVALID, "app %u: NULL descriptor", k);
   if (d->abi_version != GDROID_ABI_VERSION)
     return set_err(GDROID_E_INVALID, "app %u: abi_version %u != %u", k, d->abi_version, GDROID_ABI_VERSION);
@@ -286,12 +289,13 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   if (N == 0 || M == 0 || Dm == 0 || I == 0) return set_err(GDROID_E_INVALID, "app %u: empty ICFG", k);
   if (N >= (1ull << 32) || E >= (1ull << 32))
     return set_err(GDROID_E_LIMIT, "app %u: batch exceeds 2^32 nodes or edges", k);
-  H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
+  if (!dl) H.args.reserve(H.args.size() + d->call_arg_ptr[N]);
   const uint32_t nb = 0, mb = (uint32_t)H.meths.size();   // app-local node / method indices
   const uint32_t db = (uint32_t)H.mods.size(), tb = (uint32_t)(H.tf_ptr.size() - 1);
   // ---- CSR (structure)
   if (d->row_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: row_ptr[0] != 0", k);
-  {
+  if (dl && d->row_ptr[N] != E) return set_err(GDROID_E_INVALID, "app %u: row_ptr[n_nodes] != n_edges", k);
+  if (!dl) {
     FirstErr fc;                                             // parallel over ranges; lowest index wins
     parallel_ranges(N, 1 << 16, [&](uint64_t lo, uint64_t hi) {
       for (uint64_t n = lo; n < hi; ++n) {
@@ -428,6 +432,16 @@ gdroid_status add_app(HostImage& H, const gdroid_icfg_desc* d, uint32_t k) {
   // ---- nodes: operands -> rows (V1, V2, V4), fact offsets (parallel over node ranges)
   H.app_node_base.push_back(nb);
   if (d->call_arg_ptr[0] != 0) return set_err(GDROID_E_INVALID, "app %u: call_arg_ptr[0] != 0", k);
+  if (dl) {
+    H.n_nodes = N;
+    H.n_edges = E;
+    H.desc = d;
+    for (uint64_t i = 0; i < d->n_entries; ++i) {
+      if (d->entries[i] >= N || d->node_kind[d->entries[i]] != GK_ENTRY) return set_err(GDROID_E_INVALID, "app %u: entry %llu is not an ENTRY node", k, (unsigned long long)i);
+      H.entries.push_back(nb + d->entries[i]);
+    }
+    return GDROID_OK;
+  }
   // per range: call_arg_ptr monotone, fact-block sizes, (module, field) keys of heap accesses
   constexpr uint64_t RG = 1 << 15;
   const uint64_t n_rg = (N + RG - 1) / RG;
@@ -811,6 +825,7 @@ struct Layout {
   uint64_t fact_words = 0, N = 0, NC = 0, n_entries = 0, n_meths = 0;
   uint32_t cls_count[NCLS] = {0, 0, 0, 0, 0};
   uint32_t wide = 0;            // max logW over the modules
+  uint64_t n_edges = 0, n_args = 0, n_frow = 0, n_xmap = 0;   // table lengths (gdroid_debug_tables)
 };
 
 // Process-wide pinned staging buffer and per-app host images, reused by every load: in this
@@ -823,6 +838,13 @@ struct LoadCache {
   size_t cap_a = 0;
   bool pinned = false, pinned_a = false;
   std::vector<HostImage> img;
+  uint64_t* dl_tot = nullptr;    // pinned readback of the device layout's totals (DLTot words)
+  // device layout: per-device scratch for the raw descriptor arrays and the layout kernels'
+  // temporaries, grow-only and reused by every load (loads are serialised by mu and each one
+  // waits for its layout kernels), so it never churns the stream-ordered pool between the
+  // persistent tables and the fact stores
+  void* dl_raw[64] = {};
+  size_t dl_raw_cap[64] = {};
 };
 LoadCache g_cache;
 
@@ -922,6 +944,7 @@ gdroid_status build_image(const gdroid_icfg_desc* descs, uint32_t n_apps, Layout
   for (int c = 0; c < NCLS; ++c) nc += Lo.cls_count[c];
   if (nc >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
   Lo.N = T.node; Lo.NC = nc; Lo.n_entries = T.ent; Lo.fact_words = T.fact; Lo.n_meths = T.meth;
+  Lo.n_edges = T.edge; Lo.n_args = T.args; Lo.n_frow = T.frow; Lo.n_xmap = T.xmap;
   Lo.app_base.resize(n_apps + 1);
   for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
   const size_t bytes[NPART] = {
@@ -1073,6 +1096,8 @@ struct gdroid_app {
   std::vector<uint32_t> app_base;     // [n_apps+1] global node id ranges
   Dev D{};
   void* d_tables = nullptr;
+  void* d_tables2 = nullptr;          // device layout: field-row + projection tables (sized on the device)
+  uint64_t tab_len[9] = {};           // elements of each table (gdroid_debug_tables)
   uint64_t* d_facts = nullptr;        // nullptr after gdroid_release_facts (re-allocated by build)
   uint64_t fact_alloc_bytes = 0;
   void* d_state = nullptr;            // stamp, queue, counts, stats, bar, digests
@@ -1120,6 +1145,7 @@ void free_app(gdroid_app* a) {
   cudaGetDevice(&cur);
   cudaSetDevice(a->device);
   if (a->d_tables) cudaFreeAsync(a->d_tables, a->stream);
+  if (a->d_tables2) cudaFreeAsync(a->d_tables2, a->stream);
   if (a->d_facts) cudaFreeAsync(a->d_facts, a->stream);
   if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
   if (a->d_scratch) cudaFreeAsync(a->d_scratch, a->stream);
@@ -1199,6 +1225,274 @@ gdroid_status finish_stats(gdroid_app* a, gdroid_build_stats* out) {
   if (h.seed_err) return set_err(GDROID_E_POOL, "staged seed pair %llu is outside its node's pools (V1-V4)", (unsigned long long)(h.seed_err - 1));
   if (h.limit_hit) return set_err(GDROID_E_LIMIT, "max_rounds exceeded; facts are an under-approximation");
   return GDROID_OK;
+}
+
+
+// ---------------------------------------------------------------------------- device layout
+// (a1) with the per-node / per-edge passes on the device (layout.cu).  The host
+// validates and lays out the per-type / per-method / per-module tables of every app (add_app with
+// dl = true, apps in parallel), stages them plus the raw descriptor arrays in the pinned buffer
+// (parallel memcpy), uploads both, and the layout kernels do the rest.  One host round trip sizes
+// the field-row / projection tables.  *applicable = false: the batch's dense (module, field) or
+// (module, module) tables would be too large — the caller lays it out on the host instead.  A
+// validation error found on the device returns GDROID_E_STATE with *dev_err = the error word; the
+// caller re-runs the host validator for the exact status and message.
+enum DLPart { Q_METHS, Q_MODS, Q_COLGID, Q_COLTYPE, Q_COLHB, Q_GROWGID, Q_GROWCOL, Q_GROWFLD, Q_TFPTR, Q_TF,
+              Q_APPBASE, Q_ENTRIES, Q_UPLOAD,                                  // persistent, uploaded
+              Q_NODES = Q_UPLOAD, Q_NODEMETH, Q_ROWPTR, Q_ARGPTR, Q_ARGS, Q_EDGES, Q_INL, Q_NPART };
+enum DLRaw { W_KIND, W_METH, W_OPS, W_RP, W_AP, W_COL, W_EKIND, W_CARGS, W_MENTRY, W_APPS, W_UPLOAD,
+             W_WORDS = W_UPLOAD, W_FOFF, W_KSZ, W_KOFF, W_PSZ, W_POFF, W_SCAN, W_CLS, W_ERR, W_NPART };
+constexpr uint64_t DL_MAX_TABLE = 1ull << 27;   // dense key / pair table entries per batch
+
+gdroid_status load_dl(const gdroid_icfg_desc* descs, uint32_t n_apps, gdroid_app* a, Layout& Lo, bool* applicable,
+                      unsigned long long* dev_err) {
+  *applicable = true;
+  *dev_err = DL_NO_ERR;
+  if (g_cache.img.size() < n_apps) g_cache.img.resize(n_apps);
+  std::vector<HostImage>& img = g_cache.img;
+  std::vector<gdroid_status> st(n_apps, GDROID_OK);
+  std::vector<std::string> err(n_apps);
+  PhaseTimer* pt_saved = g_pt;
+  g_pt = nullptr;
+  parallel_for(n_apps, [&](uint32_t k) {
+    reset_image(img[k]);
+    st[k] = add_app(img[k], &descs[k], k, true);
+    if (st[k] != GDROID_OK) err[k] = g_err;
+  });
+  g_pt = pt_saved;
+  for (uint32_t k = 0; k < n_apps; ++k)
+    if (st[k] != GDROID_OK) { g_err = err[k]; return st[k]; }
+  PHASE("apps (per-module tables)");
+  struct Base { uint64_t node, edge, args, meth, mod, col, grow, type, tf, ent, key, pair; };
+  std::vector<Base> b(n_apps + 1);
+  b[0] = Base{};
+  uint32_t wide = 0;
+  for (uint32_t k = 0; k < n_apps; ++k) {
+    const HostImage& h = img[k];
+    const gdroid_icfg_desc& d = descs[k];
+    b[k + 1] = Base{b[k].node + d.n_nodes, b[k].edge + d.n_edges, b[k].args + d.call_arg_ptr[d.n_nodes],
+                    b[k].meth + h.meths.size(), b[k].mod + h.mods.size(), b[k].col + h.col_gid.size(),
+                    b[k].grow + h.grow_gid.size(), b[k].type + (h.tf_ptr.size() - 1), b[k].tf + h.tf.size(),
+                    b[k].ent + h.entries.size(), b[k].key + (uint64_t)d.n_modules * d.n_fields,
+                    b[k].pair + (uint64_t)d.n_modules * d.n_modules};
+    for (const ModRec& md : h.mods) wide = std::max<uint32_t>(wide, md.logW);
+  }
+  const Base& T = b[n_apps];
+  if (T.node >= (1ull << 27)) return set_err(GDROID_E_LIMIT, "batch exceeds 2^27 nodes");
+  if (T.edge >= (1ull << 32) || T.args >= (1ull << 32)) return set_err(GDROID_E_LIMIT, "batch tables exceed 32-bit indices");
+  if (T.key > DL_MAX_TABLE || T.pair > DL_MAX_TABLE) { *applicable = false; return GDROID_OK; }
+  const uint64_t N = T.node, E = T.edge;
+  // ---- device layout: persistent tables (A) and temporary inputs + scratch (R)
+  const size_t qbytes[Q_NPART] = {
+      T.meth * sizeof(MethRec), T.mod * sizeof(ModRec), T.col * 4, T.col * 4, T.col * 4, T.grow * 4, T.grow * 4,
+      T.grow * 4, (T.type + 1) * 4, std::max<uint64_t>(T.tf, 1) * 4, (n_apps + 1) * 4, std::max<uint64_t>(T.ent, 1) * 4,
+      N * sizeof(NodeRec), N * 4, (N + 1) * 4, (N + 1) * 4, std::max<uint64_t>(T.args, 1) * 4,
+      std::max<uint64_t>(E, 1) * sizeof(Edge), N * 4 * sizeof(InlEdge)};
+  size_t qoff[Q_NPART + 1];
+  qoff[0] = 0;
+  for (int p = 0; p < Q_NPART; ++p) qoff[p + 1] = qoff[p] + align256(qbytes[p]);
+  const uint64_t scan_n = std::max<uint64_t>(std::max<uint64_t>(N, T.key), T.pair);
+  const size_t wbytes[W_NPART] = {
+      N, N * 4, N * 16, (N + n_apps) * 8, (N + n_apps) * 8, std::max<uint64_t>(E, 1) * 4, std::max<uint64_t>(E, 1),
+      std::max<uint64_t>(T.args, 1) * 4, std::max<uint64_t>(T.meth, 1) * 4, n_apps * sizeof(DLApp),
+      N * 4, (N + 1) * 8, std::max<uint64_t>(T.key, 1) * 4, (T.key + 1) * 8, std::max<uint64_t>(T.pair, 1) * 4,
+      (T.pair + 1) * 8, scan_tmp_words((uint32_t)scan_n) * 8, 256, 8};
+  size_t woff[W_NPART + 1];
+  woff[0] = 0;
+  for (int p = 0; p < W_NPART; ++p) woff[p + 1] = woff[p] + align256(wbytes[p]);
+  const size_t up_a = qoff[Q_UPLOAD], up_r = woff[W_UPLOAD];
+  gdroid_status s2 = ensure_pinned(g_cache.stage, g_cache.cap, g_cache.pinned, up_a + up_r, "device-layout inputs");
+  if (s2 != GDROID_OK) return s2;
+  if (!g_cache.dl_tot && cudaMallocHost(&g_cache.dl_tot, 16 * 8) != cudaSuccess) {
+    g_cache.dl_tot = nullptr;
+    return set_err(GDROID_E_OOM, "pinned device-layout totals");
+  }
+  char* SA = (char*)g_cache.stage;
+  char* SR = SA + up_a;
+  MethRec* g_meths = (MethRec*)(SA + qoff[Q_METHS]);
+  ModRec* g_mods = (ModRec*)(SA + qoff[Q_MODS]);
+  uint32_t* g_colgid = (uint32_t*)(SA + qoff[Q_COLGID]);
+  int32_t* g_coltype = (int32_t*)(SA + qoff[Q_COLTYPE]);
+  uint32_t* g_colhb = (uint32_t*)(SA + qoff[Q_COLHB]);
+  uint32_t* g_growgid = (uint32_t*)(SA + qoff[Q_GROWGID]);
+  int32_t* g_growcol = (int32_t*)(SA + qoff[Q_GROWCOL]);
+  int32_t* g_growfld = (int32_t*)(SA + qoff[Q_GROWFLD]);
+  uint32_t* g_tfptr = (uint32_t*)(SA + qoff[Q_TFPTR]);
+  uint32_t* g_tf = (uint32_t*)(SA + qoff[Q_TF]);
+  uint32_t* g_appbase = (uint32_t*)(SA + qoff[Q_APPBASE]);
+  uint32_t* g_entries = (uint32_t*)(SA + qoff[Q_ENTRIES]);
+  DLApp* g_apps = (DLApp*)(SR + woff[W_APPS]);
+  g_tfptr[0] = 0; g_tf[0] = 0; g_entries[0] = 0;
+  for (uint32_t k = 0; k <= n_apps; ++k) g_appbase[k] = (uint32_t)b[k].node;
+  for (uint32_t k = 0; k < n_apps; ++k) {
+    const gdroid_icfg_desc& d = descs[k];
+    const HostImage& h = img[k];
+    const uint64_t Lt = h.meths.empty() ? 0 : (uint64_t)h.meths.back().local_base + h.meths.back().n_locals;
+    DLApp A{};
+    A.key_base = b[k].key; A.pair_base = b[k].pair; A.n_edges = d.n_edges;
+    A.node_base = (uint32_t)b[k].node; A.n_nodes = d.n_nodes; A.edge_base = (uint32_t)b[k].edge;
+    A.arg_base = (uint32_t)b[k].args; A.n_args = (uint32_t)d.call_arg_ptr[d.n_nodes];
+    A.meth_base = (uint32_t)b[k].meth; A.n_meths = d.n_methods; A.mod_base = (uint32_t)b[k].mod; A.n_mods = d.n_modules;
+    A.n_fields = d.n_fields; A.n_inst = d.n_instances;
+    A.stat_lo = (uint32_t)Lt; A.stat_hi = (uint32_t)(Lt + d.n_statics);
+    A.ptr_base = (uint32_t)(b[k].node + k);
+    g_apps[k] = A;
+  }
+  // work units: each app's per-module tables (rebased to batch indices) and slices of its raw
+  // per-node / per-edge arrays (plain copies: the values stay app-local)
+  constexpr uint64_t SLICE = 1 << 18;
+  struct Unit { uint32_t k, part; uint64_t lo, hi; };
+  std::vector<Unit> units;
+  for (uint32_t k = 0; k < n_apps; ++k) {
+    const gdroid_icfg_desc& d = descs[k];
+    units.push_back({k, 99u, 0, 0});
+    auto add = [&](uint32_t part, uint64_t n) { for (uint64_t lo = 0; lo < n; lo += SLICE) units.push_back({k, part, lo, std::min(n, lo + SLICE)}); };
+    add(W_KIND, d.n_nodes); add(W_METH, d.n_nodes); add(W_OPS, d.n_nodes); add(W_RP, d.n_nodes + 1ull);
+    add(W_AP, d.n_nodes + 1ull); add(W_COL, d.n_edges); add(W_EKIND, d.n_edges); add(W_CARGS, d.call_arg_ptr[d.n_nodes]);
+    add(W_MENTRY, d.n_methods);
+  }
+  parallel_for((uint32_t)units.size(), [&](uint32_t u) {
+    const Unit U = units[u];
+    const HostImage& h = img[U.k];
+    const gdroid_icfg_desc& d = descs[U.k];
+    const Base& B = b[U.k];
+    const uint64_t lo = U.lo, n = U.hi - U.lo;
+    switch (U.part) {
+      case W_KIND: std::memcpy(SR + woff[W_KIND] + B.node + lo, d.node_kind + lo, n); return;
+      case W_METH: std::memcpy(SR + woff[W_METH] + 4 * (B.node + lo), d.node_method + lo, 4 * n); return;
+      case W_OPS: std::memcpy(SR + woff[W_OPS] + 16 * (B.node + lo), d.node_ops + 4 * lo, 16 * n); return;
+      case W_RP: std::memcpy(SR + woff[W_RP] + 8 * (B.node + U.k + lo), d.row_ptr + lo, 8 * n); return;
+      case W_AP: std::memcpy(SR + woff[W_AP] + 8 * (B.node + U.k + lo), d.call_arg_ptr + lo, 8 * n); return;
+      case W_COL: std::memcpy(SR + woff[W_COL] + 4 * (B.edge + lo), d.col + lo, 4 * n); return;
+      case W_EKIND: std::memcpy(SR + woff[W_EKIND] + B.edge + lo, d.edge_kind + lo, n); return;
+      case W_CARGS: std::memcpy(SR + woff[W_CARGS] + 4 * (B.args + lo), d.call_args + lo, 4 * n); return;
+      case W_MENTRY: std::memcpy(SR + woff[W_MENTRY] + 4 * (B.meth + lo), d.method_entry + lo, 4 * n); return;
+      default: break;
+    }
+    for (size_t i = 0; i < h.meths.size(); ++i) { MethRec M = h.meths[i]; M.module += (uint32_t)B.mod; g_meths[B.meth + i] = M; }
+    for (size_t i = 0; i < h.mods.size(); ++i) {
+      ModRec D = h.mods[i]; D.col_off += (uint32_t)B.col; D.grow_off += (uint32_t)B.grow; g_mods[B.mod + i] = D;
+    }
+    for (size_t i = 0; i < h.col_gid.size(); ++i) {
+      g_colgid[B.col + i] = h.col_gid[i];
+      g_coltype[B.col + i] = h.col_type[i] < 0 ? -1 : h.col_type[i] + (int32_t)B.type;
+      g_colhb[B.col + i] = h.col_hbase[i];
+    }
+    std::copy(h.grow_gid.begin(), h.grow_gid.end(), g_growgid + B.grow);
+    std::copy(h.grow_col.begin(), h.grow_col.end(), g_growcol + B.grow);
+    std::copy(h.grow_field.begin(), h.grow_field.end(), g_growfld + B.grow);
+    for (size_t i = 1; i < h.tf_ptr.size(); ++i) g_tfptr[B.type + i] = h.tf_ptr[i] + (uint32_t)B.tf;
+    std::copy(h.tf.begin(), h.tf.end(), g_tf + B.tf);
+    for (size_t i = 0; i < h.entries.size(); ++i) g_entries[B.ent + i] = h.entries[i] + (uint32_t)B.node;
+  });
+  PHASE("staging");
+  // ---- upload, phase 1 (sizes), one round trip
+  const auto t0 = std::chrono::steady_clock::now();
+  if (a->device < 0 || a->device >= 64) return set_err(GDROID_E_INVALID, "device %d", a->device);
+  void*& d_raw = g_cache.dl_raw[a->device];
+  size_t& raw_cap = g_cache.dl_raw_cap[a->device];
+  if (raw_cap < woff[W_NPART]) {
+    if (d_raw) { CU(cudaFree(d_raw)); d_raw = nullptr; raw_cap = 0; }
+    const size_t want = woff[W_NPART] + (woff[W_NPART] >> 2);
+    CU(cudaMalloc(&d_raw, want));
+    raw_cap = want;
+  }
+  CU(cudaMallocAsync(&a->d_tables, qoff[Q_NPART], a->stream));
+  char* DA = (char*)a->d_tables;
+  char* DR = (char*)d_raw;
+  CU(cudaMemcpyAsync(DA, SA, up_a, cudaMemcpyHostToDevice, a->stream));
+  CU(cudaMemcpyAsync(DR, SR, up_r, cudaMemcpyHostToDevice, a->stream));
+  CU(cudaMemsetAsync(DR + woff[W_KSZ], 0, wbytes[W_KSZ], a->stream));
+  CU(cudaMemsetAsync(DR + woff[W_PSZ], 0, wbytes[W_PSZ], a->stream));
+  CU(cudaMemsetAsync(DR + woff[W_CLS], 0, 256, a->stream));
+  CU(cudaMemsetAsync(DR + woff[W_ERR], 0xff, 8, a->stream));
+  DLDev L{};
+  L.kind = (const uint8_t*)(DR + woff[W_KIND]); L.meth = (const uint32_t*)(DR + woff[W_METH]);
+  L.ops = (const int32_t*)(DR + woff[W_OPS]); L.rp = (const uint64_t*)(DR + woff[W_RP]);
+  L.ap = (const uint64_t*)(DR + woff[W_AP]); L.col = (const uint32_t*)(DR + woff[W_COL]);
+  L.ekind = (const uint8_t*)(DR + woff[W_EKIND]); L.cargs = (const int32_t*)(DR + woff[W_CARGS]);
+  L.mentry = (const uint32_t*)(DR + woff[W_MENTRY]); L.apps = (const DLApp*)(DR + woff[W_APPS]);
+  L.n_apps = n_apps; L.N = (uint32_t)N; L.K = T.key; L.P = T.pair;
+  L.words = (uint32_t*)(DR + woff[W_WORDS]); L.foff = (uint64_t*)(DR + woff[W_FOFF]);
+  L.ksz = (uint32_t*)(DR + woff[W_KSZ]); L.koff = (uint64_t*)(DR + woff[W_KOFF]);
+  L.psz = (uint32_t*)(DR + woff[W_PSZ]); L.poff = (uint64_t*)(DR + woff[W_POFF]);
+  L.cls = (uint32_t*)(DR + woff[W_CLS]); L.err = (unsigned long long*)(DR + woff[W_ERR]);
+  L.meths = (const MethRec*)(DA + qoff[Q_METHS]); L.mods = (const ModRec*)(DA + qoff[Q_MODS]);
+  L.col_gid = (const uint32_t*)(DA + qoff[Q_COLGID]); L.col_type = (const int32_t*)(DA + qoff[Q_COLTYPE]);
+  L.col_hbase = (const uint32_t*)(DA + qoff[Q_COLHB]); L.grow_gid = (const uint32_t*)(DA + qoff[Q_GROWGID]);
+  L.tf_ptr = (const uint32_t*)(DA + qoff[Q_TFPTR]); L.tf = (const uint32_t*)(DA + qoff[Q_TF]);
+  L.nodes = (NodeRec*)(DA + qoff[Q_NODES]); L.nodemeth = (uint32_t*)(DA + qoff[Q_NODEMETH]);
+  L.rowptr = (uint32_t*)(DA + qoff[Q_ROWPTR]); L.argptr = (uint32_t*)(DA + qoff[Q_ARGPTR]);
+  L.args = (int32_t*)(DA + qoff[Q_ARGS]); L.edges = (Edge*)(DA + qoff[Q_EDGES]); L.inl = (InlEdge*)(DA + qoff[Q_INL]);
+  cudaError_t e = launch_dl_sizes(L, (uint64_t*)(DR + woff[W_SCAN]), a->stream);
+  if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout kernels (sizes): %s", cudaGetErrorString(e));
+  uint64_t* tot = g_cache.dl_tot;                      // [0] fact words [1] frow [2] xmap [3] err [4..8] classes
+  CU(cudaMemcpyAsync(tot + 0, L.foff + N, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaMemcpyAsync(tot + 1, L.koff + T.key, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaMemcpyAsync(tot + 2, L.poff + T.pair, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaMemcpyAsync(tot + 3, L.err, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaMemcpyAsync(tot + 4, L.cls, NCLS * 4, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  a->h2d_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
+  PHASE("upload + layout sizes");
+  if (tot[3] != DL_NO_ERR) { *dev_err = tot[3]; return GDROID_E_STATE; }
+  const uint64_t fact_words = tot[0], n_frow = tot[1], n_xmap = tot[2];
+  uint32_t cls_count[NCLS];
+  std::memcpy(cls_count, tot + 4, NCLS * 4);
+  uint64_t nc = 0;
+  for (int c = 0; c < NCLS; ++c) nc += cls_count[c];
+  if (nc >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
+  if (n_xmap >= (1ull << 32) || n_frow >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "batch tables exceed 32-bit indices");
+  // ---- field-row + projection tables, phase 2
+  const size_t fb = align256(std::max<uint64_t>(n_frow, 1) * 4), xb = align256(std::max<uint64_t>(n_xmap, 1) * 4);
+  CU(cudaMallocAsync(&a->d_tables2, fb + xb, a->stream));
+  L.frow = (int32_t*)a->d_tables2;
+  L.xmap = (int32_t*)((char*)a->d_tables2 + fb);
+  e = launch_dl_records(L, a->stream);
+  if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout kernels (records): %s", cudaGetErrorString(e));
+  CU(cudaMemcpyAsync(tot + 3, L.err, 8, cudaMemcpyDeviceToHost, a->stream));
+  CU(cudaStreamSynchronize(a->stream));
+  PHASE("layout records");
+  if (tot[3] != DL_NO_ERR) { *dev_err = tot[3]; return GDROID_E_STATE; }
+  // ---- the handle's view
+  Lo.N = N; Lo.NC = nc; Lo.n_entries = T.ent; Lo.fact_words = fact_words; Lo.n_meths = T.meth; Lo.wide = wide;
+  Lo.n_edges = E; Lo.n_args = T.args; Lo.n_frow = n_frow; Lo.n_xmap = n_xmap;
+  for (int c = 0; c < NCLS; ++c) Lo.cls_count[c] = cls_count[c];
+  Lo.app_base.resize(n_apps + 1);
+  for (uint32_t k = 0; k <= n_apps; ++k) Lo.app_base[k] = (uint32_t)b[k].node;
+  Dev& D = a->D;
+  D.nodes = L.nodes; D.meths = L.meths; D.mods = L.mods; D.row_ptr = L.rowptr; D.edges = L.edges;
+  D.arg_ptr = L.argptr; D.args = L.args; D.col_gid = L.col_gid; D.col_type = L.col_type; D.col_hbase = L.col_hbase;
+  D.grow_gid = L.grow_gid; D.grow_col = (const int32_t*)(DA + qoff[Q_GROWCOL]);
+  D.grow_field = (const int32_t*)(DA + qoff[Q_GROWFLD]); D.tf_ptr = L.tf_ptr; D.tf = L.tf; D.xmap = L.xmap;
+  D.app_node_base = (const uint32_t*)(DA + qoff[Q_APPBASE]); D.entries = (const uint32_t*)(DA + qoff[Q_ENTRIES]);
+  D.node_method = L.nodemeth; D.frow = L.frow; D.inl = L.inl;
+  return GDROID_OK;
+}
+
+// A validation error found by the layout kernels: the host validator (the host layout path)
+// re-runs on the batch for the exact status and message of the first offending index.
+// GDROID_DL_DEVICE_ERRORS=1 reports the device's own finding instead (tests of the kernels' checks).
+gdroid_status dl_error(const gdroid_icfg_desc* descs, uint32_t n_apps, unsigned long long w) {
+  const uint32_t k = (uint32_t)(w >> 44);
+  const unsigned long long idx = (w >> 4) & ((1ull << 40) - 1);
+  const int code = (int)(w & 15);
+  if (!getenv("GDROID_DL_DEVICE_ERRORS")) {
+    Layout L2;
+    const gdroid_status st = build_image(descs, n_apps, L2, [](const Layout&) { return GDROID_OK; });
+    if (st != GDROID_OK) return st;
+  }
+  return set_err((gdroid_status)(-code), "app %u: index %llu: %s (device layout validation)", k, idx,
+                 code == 2 ? "pool closure violated (V1-V4)" : code == 8 ? "size limit" : "invalid structure (CSR, kinds, V5, V6)");
+}
+
+// Device layout unless GDROID_HOST_LAYOUT is set or there is no device (CPU-only hosts run the
+// host validator, then fail at the upload).
+bool use_device_layout() {
+  if (getenv("GDROID_HOST_LAYOUT")) return false;
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess) { cudaGetLastError(); return false; }
+  return n > 0;
 }
 
 // ---------------------------------------------------------------------------------- PLAIN
@@ -1440,7 +1734,17 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   }
   Layout Lo;
   auto t0 = std::chrono::steady_clock::now();
-  {
+  bool dl_done = false;
+  if (use_device_layout()) {
+    std::lock_guard<std::mutex> lock(g_cache.mu);
+    bool applicable = true;
+    unsigned long long derr = DL_NO_ERR;
+    const gdroid_status st = load_dl(descs, n_apps, a, Lo, &applicable, &derr);
+    if (st == GDROID_E_STATE && derr != DL_NO_ERR) return fail(dl_error(descs, n_apps, derr));
+    if (st != GDROID_OK) return fail(st);
+    dl_done = applicable;
+  }
+  if (!dl_done) {
     std::lock_guard<std::mutex> lock(g_cache.mu);
     gdroid_status st = build_image(descs, n_apps, Lo, [&](const Layout& L) -> gdroid_status {
       cudaError_t e = cudaMallocAsync(&a->d_tables, L.total, a->stream);
@@ -1458,12 +1762,18 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     cudaError_t e2 = cudaStreamSynchronize(a->stream);
     if (e != cudaSuccess || e2 != cudaSuccess) return fail(set_err(GDROID_E_CUDA, "H2D upload: %s", cudaGetErrorString(e != cudaSuccess ? e : e2)));
   }
-  a->h2d_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
-  PHASE("upload");
+  if (!dl_done) {
+    a->h2d_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
+    PHASE("upload");
+  }
   a->app_base = Lo.app_base;
+  a->tab_len[0] = Lo.N; a->tab_len[1] = Lo.n_edges; a->tab_len[2] = 4 * Lo.N; a->tab_len[3] = Lo.n_frow;
+  a->tab_len[4] = Lo.n_xmap; a->tab_len[5] = Lo.n_args; a->tab_len[6] = Lo.N + 1; a->tab_len[7] = Lo.N + 1;
+  a->tab_len[8] = Lo.N;
   const uint32_t N = (uint32_t)Lo.N, NC = (uint32_t)Lo.NC;
   char* T = (char*)a->d_tables;
   Dev& D = a->D;
+  if (!dl_done) {
   D.nodes = (const NodeRec*)(T + Lo.off[P_NODES]);
   D.meths = (const MethRec*)(T + Lo.off[P_METHS]);
   D.mods = (const ModRec*)(T + Lo.off[P_MODS]);
@@ -1485,6 +1795,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.node_method = (const uint32_t*)(T + Lo.off[P_NODEMETH]);
   D.frow = (const int32_t*)(T + Lo.off[P_FROW]);
   D.inl = (const InlEdge*)(T + Lo.off[P_INL]);
+  }
   D.n_nodes = N;
   D.n_chunks = NC;
   D.n_entries = (uint32_t)Lo.n_entries;
@@ -1494,7 +1805,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   D.n_words = Lo.fact_words;
   D.wide = Lo.wide;
   D.n_meths = (uint32_t)Lo.n_meths;
-  {
+  if (!dl_done) {
     // (a1) per-app bases added to the staged app-local node tables, then the edge records and
     // inline chunk-0 edges derived from col / edge_kind / projection offsets and the NodeRecs
     // (stream-ordered after the upload)
@@ -2068,6 +2379,21 @@ void gdroid_free(gdroid_app* a) { free_app(a); }
 gdroid_status gdroid_debug_phases(const gdroid_app* a, uint64_t* out8) {
   if (!a || !out8) return set_err(GDROID_E_INVALID, "NULL argument");
   for (int i = 0; i < 8; ++i) out8[i] = a->h_stats->phase[i];
+  return GDROID_OK;
+}
+
+gdroid_status gdroid_debug_tables(const gdroid_app* a, uint32_t which, void* host, uint64_t cap, uint64_t* bytes) {
+  if (!a || !bytes) return set_err(GDROID_E_INVALID, "NULL argument");
+  if (which > 8) return set_err(GDROID_E_RANGE, "table %u", which);
+  const Dev& D = a->D;
+  const void* src[9] = {D.nodes, D.edges, D.inl, D.frow, D.xmap, D.args, D.row_ptr, D.arg_ptr, D.node_method};
+  const uint64_t esz[9] = {sizeof(NodeRec), sizeof(Edge), sizeof(InlEdge), 4, 4, 4, 4, 4, 4};
+  *bytes = a->tab_len[which] * esz[which];
+  if (!host) return GDROID_OK;
+  if (cap < *bytes) return set_err(GDROID_E_SMALLBUF, "need %llu bytes", (unsigned long long)*bytes);
+  DeviceGuard guard(a->device);
+  CU(cudaStreamSynchronize(a->stream));
+  if (*bytes) CU(cudaMemcpy(host, src[which], *bytes, cudaMemcpyDeviceToHost));
   return GDROID_OK;
 }
 
