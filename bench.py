@@ -443,9 +443,11 @@ def run_ours(args):
         line["e2e"] = {"value": total_apps / (e2e["ms"] / 1e3), "unit": "apps/s",
                        "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
                        "ms_per_step": e2e["ms"], "readback": args.e2e_readback,
-                       "pipeline": "loader thread: host tables + pinned H2D of batch i+1 overlapped with the "
-                                   "build of batch i; gdroid_read_batch_facts of batch i (pinned) overlapped "
-                                   "with the build of batch i+1; one untimed warm-up pass sizes the buffers"}
+                       "pipeline": "loader thread: gdroid_load_batch of batch i+1 (per-module host tables, raw "
+                                   "descriptor arrays staged in pinned memory and uploaded, node/edge layout "
+                                   "kernels, DESIGN.md §4.1) overlapped with the build of batch i; "
+                                   "gdroid_read_batch_facts_async of batch i (pinned) overlapped with the build "
+                                   "of batch i+1; one untimed warm-up pass sizes the buffers"}
     if not args.no_per_config and args.workload == "corpus1000":
         line["per_config"] = per_config_runs(local, stream.cuda_stream)
     if not args.no_cpu_baseline:

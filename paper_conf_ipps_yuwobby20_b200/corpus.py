@@ -331,6 +331,7 @@ def run_pipelined(batches: List[List[int]], make_app: Callable[[int], object], d
                 apps = [make_app(i) for i in b]
                 t0 = time.perf_counter()
                 h = gd.load(apps, device=device, stream=streams[j % 2].cuda_stream)
+                h.release_facts()          # the build allocates it: two fact stores live, not three
                 q.put((b, h, (time.perf_counter() - t0) * 1e3, [a.n_nodes for a in apps],
                        sum(a.nbytes() for a in apps)))
         except BaseException as e:                         # surface it in the consumer

@@ -316,6 +316,8 @@ struct DLDev {
 cudaError_t launch_dl_sizes(const DLDev& L, uint64_t* scan_tmp, cudaStream_t s);
 // phase 2 (after the host allocated frow / xmap from the totals): records, tables, edges
 cudaError_t launch_dl_records(const DLDev& L, cudaStream_t s);
+// totals + error word into mapped pinned host memory (no copy-engine round trip)
+cudaError_t launch_dl_totals(const DLDev& L, uint64_t* host_mapped, cudaStream_t s);
 
 int plain_max_blocks(int device);
 cudaError_t launch_plain(const PlainDev& P, uint32_t blocks, cudaStream_t s);

@@ -107,6 +107,12 @@ struct CtaStage {              // per-CTA staged worklist appends of the current
   unsigned long long lid;      // local round id (pass << 32 | counter): dedupe key in D.lstamp
 };
 constexpr uint32_t LQCAP = 1024;
+#ifndef GD_CONT_STAMP
+#define GD_CONT_STAMP 1
+#endif
+#ifndef GD_CONT_PF
+#define GD_CONT_PF 1         // light rounds: prefetch the inline successors' records into L1
+#endif
 constexpr uint32_t LQ_SKIP = 0xffffffffu;
 
 // fire-and-forget 64-bit OR at L2 (RED; no return value, no scoreboard wait)
@@ -161,8 +167,11 @@ __device__ __forceinline__ void stage_init(CtaStage& st) {
 // single-chunk destination (not queued for this round or the next) wants a visit may instead hand it back to the
 // warp, which processes it at once in this round (a depth-first step).  That lane
 // does not queue it: the warp reads IN(dst) after its own ORs, and a later grower of dst sees a
-// stamp below round+1 and queues dst as usual, so no growth is lost.  cont[dst] == round keeps
-// a second warp from continuing into the same node in the same round (it queues it instead).
+// stamp below round+1 and queues dst as usual, so no growth is lost.  The claim is one
+// atomicMax(stamp[dst], round) returning a value below round: it keeps a second warp from
+// continuing into the same node in the same round (it queues it instead) and a node already
+// queued for this round or the next from being continued into (GD_CONT_STAMP; the round-2 claim
+// was a stamp load, an atomicExch on cont[dst] and the atomicMax: three dependent L2 hops).
 template <bool SB = false>
 __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lane, bool active,
                                              uint32_t dst, uint32_t info, bool grew, uint32_t round,
@@ -199,7 +208,30 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
       }
     }
   }
+  bool decided = false;                                     // pushes already decided below
   if (cont && *cont == NO_CONT && (D.flags & F_CONT)) {
+#if GD_CONT_STAMP
+    // One memory hop for every wanting lane: the candidate claims the continuation with
+    // atomicMax(stamp[dst], round) — below round before: not queued for this round or the next,
+    // not continued into by another warp this round — while the other lanes queue theirs for the
+    // next round (stamp -> round + 1) with the same instruction.  The stamp loaded with the item's
+    // first hop (sv, possibly stale: stamps only grow) picks the candidate.
+    const unsigned cand = __ballot_sync(FULL, want && sv < round && (cont_dense || (info & INFO_WIDE)) &&
+                                                  ((info >> 5) & 31u) == 0);
+    const int l = cand ? __ffs(cand) - 1 : -1;
+    const bool issue = active && want && (lane == l || sv != round + 1);
+    uint32_t old = 0;
+    if (issue) old = atomicMax(&D.stamp[dst], lane == l ? round : round + 1);
+    uint32_t ok = 0;
+    if (lane == l) {
+      if (old < round) { ok = 1; want = false; }
+      else if (old == round) push = atomicMax(&D.stamp[dst], round + 1) < round + 1;   // rare: queue it
+    } else if (issue) {
+      push = old < round + 1;
+    }
+    decided = true;
+    if (l >= 0 && __shfl_sync(FULL, ok, l)) *cont = __shfl_sync(FULL, dst, l);
+#else
     const unsigned cand = __ballot_sync(FULL, want && (cont_dense || (info & INFO_WIDE)) && ((info >> 5) & 31u) == 0);
     if (cand) {
       const int l = __ffs(cand) - 1;
@@ -211,8 +243,9 @@ __device__ __forceinline__ void flush_pushes(const Dev& D, CtaStage& st, int lan
       }
       if (__shfl_sync(FULL, ok, l)) *cont = __shfl_sync(FULL, dst, l);
     }
+#endif
   }
-  if (active) {
+  if (active && !decided) {
     // sv == round + 1: already queued for the next round (stamps never exceed round + 1 during
     // round `round`, and a stale value is never larger than the true one) — no atomic needed
     if (want && sv != round + 1) {
@@ -648,6 +681,10 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     }
   }
   const uint32_t my_stamp = lane < (int)ne ? D.stamp[me.dst] : 1u;
+  if (GD_CONT_PF && CD && cont_ok && lane < (int)ne) {       // a continuation's first hop hits L1
+    asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.nodes + me.dst)));
+    asm volatile("prefetch.global.L1 [%0];" :: "l"((const char*)(D.inl + 4 * me.dst)));
+  }
   const bool dbl = kind == GK_FLOAD || kind == GK_ALOAD || kind == GK_FSTORE || kind == GK_ASTORE;
   int hr[2] = {-1, -1};                                     // heap rows of this lane's columns
   if (dbl) {

@@ -275,88 +275,177 @@ __global__ void __launch_bounds__(256) k_dl_xmap(DLDev L) {
   }
 }
 
-// V5 / V6 of every out-edge, Edge records (destination layout copied in; CALL aux = the callee's
-// n_params, RET aux = lhs(c) row at the return site), and chunk 0 inline when it holds only
-// INTRA / C2R edges of a narrow block of <= INL_MAX_B words (as k_edges of kernels.cu).
-__global__ void __launch_bounds__(256) k_dl_edges(DLDev L) {
+// V5 / V6 of out-edge el of node n (app-local i), and its Edge record (destination layout copied
+// in; CALL aux = the callee's n_params, RET aux = lhs(c) row at the return site).  Returns 0 or the
+// error code.
+struct EdgeCtx {
+  uint32_t n, i, kind, lm, sm, my_entry;
+  uint64_t a0, a1;
+};
+__device__ __forceinline__ unsigned long long dl_edge(const DLDev& L, const DLApp& A, const EdgeCtx& c, uint64_t el,
+                                                      uint32_t& ek_out, Edge& E2) {
+  const uint64_t e = A.edge_base + el;
+  const uint32_t sl = L.col[e], ek = L.ekind[e];
+  ek_out = ek;
+  if (sl >= A.n_nodes || ek > GE_C2R) return ERR_INVALID;
+  const uint32_t s = A.node_base + sl, skind = L.kind[s], tm = L.meth[s];
+  if (tm >= A.n_meths) return ERR_INVALID;
+  bool ok = true;
+  switch (ek) {
+    case GE_INTRA: ok = c.kind != GK_CALL && c.kind != GK_EXIT && tm == c.lm; break;
+    case GE_C2R: ok = c.kind == GK_CALL && skind == GK_RETSITE && L.ops[4ull * s + 3] == (int32_t)c.i; break;
+    case GE_CALL:                                              // V5 + V6 (arity)
+      ok = c.kind == GK_CALL && skind == GK_ENTRY && L.mentry[A.meth_base + tm] == sl &&
+           c.a1 - c.a0 == L.meths[A.meth_base + tm].n_params;
+      break;
+    case GE_RET: {                                             // to a site that calls this method
+      ok = c.kind == GK_EXIT && skind == GK_RETSITE;
+      const int32_t cs = ok ? L.ops[4ull * s + 3] : -1;
+      if (ok && (cs < 0 || (uint32_t)cs >= A.n_nodes)) ok = false;
+      if (ok) {
+        const uint64_t c0 = L.rp[A.ptr_base + cs], c1 = L.rp[A.ptr_base + cs + 1];
+        bool found = false;
+        if (c1 >= c0 && c1 <= A.n_edges)
+          for (uint64_t e2 = c0; e2 < c1 && !found; ++e2)
+            found = L.ekind[A.edge_base + e2] == GE_CALL && L.col[A.edge_base + e2] == c.my_entry;
+        ok = found;
+      }
+      break;
+    }
+  }
+  if (!ok) return ERR_INVALID;
+  uint32_t xoff = NO_XMAP;
+  if (ek == GE_CALL || ek == GE_RET) {
+    const uint32_t dm = L.meths[A.meth_base + tm].module;
+    if (dm != c.sm) xoff = (uint32_t)L.poff[A.pair_base + (uint64_t)(c.sm - A.mod_base) * A.n_mods + (dm - A.mod_base)];
+  }
+  const NodeRec RS = L.nodes[s];
+  const uint32_t nch = n_chunks_of(RS.e1 - RS.e0, RS.cls, RS.logW);
+  E2.dst = s;
+  E2.info = ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5) | (RS.logW >= 1 ? INFO_WIDE : 0u);
+  E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = RS.logW; E2.pad = 0;
+  E2.aux = ek == GE_CALL ? RS.r1 : (ek == GE_RET ? RS.r0 : -1);
+  E2.xoff = xoff;
+  L.edges[e] = E2;
+  return 0;
+}
+
+// Node n's edge context; false if k_dl_sizes already rejected the node.
+__device__ __forceinline__ bool dl_edge_ctx(const DLDev& L, uint32_t n, uint32_t& k, EdgeCtx& c, uint64_t& r0, uint64_t& r1) {
+  k = app_of_node(L, n);
+  const DLApp& A = L.apps[k];
+  c.n = n; c.i = n - A.node_base;
+  c.kind = L.kind[n]; c.lm = L.meth[n];
+  if (c.kind > GK_ASTORE || c.lm >= A.n_meths) return false;
+  r0 = L.rp[A.ptr_base + c.i]; r1 = L.rp[A.ptr_base + c.i + 1];
+  c.a0 = L.ap[A.ptr_base + c.i]; c.a1 = L.ap[A.ptr_base + c.i + 1];
+  if (r1 < r0 || r1 > A.n_edges || c.a1 < c.a0 || c.a1 > A.n_args || r1 - r0 > 32768) return false;
+  c.sm = L.meths[A.meth_base + c.lm].module;
+  c.my_entry = L.mentry[A.meth_base + c.lm];
+  return true;
+}
+
+// Inline chunk-0 records: chunk 0 goes inline when it holds only INTRA / C2R edges of a narrow
+// block of <= INL_MAX_B words (as k_edges of kernels.cu).
+constexpr uint32_t DL_WARP_DEG = 32;     // nodes with more out-edges: one warp each (k_dl_edges_big)
+
+// V5 / V6 and Edge records, thread per node of out-degree <= DL_WARP_DEG; the others are listed in
+// big[] for k_dl_edges_big.
+__global__ void __launch_bounds__(256) k_dl_edges(DLDev L, uint32_t* big, uint32_t* n_big) {
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t n = blockIdx.x * blockDim.x + threadIdx.x; n < L.N; n += stride) {
-    const uint32_t k = app_of_node(L, n);
+    uint32_t k;
+    EdgeCtx c;
+    uint64_t r0, r1;
+    if (!dl_edge_ctx(L, n, k, c, r0, r1)) continue;
+    const uint32_t deg = (uint32_t)(r1 - r0);
+    if (deg > DL_WARP_DEG) { big[atomicAdd(n_big, 1u)] = n; continue; }
     const DLApp& A = L.apps[k];
-    const uint32_t i = n - A.node_base;
-    const uint32_t kind = L.kind[n], lm = L.meth[n];
-    if (kind > GK_ASTORE || lm >= A.n_meths) continue;       // reported by k_dl_sizes
-    const uint64_t r0 = L.rp[A.ptr_base + i], r1 = L.rp[A.ptr_base + i + 1];
-    const uint64_t a0 = L.ap[A.ptr_base + i], a1 = L.ap[A.ptr_base + i + 1];
-    if (r1 < r0 || r1 > A.n_edges || a1 < a0 || a1 > A.n_args || r1 - r0 > 32768) continue;
     const NodeRec R = L.nodes[n];
-    const uint32_t sm = L.meths[A.meth_base + lm].module;
-    const uint32_t my_entry = L.mentry[A.meth_base + lm];
-    const uint32_t deg = (uint32_t)(r1 - r0), n0 = min(deg, chunk_edges(deg, R.cls, R.logW));
+    const uint32_t n0 = min(deg, chunk_edges(deg, R.cls, R.logW));
     bool inl_ok = deg > 0 && n0 <= 4 && R.logW == 0 && R.B <= INL_MAX_B;
     InlEdge rec[4];
     uint32_t n_c2r = 0;
     unsigned long long err = 0;
     uint64_t err_e = 0;
     for (uint64_t el = r0; el < r1; ++el) {
-      const uint64_t e = A.edge_base + el;
-      const uint32_t sl = L.col[e], ek = L.ekind[e];
-      if (sl >= A.n_nodes || ek > GE_C2R) { err = ERR_INVALID; err_e = el; break; }
-      const uint32_t s = A.node_base + sl, skind = L.kind[s], tm = L.meth[s];
-      if (tm >= A.n_meths) { err = ERR_INVALID; err_e = el; break; }
-      bool ok = true;
-      switch (ek) {
-        case GE_INTRA: ok = kind != GK_CALL && kind != GK_EXIT && tm == lm; break;
-        case GE_C2R:
-          ok = kind == GK_CALL && skind == GK_RETSITE && L.ops[4ull * s + 3] == (int32_t)i;
-          ++n_c2r;
-          break;
-        case GE_CALL:                                          // V5 + V6 (arity)
-          ok = kind == GK_CALL && skind == GK_ENTRY && L.mentry[A.meth_base + tm] == sl &&
-               a1 - a0 == L.meths[A.meth_base + tm].n_params;
-          break;
-        case GE_RET: {                                         // to a site that calls this method
-          ok = kind == GK_EXIT && skind == GK_RETSITE;
-          const int32_t c = ok ? L.ops[4ull * s + 3] : -1;
-          if (ok && (c < 0 || (uint32_t)c >= A.n_nodes)) ok = false;
-          if (ok) {
-            const uint64_t c0 = L.rp[A.ptr_base + c], c1 = L.rp[A.ptr_base + c + 1];
-            bool found = false;
-            if (c1 >= c0 && c1 <= A.n_edges)
-              for (uint64_t e2 = c0; e2 < c1 && !found; ++e2)
-                found = L.ekind[A.edge_base + e2] == GE_CALL && L.col[A.edge_base + e2] == my_entry;
-            ok = found;
-          }
-          break;
-        }
-      }
-      if (!ok) { err = ERR_INVALID; err_e = el; break; }
-      uint32_t xoff = NO_XMAP;
-      if (ek == GE_CALL || ek == GE_RET) {
-        const uint32_t dm = L.meths[A.meth_base + tm].module;
-        if (dm != sm) xoff = (uint32_t)L.poff[A.pair_base + (uint64_t)(sm - A.mod_base) * A.n_mods + (dm - A.mod_base)];
-      }
-      const NodeRec RS = L.nodes[s];
-      const uint32_t nch = n_chunks_of(RS.e1 - RS.e0, RS.cls, RS.logW);
+      uint32_t ek;
       Edge E2;
-      E2.dst = s;
-      E2.info = ek | ((uint32_t)RS.cls << 2) | ((nch - 1) << 5) | (RS.logW >= 1 ? INFO_WIDE : 0u);
-      E2.off = RS.off; E2.B = RS.B; E2.L = (uint16_t)RS.L; E2.logW = RS.logW; E2.pad = 0;
-      E2.aux = ek == GE_CALL ? RS.r1 : (ek == GE_RET ? RS.r0 : -1);
-      E2.xoff = xoff;
-      L.edges[e] = E2;
+      err = dl_edge(L, A, c, el, ek, E2);
+      if (err) { err_e = el; break; }
+      n_c2r += ek == GE_C2R;
       const uint32_t jj = (uint32_t)(el - r0);
       if (jj < 4) rec[jj] = InlEdge{E2.dst, E2.info, E2.off};
       if (jj < n0) inl_ok = inl_ok && (ek == GE_INTRA || ek == GE_C2R);
     }
-    if (!err && kind == GK_CALL && n_c2r != 1) { err = ERR_INVALID; err_e = ~0ull; }
+    if (!err && c.kind == GK_CALL && n_c2r != 1) { err = ERR_INVALID; err_e = ~0ull; }
     if (err) {
-      dl_fail(L, k, err_e == ~0ull ? i : (uint64_t)A.n_nodes + err_e, err);
+      dl_fail(L, k, err_e == ~0ull ? c.i : (uint64_t)A.n_nodes + err_e, err);
       continue;
     }
     for (uint32_t j = 0; j < 4; ++j) L.inl[4ull * n + j] = (inl_ok && j < n0) ? rec[j] : InlEdge{0u, 0u, 0ull};
     L.nodes[n].n_inl = inl_ok ? (uint8_t)n0 : (uint8_t)0;   // (other threads read other fields only)
   }
+}
+
+// The same for the listed high-degree nodes (method exits with many return sites, virtual calls
+// with many targets), one warp per node, lanes over the edges.
+__global__ void __launch_bounds__(256) k_dl_edges_big(DLDev L, const uint32_t* big, const uint32_t* n_big) {
+  const uint32_t lane = threadIdx.x & 31, nb = *n_big;
+  const uint32_t stride = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nb; w += stride) {
+    const uint32_t n = big[w];
+    uint32_t k;
+    EdgeCtx c;
+    uint64_t r0, r1;
+    dl_edge_ctx(L, n, k, c, r0, r1);                          // listed: the checks passed
+    const DLApp& A = L.apps[k];
+    const NodeRec R = L.nodes[n];
+    const uint32_t deg = (uint32_t)(r1 - r0), n0 = min(deg, chunk_edges(deg, R.cls, R.logW));
+    bool inl_ok = n0 <= 4 && R.logW == 0 && R.B <= INL_MAX_B;
+    uint32_t n_c2r = 0;
+    unsigned long long err_w = ~0ull;                          // (edge index << 4 | code), lowest wins
+    InlEdge rec{0u, 0u, 0ull};
+    bool rec_ok = true;
+    for (uint64_t el = r0 + lane; el < r1; el += 32) {
+      uint32_t ek;
+      Edge E2;
+      const unsigned long long err = dl_edge(L, A, c, el, ek, E2);
+      if (err) { err_w = min(err_w, ((el - r0) << 4) | err); continue; }
+      n_c2r += ek == GE_C2R;
+      const uint32_t jj = (uint32_t)(el - r0);
+      if (jj < 4) rec = InlEdge{E2.dst, E2.info, E2.off};
+      if (jj < n0) rec_ok = ek == GE_INTRA || ek == GE_C2R;
+    }
+    for (int o = 16; o; o >>= 1) {
+      err_w = min(err_w, (unsigned long long)__shfl_xor_sync(0xffffffffu, err_w, o));
+      n_c2r += __shfl_xor_sync(0xffffffffu, n_c2r, o);
+    }
+    inl_ok = inl_ok && __all_sync(0xffffffffu, rec_ok);
+    if (err_w == ~0ull && c.kind == GK_CALL && n_c2r != 1) err_w = (1ull << 44) | ERR_INVALID;
+    if (err_w != ~0ull) {
+      if (lane == 0) {
+        const uint64_t el = err_w >> 4;
+        dl_fail(L, k, el >= (1ull << 40) ? c.i : (uint64_t)A.n_nodes + r0 + el, err_w & 15);
+      }
+      continue;
+    }
+    if (lane < 4) L.inl[4ull * n + lane] = (inl_ok && lane < n0) ? rec : InlEdge{0u, 0u, 0ull};
+    if (lane == 0) L.nodes[n].n_inl = inl_ok ? (uint8_t)n0 : (uint8_t)0;
+  }
+}
+
+// totals of the layout for the host, stored into mapped pinned memory: fact words, field-row and
+// projection table sizes, the error word, class counts (two per word)
+__global__ void k_dl_totals(DLDev L, uint64_t* out) {
+  if (threadIdx.x != 0) return;
+  out[0] = L.foff[L.N];
+  out[1] = L.koff[L.K];
+  out[2] = L.poff[L.P];
+  out[3] = *L.err;
+  for (int c = 0; c < NCLS; c += 2)
+    out[4 + c / 2] = (uint64_t)L.cls[c] | (c + 1 < NCLS ? (uint64_t)L.cls[c + 1] << 32 : 0ull);
+  __threadfence_system();
 }
 
 uint32_t grid_for(uint64_t n) {
@@ -374,11 +463,19 @@ cudaError_t launch_dl_sizes(const DLDev& L, uint64_t* scan_tmp, cudaStream_t s) 
   return e != cudaSuccess ? e : cudaGetLastError();
 }
 
+cudaError_t launch_dl_totals(const DLDev& L, uint64_t* host_mapped, cudaStream_t s) {
+  k_dl_totals<<<1, 32, 0, s>>>(L, host_mapped);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_dl_records(const DLDev& L, cudaStream_t s) {
   k_dl_nodes<<<grid_for(L.N), 256, 0, s>>>(L);
   if (L.K) k_dl_frow<<<grid_for(L.K), 256, 0, s>>>(L);
   if (L.P) k_dl_xmap<<<grid_for(L.P), 256, 0, s>>>(L);
-  k_dl_edges<<<grid_for(L.N), 256, 0, s>>>(L);
+  // the high-degree list reuses the phase-1 words[] (scan input, dead by now); its counter sits
+  // in cls[8] (zeroed with the class counts)
+  k_dl_edges<<<grid_for(L.N), 256, 0, s>>>(L, L.words, L.cls + 8);
+  k_dl_edges_big<<<148 * 8, 256, 0, s>>>(L, L.words, L.cls + 8);
   return cudaGetLastError();
 }
 

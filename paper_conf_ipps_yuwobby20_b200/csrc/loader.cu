@@ -838,7 +838,8 @@ struct LoadCache {
   size_t cap_a = 0;
   bool pinned = false, pinned_a = false;
   std::vector<HostImage> img;
-  uint64_t* dl_tot = nullptr;    // pinned readback of the device layout's totals (DLTot words)
+  uint64_t* dl_tot = nullptr;    // mapped pinned totals of the device layout (written by k_dl_totals)
+  uint64_t* dl_tot_dev = nullptr;
   // device layout: per-device scratch for the raw descriptor arrays and the layout kernels'
   // temporaries, grow-only and reused by every load (loads are serialised by mu and each one
   // waits for its layout kernels), so it never churns the stream-ordered pool between the
@@ -1100,6 +1101,7 @@ struct gdroid_app {
   uint64_t tab_len[9] = {};           // elements of each table (gdroid_debug_tables)
   uint64_t* d_facts = nullptr;        // nullptr after gdroid_release_facts (re-allocated by build)
   uint64_t fact_alloc_bytes = 0;
+  size_t fact_block_bytes = 0;        // size of the block behind d_facts (fact cache, facts_free)
   void* d_state = nullptr;            // stamp, queue, counts, stats, bar, digests
   uint32_t cls_count[NCLS] = {};      // work items per GRP class (queue segment sizes)
   DevStats* h_stats = nullptr;        // pinned slot (StatsSlots)
@@ -1139,6 +1141,8 @@ struct gdroid_app {
 
 namespace {
 
+void facts_free(int device, uint64_t* p, size_t bytes, cudaStream_t s);
+
 void free_app(gdroid_app* a) {
   if (!a) return;
   int cur = 0;
@@ -1146,9 +1150,9 @@ void free_app(gdroid_app* a) {
   cudaSetDevice(a->device);
   if (a->d_tables) cudaFreeAsync(a->d_tables, a->stream);
   if (a->d_tables2) cudaFreeAsync(a->d_tables2, a->stream);
-  if (a->d_facts) cudaFreeAsync(a->d_facts, a->stream);
+  if (a->d_facts) facts_free(a->device, a->d_facts, a->fact_block_bytes, a->stream);
   if (a->d_state) cudaFreeAsync(a->d_state, a->stream);
-  if (a->d_scratch) cudaFreeAsync(a->d_scratch, a->stream);
+  if (a->d_scratch) facts_free(a->device, a->d_scratch, a->scratch_bytes, a->stream);
   if (a->d_plain) cudaFree(a->d_plain);
   if (a->D.trace) cudaFree(a->D.trace);
   if (a->pending || a->h_seed) cudaStreamSynchronize(a->stream);   // copies target host slots
@@ -1168,21 +1172,43 @@ struct DeviceGuard {
   ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
 };
 
-// Readback scratch: stream-ordered (cudaFreeAsync / cudaMallocAsync on the handle's stream), so
-// growing it never synchronises the device.
+// Stream-ordered allocation (the device's default pool, release threshold raised) with large
+// sizes rounded up to one of 8 size classes per octave (<= 12.5 % slack): the batches of a corpus
+// differ by a few percent, and equal sizes let the pool hand a freed block straight to the next
+// batch on the same stream instead of mapping new memory — a mapping of a wide app's ~30 GB fact
+// store stalled the end-to-end pipeline for ~one build.
+size_t size_class(size_t bytes) {
+  if (bytes < (256ull << 20)) return bytes;
+  int b = 63 - __builtin_clzll(bytes);                        // 2^b <= bytes < 2^(b+1)
+  const size_t step = 1ull << (b - 3);
+  return (bytes + step - 1) / step * step;
+}
+
+cudaError_t pool_alloc(void** p, size_t bytes, cudaStream_t s) {
+  return cudaMallocAsync(p, size_class(bytes), s);
+}
+
+cudaError_t facts_alloc(int, size_t bytes, cudaStream_t s, uint64_t** p, size_t* got) {
+  *got = size_class(bytes);
+  return cudaMallocAsync((void**)p, *got, s);
+}
+
+void facts_free(int, uint64_t* p, size_t, cudaStream_t s) { cudaFreeAsync(p, s); }
+
 gdroid_status ensure_scratch(gdroid_app* a, size_t bytes) {
   if (a->scratch_bytes >= bytes) return GDROID_OK;
-  if (a->d_scratch) CU(cudaFreeAsync(a->d_scratch, a->stream));
+  if (a->d_scratch) facts_free(a->device, a->d_scratch, a->scratch_bytes, a->stream);
   a->d_scratch = nullptr;
   a->scratch_bytes = 0;
-  CU(cudaMallocAsync(&a->d_scratch, bytes, a->stream));
-  a->scratch_bytes = bytes;
+  size_t got = 0;
+  CU(facts_alloc(a->device, bytes, a->stream, &a->d_scratch, &got));   // large: the block cache
+  a->scratch_bytes = got;
   return GDROID_OK;
 }
 
 gdroid_status ensure_facts(gdroid_app* a) {
   if (a->d_facts) return GDROID_OK;
-  const cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, a->stream);
+  const cudaError_t e = facts_alloc(a->device, a->fact_alloc_bytes, a->stream, &a->d_facts, &a->fact_block_bytes);
   if (e != cudaSuccess) return set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e));
   a->D.facts = a->d_facts;
   a->D.delta = a->D.wide ? a->d_facts + std::max<uint64_t>(a->D.n_words, 4) : nullptr;
@@ -1303,9 +1329,14 @@ gdroid_status load_dl(const gdroid_icfg_desc* descs, uint32_t n_apps, gdroid_app
   const size_t up_a = qoff[Q_UPLOAD], up_r = woff[W_UPLOAD];
   gdroid_status s2 = ensure_pinned(g_cache.stage, g_cache.cap, g_cache.pinned, up_a + up_r, "device-layout inputs");
   if (s2 != GDROID_OK) return s2;
-  if (!g_cache.dl_tot && cudaMallocHost(&g_cache.dl_tot, 16 * 8) != cudaSuccess) {
-    g_cache.dl_tot = nullptr;
-    return set_err(GDROID_E_OOM, "pinned device-layout totals");
+  if (!g_cache.dl_tot) {
+    if (cudaHostAlloc(&g_cache.dl_tot, 16 * 8, cudaHostAllocMapped | cudaHostAllocPortable) != cudaSuccess ||
+        cudaHostGetDevicePointer((void**)&g_cache.dl_tot_dev, g_cache.dl_tot, 0) != cudaSuccess) {
+      cudaGetLastError();
+      if (g_cache.dl_tot) cudaFreeHost(g_cache.dl_tot);
+      g_cache.dl_tot = nullptr;
+      return set_err(GDROID_E_OOM, "mapped pinned device-layout totals");
+    }
   }
   char* SA = (char*)g_cache.stage;
   char* SR = SA + up_a;
@@ -1397,7 +1428,7 @@ gdroid_status load_dl(const gdroid_icfg_desc* descs, uint32_t n_apps, gdroid_app
     CU(cudaMalloc(&d_raw, want));
     raw_cap = want;
   }
-  CU(cudaMallocAsync(&a->d_tables, qoff[Q_NPART], a->stream));
+  CU(pool_alloc(&a->d_tables, qoff[Q_NPART], a->stream));
   char* DA = (char*)a->d_tables;
   char* DR = (char*)d_raw;
   CU(cudaMemcpyAsync(DA, SA, up_a, cudaMemcpyHostToDevice, a->stream));
@@ -1426,31 +1457,32 @@ gdroid_status load_dl(const gdroid_icfg_desc* descs, uint32_t n_apps, gdroid_app
   L.args = (int32_t*)(DA + qoff[Q_ARGS]); L.edges = (Edge*)(DA + qoff[Q_EDGES]); L.inl = (InlEdge*)(DA + qoff[Q_INL]);
   cudaError_t e = launch_dl_sizes(L, (uint64_t*)(DR + woff[W_SCAN]), a->stream);
   if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout kernels (sizes): %s", cudaGetErrorString(e));
-  uint64_t* tot = g_cache.dl_tot;                      // [0] fact words [1] frow [2] xmap [3] err [4..8] classes
-  CU(cudaMemcpyAsync(tot + 0, L.foff + N, 8, cudaMemcpyDeviceToHost, a->stream));
-  CU(cudaMemcpyAsync(tot + 1, L.koff + T.key, 8, cudaMemcpyDeviceToHost, a->stream));
-  CU(cudaMemcpyAsync(tot + 2, L.poff + T.pair, 8, cudaMemcpyDeviceToHost, a->stream));
-  CU(cudaMemcpyAsync(tot + 3, L.err, 8, cudaMemcpyDeviceToHost, a->stream));
-  CU(cudaMemcpyAsync(tot + 4, L.cls, NCLS * 4, cudaMemcpyDeviceToHost, a->stream));
+  // [0] fact words [1] frow [2] xmap [3] err [4..6] class counts: stored into the mapped pinned
+  // words by a kernel (posted PCIe writes), not by copies — a copy would queue behind the
+  // previous batch's fact readback on the D2H engine
+  volatile uint64_t* tot = g_cache.dl_tot;
+  e = launch_dl_totals(L, g_cache.dl_tot_dev, a->stream);
+  if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout totals: %s", cudaGetErrorString(e));
   CU(cudaStreamSynchronize(a->stream));
   a->h2d_ns = (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(std::chrono::steady_clock::now() - t0).count();
   PHASE("upload + layout sizes");
   if (tot[3] != DL_NO_ERR) { *dev_err = tot[3]; return GDROID_E_STATE; }
   const uint64_t fact_words = tot[0], n_frow = tot[1], n_xmap = tot[2];
   uint32_t cls_count[NCLS];
-  std::memcpy(cls_count, tot + 4, NCLS * 4);
+  for (int c = 0; c < NCLS; ++c) cls_count[c] = (uint32_t)(tot[4 + c / 2] >> (32 * (c & 1)));
   uint64_t nc = 0;
   for (int c = 0; c < NCLS; ++c) nc += cls_count[c];
   if (nc >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "too many work items");
   if (n_xmap >= (1ull << 32) || n_frow >= (1ull << 31)) return set_err(GDROID_E_LIMIT, "batch tables exceed 32-bit indices");
   // ---- field-row + projection tables, phase 2
   const size_t fb = align256(std::max<uint64_t>(n_frow, 1) * 4), xb = align256(std::max<uint64_t>(n_xmap, 1) * 4);
-  CU(cudaMallocAsync(&a->d_tables2, fb + xb, a->stream));
+  CU(pool_alloc(&a->d_tables2, fb + xb, a->stream));
   L.frow = (int32_t*)a->d_tables2;
   L.xmap = (int32_t*)((char*)a->d_tables2 + fb);
   e = launch_dl_records(L, a->stream);
   if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout kernels (records): %s", cudaGetErrorString(e));
-  CU(cudaMemcpyAsync(tot + 3, L.err, 8, cudaMemcpyDeviceToHost, a->stream));
+  e = launch_dl_totals(L, g_cache.dl_tot_dev, a->stream);
+  if (e != cudaSuccess) return set_err(GDROID_E_CUDA, "layout totals: %s", cudaGetErrorString(e));
   CU(cudaStreamSynchronize(a->stream));
   PHASE("layout records");
   if (tot[3] != DL_NO_ERR) { *dev_err = tot[3]; return GDROID_E_STATE; }
@@ -1747,7 +1779,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
   if (!dl_done) {
     std::lock_guard<std::mutex> lock(g_cache.mu);
     gdroid_status st = build_image(descs, n_apps, Lo, [&](const Layout& L) -> gdroid_status {
-      cudaError_t e = cudaMallocAsync(&a->d_tables, L.total, a->stream);
+      cudaError_t e = pool_alloc(&a->d_tables, L.total, a->stream);
       if (e != cudaSuccess) return set_err(e == cudaErrorMemoryAllocation ? GDROID_E_OOM : GDROID_E_CUDA, "device tables (%zu B): %s", L.total, cudaGetErrorString(e));
       e = cudaMemcpyAsync(a->d_tables, g_cache.stage_a, L.off[P_REGION_B], cudaMemcpyHostToDevice, a->stream);
       return e == cudaSuccess ? GDROID_OK : set_err(GDROID_E_CUDA, "H2D upload (A): %s", cudaGetErrorString(e));
@@ -1825,7 +1857,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     keep_pool_reserved(device);
     // wide batches: the Δ store of the semi-naive wide path follows the facts (same layout)
     a->fact_alloc_bytes = std::max<uint64_t>(Lo.fact_words, 4) * 8 * (Lo.wide ? 2 : 1);
-    cudaError_t e = cudaMallocAsync(&a->d_facts, a->fact_alloc_bytes, a->stream);
+    cudaError_t e = facts_alloc(device, a->fact_alloc_bytes, a->stream, &a->d_facts, &a->fact_block_bytes);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "fact store (%llu B): %s", (unsigned long long)a->fact_alloc_bytes, cudaGetErrorString(e)));
     D.facts = a->d_facts;
     D.delta = Lo.wide ? a->d_facts + std::max<uint64_t>(Lo.fact_words, 4) : nullptr;
@@ -1834,7 +1866,7 @@ gdroid_status gdroid_load_batch(const gdroid_icfg_desc* descs, uint32_t n_apps, 
     size_t s_stats = align256(sizeof(DevStats)), s_bar = 256, s_nd = align256((size_t)N * 8), s_ad = align256((size_t)n_apps * 8);
     size_t s_pc = align256((size_t)N * 4);
     size_t st = s_mask + s_stamp + s_queue + s_counts + s_stats + s_bar + s_nd + s_ad + s_pc;
-    e = cudaMallocAsync(&a->d_state, st, a->stream);
+    e = pool_alloc(&a->d_state, st, a->stream);
     if (e != cudaSuccess) return fail(set_err(GDROID_E_OOM, "device state (%zu B): %s", st, cudaGetErrorString(e)));
     char* S = (char*)a->d_state;
     D.smask = (uint64_t*)S; S += s_mask;
@@ -2029,7 +2061,7 @@ gdroid_status gdroid_build_idfg(gdroid_app* a, const gdroid_build_opts* opts, gd
   a->state_valid = true;
   a->facts_valid = true;
   if (o.release_facts) {                              // stream-ordered: after the digest kernel
-    CU(cudaFreeAsync(a->d_facts, s));
+    facts_free(a->device, a->d_facts, a->fact_block_bytes, s);
     a->d_facts = nullptr;
     D.facts = D.delta = nullptr;
     a->facts_valid = false;
@@ -2269,7 +2301,7 @@ gdroid_status gdroid_release_facts(gdroid_app* a) {
   if (a->pending) return set_err(GDROID_E_STATE, "an async build is still pending; call gdroid_sync");
   if (!a->d_facts) return GDROID_OK;
   DeviceGuard guard(a->device);
-  CU(cudaFreeAsync(a->d_facts, a->stream));
+  facts_free(a->device, a->d_facts, a->fact_block_bytes, a->stream);
   a->d_facts = nullptr;
   a->D.facts = a->D.delta = nullptr;
   a->facts_valid = false;
