@@ -110,8 +110,11 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_CONT_STAMP
 #define GD_CONT_STAMP 1
 #endif
+#ifndef GD_DYN
+#define GD_DYN 1             // wide batches: dynamic item hand-out within a round (run_round)
+#endif
 #ifndef GD_CONT_PF
-#define GD_CONT_PF 1         // light rounds: prefetch the inline successors' records into L1
+#define GD_CONT_PF 0         // light rounds: prefetch the inline successors' records into L1 (A/B: small +6 %, off)
 #endif
 constexpr uint32_t LQ_SKIP = 0xffffffffu;
 
@@ -1336,6 +1339,17 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
       return total;
     }
   }
+  // Wide batches (GD_DYN): item costs differ by orders of magnitude (a wide node is visited
+  // whole, over every out-edge), so after its first item a warp takes the next unclaimed one from
+  // a per-round counter (counts slot 6 of this rotation, cleared with the others) instead of
+  // striding by the warp count; a warp that drew heavy items no longer holds the round open.
+  const bool dyn = GD_DYN && WIDE && total > nw;
+  auto next_item = [&](uint32_t it) -> uint32_t {
+    if (!dyn) return it + nw;
+    uint32_t v = 0;
+    if (lane == 0) v = nw + atomicAdd(&D.counts[cur * CNT_STRIDE + 6], 1u);
+    return __shfl_sync(FULL, v, 0);
+  };
   uint32_t item = gw;
   uint32_t entry = item < total ? entry_of(item) : 0u;
   while (item < total) {
@@ -1347,11 +1361,11 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
         info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls, R.logW) - 1) << 5);
       }
       flush_pushes(D, st, lane, lane == 0, n, info, true, round, nxt);
-      item += nw;
+      item = next_item(item);
       entry = item < total ? entry_of(item) : 0u;
       continue;
     }
-    const uint32_t nitem = item + nw;
+    const uint32_t nitem = next_item(item);
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
     if constexpr (GD_PF) {
       // two-stage software pipeline: the records of item i+2 into L1, and — from item i+1's

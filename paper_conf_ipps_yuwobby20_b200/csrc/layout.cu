@@ -17,8 +17,10 @@
 //   k_dl_frow    thread per used key: column -> global heap row of (column instance, field).
 //   k_dl_xmap    thread per used module pair: colmap, rowmap, inverse rowmap (merge of the
 //                sorted pools).
-//   k_dl_edges   thread per node: V5 / V6 of every out-edge, Edge records with the destination
-//                layout and projection offset, inline chunk-0 records.
+//   k_dl_edges   thread per node of out-degree <= 32: V5 / V6 of every out-edge, Edge records
+//                with the destination layout and projection offset, inline chunk-0 records;
+//                higher-degree nodes are listed for k_dl_edges_big (one warp per node).
+//   k_dl_totals  the totals and the error word, stored into mapped pinned host memory.
 // Errors never fault: every index read from the input is range-checked, and the first error
 // (lowest app, then lowest node index) lands in err; the host then re-runs its own validator for
 // the exact message (loader.cu).

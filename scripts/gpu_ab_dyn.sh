@@ -1,0 +1,17 @@
+#!/bin/bash
+# A/B: dynamic item hand-out in wide rounds (GD_DYN=1, default) vs warp-strided items (GD_DYN=0).
+cd "${GRAFT_REPO_ROOT:-/root/repo}"
+mkdir -p gpurun_out
+out=gpurun_out/ab_dyn.log
+: > $out
+for v in 1 0 1 0; do
+  GDROID_NVCC_FLAGS="-DGD_DYN=$v" python -c "import __graft_entry__ as g; g.build()" >> gpurun_out/ab_build.log 2>&1
+  echo "== GD_DYN=$v worst" >> $out
+  timeout 600 python bench.py --workload worst --steps 5 --warmup 2 --no-cpu-baseline --e2e-steps 0 2>/dev/null | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print(round(d['ms_per_step'],2), d.get('rounds_rank0'), round(d['node_visits_per_s']/1e6,1))" >> $out
+  echo "== GD_DYN=$v corpus1000" >> $out
+  timeout 900 python bench.py --steps 3 --warmup 2 --no-cpu-baseline --e2e-steps 0 --no-per-config 2>/dev/null | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print(round(d['ms_per_step'],1), d['batch_ms_rank0'], d['parity']['mismatches'][:3])" >> $out
+done
+GDROID_NVCC_FLAGS="" python -c "import __graft_entry__ as g; g.build()" >> gpurun_out/ab_build.log 2>&1
+timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/ab_dyn_gpu_tests.log 2>&1
