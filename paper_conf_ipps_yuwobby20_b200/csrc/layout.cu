@@ -14,9 +14,9 @@
 //                then exclusive scans of the words, key sizes and pair sizes.
 //   k_dl_nodes   thread per node: NodeRec (rows of every operand, fact offset, layout), argument
 //                rows, global node-method / row_ptr / arg_ptr.
-//   k_dl_frow    thread per used key: column -> global heap row of (column instance, field).
-//   k_dl_xmap    thread per used module pair: colmap, rowmap, inverse rowmap (merge of the
-//                sorted pools).
+//   k_dl_frow    warp per used key: column -> global heap row of (column instance, field).
+//   k_dl_xmap    warp per used module pair: colmap, rowmap, inverse rowmap (binary searches
+//                in the sorted pools).
 //   k_dl_edges   thread per node of out-degree <= 32: V5 / V6 of every out-edge, Edge records
 //                with the destination layout and projection offset, inline chunk-0 records;
 //                higher-degree nodes are listed for k_dl_edges_big (one warp per node).
@@ -215,22 +215,30 @@ __global__ void __launch_bounds__(256) k_dl_nodes(DLDev L) {
 }
 
 // field-row table of one used (module, field) key: column c -> global row of (Q[c], f) or -1
+// One warp per 32 consecutive key entries; every used key's table is filled by the whole warp
+// (lanes over the columns).
 __global__ void __launch_bounds__(256) k_dl_frow(DLDev L) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < L.K; j += stride) {
-    if (!L.ksz[j]) continue;
-    const DLApp& A = L.apps[app_of_entry(L, j, 0)];
-    const uint64_t loc = j - A.key_base;
-    const uint32_t d = (uint32_t)(loc / A.n_fields), f = (uint32_t)(loc % A.n_fields);
-    const ModRec md = L.mods[A.mod_base + d];
-    int32_t* out = L.frow + L.koff[j];
-    for (uint32_t c = 0; c < md.n_cols; ++c) {
-      const int32_t ty = L.col_type[md.col_off + c];
-      int32_t row = -1;
-      if (c != 0 && ty >= 0)
-        for (uint32_t q = L.tf_ptr[ty]; q < L.tf_ptr[ty + 1]; ++q)
-          if (L.tf[q] == f) row = (int32_t)(L.col_hbase[md.col_off + c] + (q - L.tf_ptr[ty]));
-      out[c] = row;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t nwarp = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t j0 = (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; j0 < L.K; j0 += nwarp * 32) {
+    const uint64_t jl = j0 + lane;
+    unsigned used = __ballot_sync(0xffffffffu, jl < L.K && L.ksz[jl] != 0);
+    while (used) {
+      const uint64_t j = j0 + (__ffs(used) - 1);
+      used &= used - 1;
+      const DLApp& A = L.apps[app_of_entry(L, j, 0)];
+      const uint64_t loc = j - A.key_base;
+      const uint32_t d = (uint32_t)(loc / A.n_fields), f = (uint32_t)(loc % A.n_fields);
+      const ModRec md = L.mods[A.mod_base + d];
+      int32_t* out = L.frow + L.koff[j];
+      for (uint32_t c = lane; c < md.n_cols; c += 32) {
+        const int32_t ty = L.col_type[md.col_off + c];
+        int32_t row = -1;
+        if (c != 0 && ty >= 0)
+          for (uint32_t q = L.tf_ptr[ty]; q < L.tf_ptr[ty + 1]; ++q)
+            if (L.tf[q] == f) row = (int32_t)(L.col_hbase[md.col_off + c] + (q - L.tf_ptr[ty]));
+        out[c] = row;
+      }
     }
   }
 }
@@ -238,41 +246,46 @@ __global__ void __launch_bounds__(256) k_dl_frow(DLDev L) {
 // projection table π of one (source module, target module) pair: a column
 // is kept iff its instance is in Q_dst, a global row iff its slot is in P_src.  colmap[|Q_src|]
 // (src column -> dst column), rowmap[n_glob(dst)] (dst global row -> src global row), inverse
-// rowmap[n_glob(src)]; -1 = dropped.  Built by merging the ascending pools.
+// rowmap[n_glob(src)]; -1 = dropped.  One warp per 32 consecutive pair entries; a used pair's
+// table is filled by the whole warp: -1 everywhere, then lanes over the target's columns and
+// statics, each found in the source's ascending pool by binary search.
 __global__ void __launch_bounds__(256) k_dl_xmap(DLDev L) {
-  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < L.P; j += stride) {
-    const uint32_t sz = L.psz[j];
-    if (!sz) continue;
-    const DLApp& A = L.apps[app_of_entry(L, j, 1)];
-    const uint64_t loc = j - A.pair_base;
-    const ModRec ms = L.mods[A.mod_base + (uint32_t)(loc / A.n_mods)];
-    const ModRec mt = L.mods[A.mod_base + (uint32_t)(loc % A.n_mods)];
-    int32_t* cmap = L.xmap + L.poff[j];
-    int32_t* rmap = cmap + ms.n_cols;
-    int32_t* rinv = rmap + mt.n_glob;
-    for (uint32_t q = 0; q < sz; ++q) cmap[q] = -1;
-    const uint32_t* Ps = L.col_gid + ms.col_off;
-    const uint32_t* Pt = L.col_gid + mt.col_off;
-    for (uint32_t a = 0, b = 0; a < ms.n_cols && b < mt.n_cols;) {
-      if (Ps[a] == Pt[b]) {
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t nwarp = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t j0 = (((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; j0 < L.P; j0 += nwarp * 32) {
+    const uint64_t jl = j0 + lane;
+    unsigned used = __ballot_sync(0xffffffffu, jl < L.P && L.psz[jl] != 0);
+    while (used) {
+      const uint64_t j = j0 + (__ffs(used) - 1);
+      used &= used - 1;
+      const uint32_t sz = L.psz[j];
+      const DLApp& A = L.apps[app_of_entry(L, j, 1)];
+      const uint64_t loc = j - A.pair_base;
+      const ModRec ms = L.mods[A.mod_base + (uint32_t)(loc / A.n_mods)];
+      const ModRec mt = L.mods[A.mod_base + (uint32_t)(loc % A.n_mods)];
+      int32_t* cmap = L.xmap + L.poff[j];
+      int32_t* rmap = cmap + ms.n_cols;
+      int32_t* rinv = rmap + mt.n_glob;
+      for (uint32_t q = lane; q < sz; q += 32) cmap[q] = -1;
+      __syncwarp();                                            // the -1 fill before the entries
+      const uint32_t* Ps = L.col_gid + ms.col_off;
+      for (uint32_t b = lane; b < mt.n_cols; b += 32) {       // instances of Q_dst found in Q_src
+        const int64_t a = dl_bsearch(Ps, ms.n_cols, L.col_gid[mt.col_off + b]);
+        if (a < 0) continue;
         cmap[a] = (int32_t)b;
-        const int32_t ty = L.col_type[mt.col_off + b];     // heap rows of a shared instance
+        const int32_t ty = L.col_type[mt.col_off + b];       // heap rows of a shared instance
         if (b != 0 && ty >= 0) {
           const uint32_t nf = L.tf_ptr[ty + 1] - L.tf_ptr[ty];
-          const uint32_t gt = L.col_hbase[mt.col_off + b], gs = L.col_hbase[ms.col_off + a];
+          const uint32_t gt = L.col_hbase[mt.col_off + b], gs = L.col_hbase[ms.col_off + (uint32_t)a];
           for (uint32_t q = 0; q < nf; ++q) { rmap[gt + q] = (int32_t)(gs + q); rinv[gs + q] = (int32_t)(gt + q); }
         }
-        ++a; ++b;
-      } else if (Ps[a] < Pt[b]) ++a;
-      else ++b;
-    }
-    const uint32_t* Ss = L.grow_gid + ms.grow_off;          // static rows: ascending slot gids
-    const uint32_t* St = L.grow_gid + mt.grow_off;
-    for (uint32_t a = 0, b = 0; a < ms.n_stat && b < mt.n_stat;) {
-      if (Ss[a] == St[b]) { rmap[b] = (int32_t)a; rinv[a] = (int32_t)b; ++a; ++b; }
-      else if (Ss[a] < St[b]) ++a;
-      else ++b;
+      }
+      const uint32_t* Ss = L.grow_gid + ms.grow_off;        // static rows: ascending slot gids
+      for (uint32_t b = lane; b < mt.n_stat; b += 32) {
+        const int64_t a = dl_bsearch(Ss, ms.n_stat, L.grow_gid[mt.grow_off + b]);
+        if (a >= 0) { rmap[b] = (int32_t)a; rinv[a] = (int32_t)b; }
+      }
+      __syncwarp();
     }
   }
 }
@@ -472,8 +485,8 @@ cudaError_t launch_dl_totals(const DLDev& L, uint64_t* host_mapped, cudaStream_t
 
 cudaError_t launch_dl_records(const DLDev& L, cudaStream_t s) {
   k_dl_nodes<<<grid_for(L.N), 256, 0, s>>>(L);
-  if (L.K) k_dl_frow<<<grid_for(L.K), 256, 0, s>>>(L);
-  if (L.P) k_dl_xmap<<<grid_for(L.P), 256, 0, s>>>(L);
+  if (L.K) k_dl_frow<<<grid_for((L.K + 31) / 32 * 32), 256, 0, s>>>(L);
+  if (L.P) k_dl_xmap<<<grid_for((L.P + 31) / 32 * 32), 256, 0, s>>>(L);
   // the high-degree list reuses the phase-1 words[] (scan input, dead by now); its counter sits
   // in cls[8] (zeroed with the class counts)
   k_dl_edges<<<grid_for(L.N), 256, 0, s>>>(L, L.words, L.cls + 8);
