@@ -102,3 +102,14 @@ def test_loader_size_limits():
     assert _load_status(app(n_inst=100, n_stat=1100)) == -8 # wide block (> 64 instances) of > 1024 rows
     assert _load_status(app(fanout=32769)) == -8            # out-degree > 32768
     assert _load_status(app(n_inst=100, n_stat=10, fanout=3)) not in (-1, -2, -8)   # within limits
+
+
+def test_null_handles_rejected():
+    """Every entry point taking a handle rejects NULL with GDROID_E_INVALID (no device needed)."""
+    L = gd.lib()
+    n = C.c_uint64(0)
+    assert L.gdroid_debug_tables(None, 0, None, 0, C.byref(n)) == -1
+    assert L.gdroid_release_facts(None) == -1
+    assert L.gdroid_n_apps(None) == 0
+    assert L.gdroid_fact_bytes(None) == 0
+    L.gdroid_free(None)                                   # accepts NULL
