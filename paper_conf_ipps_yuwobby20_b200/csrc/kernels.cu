@@ -113,6 +113,12 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_DYN
 #define GD_DYN 1             // wide batches: dynamic item hand-out within a round (run_round)
 #endif
+#ifndef GD_INL3
+#define GD_INL3 1            // inline items of blocks <= 96 words: 3 words per lane instead of 4
+#endif
+#ifndef GD_DYN_NARROW
+#define GD_DYN_NARROW 0      // narrow batches too (A/B)
+#endif
 #ifndef GD_CONT_PF
 #define GD_CONT_PF 0         // light rounds: prefetch the inline successors' records into L1 (A/B: small +6 %, off)
 #endif
@@ -642,16 +648,18 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
 }
 // Word r of a block held as y[k] = word lane + 32k.  uword_of: r warp-uniform (one shuffle);
 // word_of: r per lane (every lane takes part).
-__device__ __forceinline__ uint64_t uword_of(const uint64_t (&y)[KW], uint32_t r) {
+template <int K>
+__device__ __forceinline__ uint64_t uword_of(const uint64_t (&y)[K], uint32_t r) {
   uint64_t s = y[0];
 #pragma unroll
-  for (int k = 1; k < KW; ++k) if ((r >> 5) == (uint32_t)k) s = y[k];
+  for (int k = 1; k < K; ++k) if ((r >> 5) == (uint32_t)k) s = y[k];
   return shfl64(s, (int)(r & 31u));
 }
-__device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r) {
+template <int K>
+__device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[K], uint32_t r) {
   uint64_t s = 0;
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint64_t v = shfl64(y[k], (int)(r & 31u));
     if ((r >> 5) == (uint32_t)k) s = v;
   }
@@ -663,17 +671,17 @@ __device__ __forceinline__ uint64_t word_of(const uint64_t (&y)[KW], uint32_t r)
 // path, with every read that the chain allows issued in the first memory hop: IN(src), the
 // destinations' round stamps and (FLOAD/FSTORE) the field-row table; the rows the transfer
 // function reads are taken from the IN(src) registers by shuffles instead of reloads.
-template <bool CNT, bool CD, bool SB = false>
+template <bool CNT, bool CD, bool SB = false, int K = KW>
 __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, const NodeRec& R, const InlEdge& me,
                                                    uint32_t round, uint32_t nxt, int lane, Acc& acc,
                                                    bool cont_ok, uint64_t mk0, uint64_t mk1) {
   const uint32_t B = R.B, L = R.L, ne = R.n_inl, kind = R.kind;
   const uint64_t* X = D.facts + R.off;             // coherent loads (no __restrict__: see process_wide)
-  uint64_t y[KW], p0[KW], p1[KW];
+  uint64_t y[K], p0[K], p1[K];
   const uint64_t off0 = shfl64(me.off, 0), off1 = shfl64(me.off, 1);
   uint32_t hasm = 0;                                        // bit k: word lane + 32k may be non-zero
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint32_t w = lane + 32 * k;
     const bool h = w < B && nmask_has(mk0, mk1, w);
     hasm |= (uint32_t)h << k;
@@ -724,7 +732,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     const uint64_t vrow = uword_of(y, (uint32_t)R.r0);
     genv = uword_of(y, (uint32_t)R.r1);                     // row w, OR-ed into rows (o1, f)
 #pragma unroll
-    for (int k = 0; k < KW; ++k) {
+    for (int k = 0; k < K; ++k) {
       uint32_t m = 0;
 #pragma unroll
       for (int q = 0; q < 2; ++q) {
@@ -740,7 +748,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
   }
   uint32_t nzx = 0, nz = 0, red = 0;
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint32_t w = lane + 32 * k;
     if (CNT) nzx += (y[k] != 0);
     if (mode == 1) { if ((int)w == t) y[k] = genv; }
@@ -755,9 +763,9 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     const int kill = ((info & 3u) == GE_C2R) ? R.r0 : -1;  // C2R drops lhs(c)
     uint64_t* Z = D.facts + off;
     uint64_t* zm = D.smask + (uint64_t)NMW * __shfl_sync(FULL, me.dst, (int)i);
-    uint64_t cur[KW];
+    uint64_t cur[K];
 #pragma unroll
-    for (int k = 0; k < KW; ++k) {
+    for (int k = 0; k < K; ++k) {
       const uint32_t w = lane + 32 * k;
       const bool keep = y[k] && (int)w != kill;
       const bool pre = (hasm >> k) & 1u;                    // pre-read done for this word
@@ -767,7 +775,7 @@ __device__ __forceinline__ uint32_t process_inline(const Dev& D, CtaStage& st, c
     }
     bool g = false;
 #pragma unroll
-    for (int k = 0; k < KW; ++k) {
+    for (int k = 0; k < K; ++k) {
       const uint32_t w = lane + 32 * k;
       const uint64_t z = (int)w == kill ? 0ull : y[k];
       nz += (z != 0);
@@ -980,6 +988,8 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     }
   }
   if (GD_INL && !WIDE && first && R.n_inl) {               // (wide batches: measured slower)
+    if (GD_INL3 && R.B <= 96u)                             // every row in words 0..95: 3 per lane
+      return process_inline<CNT, CD, SB, 3>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
     return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
   }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
@@ -1343,16 +1353,26 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   // whole, over every out-edge), so after its first item a warp takes the next unclaimed one from
   // a per-round counter (counts slot 6 of this rotation, cleared with the others) instead of
   // striding by the warp count; a warp that drew heavy items no longer holds the round open.
-  const bool dyn = GD_DYN && WIDE && total > nw;
-  auto next_item = [&](uint32_t it) -> uint32_t {
-    if (!dyn) return it + nw;
+  // Dynamic hand-out (GD_DYN: wide batches; GD_DYN_NARROW: narrow ones): item costs differ by
+  // orders of magnitude (a wide node is visited whole, over every out-edge; a CALL or EXIT chunk
+  // remaps a whole block), so after its first item a warp takes the next unclaimed one from a
+  // per-round counter (counts slot 6 of this rotation, cleared with the others) instead of
+  // striding by the warp count, and a warp that drew heavy items no longer holds the round open.
+  // The claim for the item after next is issued one item ahead (lane 0 holds it until the
+  // broadcast), so its latency hides behind the current item.  A warp's claims increase, so a
+  // claimed index < total is always processed by its claimer.
+  const bool dyn = GD_DYN && (WIDE || GD_DYN_NARROW) && total > nw;
+  uint32_t* const ctr = D.counts + cur * CNT_STRIDE + 6;
+  uint32_t item = gw, nitem = gw + nw;
+  if (dyn) {
     uint32_t v = 0;
-    if (lane == 0) v = nw + atomicAdd(&D.counts[cur * CNT_STRIDE + 6], 1u);
-    return __shfl_sync(FULL, v, 0);
-  };
-  uint32_t item = gw;
+    if (lane == 0) v = nw + atomicAdd(ctr, 1u);
+    nitem = __shfl_sync(FULL, v, 0);
+  }
   uint32_t entry = item < total ? entry_of(item) : 0u;
   while (item < total) {
+    uint32_t pend = 0;                                                 // lane 0: the item after next
+    if (dyn && lane == 0) pend = nw + atomicAdd(ctr, 1u);
     if (item >= head) {                                                // tail: defer to round+1
       const uint32_t n = entry >> 5;
       uint32_t info = 0;
@@ -1361,11 +1381,11 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
         info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls, R.logW) - 1) << 5);
       }
       flush_pushes(D, st, lane, lane == 0, n, info, true, round, nxt);
-      item = next_item(item);
+      item = nitem;
+      nitem = dyn ? __shfl_sync(FULL, pend, 0) : nitem + nw;
       entry = item < total ? entry_of(item) : 0u;
       continue;
     }
-    const uint32_t nitem = next_item(item);
     const uint32_t nentry = nitem < total ? entry_of(nitem) : 0u;    // prefetch the next item
     if constexpr (GD_PF) {
       // two-stage software pipeline: the records of item i+2 into L1, and — from item i+1's
@@ -1408,6 +1428,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
     }
     item = nitem;
     entry = nentry;
+    nitem = dyn ? __shfl_sync(FULL, pend, 0) : nitem + nw;
   }
   return total;
 }
