@@ -113,6 +113,12 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_DYN
 #define GD_DYN 1             // wide batches: dynamic item hand-out within a round (run_round)
 #endif
+#ifndef GD_ITEM3
+#define GD_ITEM3 1           // non-inline narrow items of blocks <= 96 words: 3 words per lane
+#endif
+#ifndef GD_INL2
+#define GD_INL2 0            // inline items of blocks <= 64 words: 2 words per lane (A/B: corpus +5.7 %, off)
+#endif
 #ifndef GD_INL3
 #define GD_INL3 1            // inline items of blocks <= 96 words: 3 words per lane instead of 4
 #endif
@@ -335,18 +341,19 @@ __device__ __forceinline__ void stage_publish(const Dev& D, CtaStage& st, uint32
 // OR KW words into IN(dst): a (possibly stale) load, then RED.OR only where bits are missing.
 // Words of row `kill` are dropped (C2R).  Returns the number of non-zero words in the low
 // 16 bits and the number of REDs issued in the high bits.
-__device__ __forceinline__ uint32_t or_chunk(uint64_t* Z, const uint64_t (&y)[KW], uint32_t c0,
+template <int K>
+__device__ __forceinline__ uint32_t or_chunk(uint64_t* Z, const uint64_t (&y)[K], uint32_t c0,
                                              int lane, int kill, uint32_t logW, uint64_t* zm) {
-  uint64_t cur[KW];
+  uint64_t cur[K];
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint32_t w = c0 + lane + 32 * k;
     const bool keep = y[k] && !(kill >= 0 && (int)(w >> logW) == kill);
     cur[k] = keep ? Z[w] : ~0ull;
   }
   uint32_t nz = 0, red = 0;
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint32_t w = c0 + lane + 32 * k;
     const uint64_t z = (kill >= 0 && (int)(w >> logW) == kill) ? 0ull : y[k];
     nz += (z != 0);
@@ -959,39 +966,14 @@ __device__ __forceinline__ void process_inline2(const Dev& D, CtaStage& st, cons
 }
 
 // ---------------------------------------------------------------------------------- one item
-template <bool WIDE, bool CNT, int MW, bool CD, bool SB = false>
-__device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
-                                 uint32_t nxt, int lane, WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont,
-                                 bool light = false) {
-  const uint64_t mk0 = GD_NMASK ? D.smask[(uint64_t)NMW * n] : ~0ull;       // (issued with the NodeRec load)
-  const uint64_t mk1 = GD_NMASK ? D.smask[(uint64_t)NMW * n + 1] : ~0ull;
-  const NodeRec R = D.nodes[n];
-  InlEdge me{0u, 0u, 0ull};                                 // inline chunk-0 edge of this lane (same hop)
-  if (GD_INL && !WIDE && lane < 4) me = D.inl[4 * n + lane];
-  const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls, R.logW);
-  const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
-  const bool first = ci == 0;
+// The narrow part of process_item (chunk of a narrow node that is not an inline item: CALL / EXIT /
+// multi-chunk nodes, blocks over the inline limit), K words per lane per pass over a block.
+template <bool WIDE, bool CNT, int MW, bool CD, bool SB, int K>
+__device__ __forceinline__ uint32_t narrow_item(const Dev& D, CtaStage& st, const NodeRec& R, uint32_t n, uint32_t e0,
+                                             uint32_t e1, bool first, uint32_t round, uint32_t nxt, int lane,
+                                             WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont, bool light,
+                                             uint32_t alg_l0, uint64_t mk0, uint64_t mk1) {
   const uint32_t L = R.L, B = R.B;
-  // SURVEY §8(d) constants: statement record + row_ptr once per node visit (chunk 0), 5 B per
-  // edge, 8 B queue entry in/out per item
-  uint32_t alg_l0 = (first ? 16u + 8u : 0u) + 5u * (e1 - e0) + 8u;
-  if (e0 >= e1) {                                           // no successor: nothing to propagate
-    if (CNT && lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
-    return NO_CONT;
-  }
-  if constexpr (WIDE) {
-    if (R.logW >= 1) {                                      // wide block: row-sparse path
-      uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
-      process_wide<CNT, MW, SB>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
-                   (GD_CONT_WIDE && allow_cont) ? &cont_v : nullptr, CD && light);
-      return cont_v;
-    }
-  }
-  if (GD_INL && !WIDE && first && R.n_inl) {               // (wide batches: measured slower)
-    if (GD_INL3 && R.B <= 96u)                             // every row in words 0..95: 3 per lane
-      return process_inline<CNT, CD, SB, 3>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
-    return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
-  }
   // From here on the source block is narrow (one 64-bit word per row: |Q| <= 64), in both
   // instantiations: word index = row index.
   constexpr uint32_t logW = 0u, W = 1u;
@@ -1001,9 +983,9 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
   // ---- independent loads first: this item's edge records, the first chunk of IN(src), and
   //      the rows the transfer function reads
   auto has = [&](uint32_t w) -> bool { return nmask_has(mk0, mk1, w); };
-  uint64_t y[KW];
+  uint64_t y[K];
 #pragma unroll
-  for (int k = 0; k < KW; ++k) {
+  for (int k = 0; k < K; ++k) {
     const uint32_t w = lane + 32 * k;
     y[k] = (w < B && has(w)) ? X[w] : 0ull;
   }
@@ -1046,7 +1028,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
       const int hr = D.frow[R.r3 + c];
       if (hr < 0) continue;
       const uint32_t w = L + (uint32_t)hr;
-      if (w < 32u * KW && (w & 31u) == (uint32_t)lane) fmask |= 1u << (w >> 5);
+      if (w < 32u * K && (w & 31u) == (uint32_t)lane) fmask |= 1u << (w >> 5);
     }
   }
   const uint64_t gsel = genv, rwsel = genv;                // identical on every lane
@@ -1063,16 +1045,16 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     unsigned gmask = 0;
     // -- INTRA / C2R: identical layouts; OUT computed once per chunk and reused by every edge
     if (same) {
-      for (uint32_t c0 = 0; c0 < B; c0 += 32 * KW) {
+      for (uint32_t c0 = 0; c0 < B; c0 += 32 * K) {
         if (c0 != 0 || eb != e0) {
 #pragma unroll
-          for (int k = 0; k < KW; ++k) {
+          for (int k = 0; k < K; ++k) {
             const uint32_t w = c0 + lane + 32 * k;
             y[k] = (w < B && has(w)) ? X[w] : 0ull;
           }
         }
 #pragma unroll
-        for (int k = 0; k < KW; ++k) {
+        for (int k = 0; k < K; ++k) {
           const uint32_t w = c0 + lane + 32 * k;
           if (first && eb == e0) nzx += (y[k] != 0);
           if (mode == 1) { if ((int)w == t) y[k] = gsel; }
@@ -1130,10 +1112,10 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
       };
       bool g = false;
       if (xoff == NO_XMAP) {                                // same module: word-parallel
-        for (uint32_t c0 = 0; c0 < Bt; c0 += 32 * KW) {
-          uint64_t z[KW];
+        for (uint32_t c0 = 0; c0 < Bt; c0 += 32 * K) {
+          uint64_t z[K];
 #pragma unroll
-          for (int k = 0; k < KW; ++k) {
+          for (int k = 0; k < K; ++k) {
             const uint32_t w = c0 + lane + 32 * k, r = w >> logW, j = w & (W - 1);
             int src = -1;
             if (w < Bt) src = (r < Lt) ? local_src(r) : (int)(L + (r - Lt));
@@ -1150,12 +1132,12 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
         for (uint32_t c = lane; c < R.n_cols; c += 32) ws.cmap[c] = (int16_t)D.xmap[xoff + c];
         const int32_t* rowmap = D.xmap + xoff + R.n_cols;
         const uint32_t rows_t = Bt >> logWt;
-        int src[KW];
+        int src[K];
 #pragma unroll
-        for (int k = 0; k < KW; ++k) src[k] = -1;
-        for (uint32_t r0 = 0; r0 < rows_t; r0 += 32 * KW) {
+        for (int k = 0; k < K; ++k) src[k] = -1;
+        for (uint32_t r0 = 0; r0 < rows_t; r0 += 32 * K) {
 #pragma unroll
-          for (int k = 0; k < KW; ++k) {                    // source row of each target row
+          for (int k = 0; k < K; ++k) {                    // source row of each target row
             const uint32_t r = r0 + lane + 32 * k;
             src[k] = -1;
             if (r < rows_t) {
@@ -1168,11 +1150,11 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
           }
           __syncwarp();
           if (!WIDE || (W == 1 && logWt == 0)) {            // one word per row on both sides
-            uint64_t v[KW], cur[KW];
+            uint64_t v[K], cur[K];
 #pragma unroll
-            for (int k = 0; k < KW; ++k) v[k] = (src[k] >= 0 && has((uint32_t)src[k])) ? X[src[k]] : 0ull;
+            for (int k = 0; k < K; ++k) v[k] = (src[k] >= 0 && has((uint32_t)src[k])) ? X[src[k]] : 0ull;
 #pragma unroll
-            for (int k = 0; k < KW; ++k) {
+            for (int k = 0; k < K; ++k) {
               uint64_t o = 0, b = v[k];
               while (b) {
                 const int bit = __ffsll((long long)b) - 1;
@@ -1184,7 +1166,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
               cur[k] = o ? Z[r0 + lane + 32 * k] : ~0ull;
             }
 #pragma unroll
-            for (int k = 0; k < KW; ++k) {
+            for (int k = 0; k < K; ++k) {
               nz += (v[k] != 0);
               if (v[k] & ~cur[k]) {
                 red_or(Z + r0 + lane + 32 * k, v[k]);
@@ -1195,7 +1177,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
             }
           } else if constexpr (WIDE) {
 #pragma unroll
-            for (int k = 0; k < KW; ++k) {
+            for (int k = 0; k < K; ++k) {
               if (src[k] < 0) continue;
               const uint32_t r = r0 + lane + 32 * k;
               uint64_t out[MW];
@@ -1233,6 +1215,49 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
     if (lane == 0) acc.dense += dense_l0 + alg_l0;
   }
   return cont_v;
+}
+
+
+template <bool WIDE, bool CNT, int MW, bool CD, bool SB = false>
+__device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_t ci, uint32_t round,
+                                 uint32_t nxt, int lane, WarpScratchT<WIDE>& ws, Acc& acc, bool allow_cont,
+                                 bool light = false) {
+  const uint64_t mk0 = GD_NMASK ? D.smask[(uint64_t)NMW * n] : ~0ull;       // (issued with the NodeRec load)
+  const uint64_t mk1 = GD_NMASK ? D.smask[(uint64_t)NMW * n + 1] : ~0ull;
+  const NodeRec R = D.nodes[n];
+  InlEdge me{0u, 0u, 0ull};                                 // inline chunk-0 edge of this lane (same hop)
+  if (GD_INL && !WIDE && lane < 4) me = D.inl[4 * n + lane];
+  const uint32_t deg = R.e1 - R.e0, ebs = chunk_edges(deg, R.cls, R.logW);
+  const uint32_t e0 = R.e0 + ci * ebs, e1 = min(R.e1, e0 + ebs);
+  const bool first = ci == 0;
+  const uint32_t L = R.L, B = R.B;
+  // SURVEY §8(d) constants: statement record + row_ptr once per node visit (chunk 0), 5 B per
+  // edge, 8 B queue entry in/out per item
+  uint32_t alg_l0 = (first ? 16u + 8u : 0u) + 5u * (e1 - e0) + 8u;
+  if (e0 >= e1) {                                           // no successor: nothing to propagate
+    if (CNT && lane == 0) { acc.alg += alg_l0; acc.dense += alg_l0; }
+    return NO_CONT;
+  }
+  if constexpr (WIDE) {
+    if (R.logW >= 1) {                                      // wide block: row-sparse path
+      uint32_t cont_v = NO_CONT;                            // node to continue into (warp-uniform)
+      process_wide<CNT, MW, SB>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, alg_l0,
+                   (GD_CONT_WIDE && allow_cont) ? &cont_v : nullptr, CD && light);
+      return cont_v;
+    }
+  }
+  if (GD_INL && !WIDE && first && R.n_inl) {               // (wide batches: measured slower)
+    if (GD_INL2 && R.B <= 64u)                             // every row in words 0..63: 2 per lane
+      return process_inline<CNT, CD, SB, 2>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
+    if (GD_INL3 && R.B <= 96u)                             // every row in words 0..95: 3 per lane
+      return process_inline<CNT, CD, SB, 3>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
+    return process_inline<CNT, CD, SB>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
+  }
+  if (!WIDE && GD_ITEM3 && B <= 96u)
+    return narrow_item<WIDE, CNT, MW, CD, SB, 3>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, allow_cont,
+                                                 light, alg_l0, mk0, mk1);
+  return narrow_item<WIDE, CNT, MW, CD, SB, KW>(D, st, R, n, e0, e1, first, round, nxt, lane, ws, acc, allow_cont,
+                                                light, alg_l0, mk0, mk1);
 }
 
 // ---------------------------------------------------------------------------------- rounds
