@@ -113,6 +113,9 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_DYN
 #define GD_DYN 1             // wide batches: dynamic item hand-out within a round (run_round)
 #endif
+#ifndef GD_DIG2
+#define GD_DIG2 0            // k_digest: bits spread over the lanes (digest_words2; A/B: corpus +8.8 %, off)
+#endif
 #ifndef GD_ITEM3
 #define GD_ITEM3 1           // non-inline narrow items of blocks <= 96 words: 3 words per lane
 #endif
@@ -1858,6 +1861,79 @@ __device__ __forceinline__ unsigned long long digest_words(const Dev& D, const N
   return s;
 }
 
+// The same digest with the work spread over the warp by bit position instead of by word
+// (GD_DIG2): the warp walks the node's non-zero words (narrow: the ballot of y; wide: the rows of
+// the occupancy bitmap) in lockstep, and lane l hashes bits l and l + 32 of each word, whose
+// instance gids it holds in registers for the whole node (the columns are the module's).  The
+// per-word row slot is one broadcast load; no lane loops over another lane's bits.
+__device__ __forceinline__ unsigned long long digest_words2(const Dev& D, const NodeRec& R, uint64_t hn,
+                                                            const uint64_t (&y)[DKW], int lane, uint32_t& pc) {
+  const uint32_t logW = R.logW, L = R.L, B = R.B, W = 1u << logW;
+  constexpr int OVQ = 8;                                   // columns held in registers: 256
+  uint32_t ov[OVQ];                                        // instance gid of column 32 q + lane
+#pragma unroll
+  for (int q = 0; q < OVQ; ++q) {
+    const uint32_t c = 32u * q + lane;
+    ov[q] = ((uint32_t)q < 2 * W && c < R.n_cols) ? D.col_gid[R.col_off + c] : 0u;
+  }
+  auto col = [&](int q) -> uint32_t {                      // q >= OVQ (|Q| > 256): from L1
+    const uint32_t c = 32u * q + lane;
+    return c < R.n_cols ? D.col_gid[R.col_off + c] : 0u;
+  };
+  unsigned long long s = 0;
+  auto slot_of = [&](uint32_t r) -> uint64_t {
+    return r < L ? (uint64_t)(R.local_base + r) : (uint64_t)D.grow_gid[R.grow_off + r - L];
+  };
+  auto bits = [&](uint64_t hs, uint64_t x, uint32_t o0, uint32_t o1) {
+    const bool b0 = (x >> lane) & 1ull, b1 = (x >> (lane + 32)) & 1ull;
+    pc += (uint32_t)b0 + (uint32_t)b1;
+    if (b0) s += mix64(hs ^ o0);
+    if (b1) s += mix64(hs ^ o1);
+  };
+  const uint64_t* X = D.facts + R.off;
+  if (logW >= 1) {                                         // wide block: occupied rows only
+    const uint32_t rows = B >> logW, nocc = occ_words(rows);
+    const uint64_t* OCC = X + occ_offset(B);
+    for (uint32_t i = 0; i < nocc; ++i) {
+      uint64_t ow = OCC[i];
+      while (ow) {
+        const uint32_t r = i * 64 + (__ffsll((long long)ow) - 1);
+        ow &= ow - 1;
+        const uint64_t hs = hn ^ (slot_of(r) << 32);
+#pragma unroll
+        for (int q = 0; q < MAXW; ++q) {
+          if ((uint32_t)q >= W) break;
+          const uint64_t x = X[((uint64_t)r << logW) + q];
+          if (!x) continue;
+          if (2 * q + 1 < OVQ) bits(hs, x, ov[2 * q], ov[2 * q + 1]);
+          else bits(hs, x, col(2 * q), col(2 * q + 1));
+        }
+      }
+    }
+    return s;
+  }
+#pragma unroll
+  for (int k = 0; k < DKW; ++k) {                          // narrow: one word per row
+    unsigned m = __ballot_sync(FULL, y[k] != 0);
+    while (m) {
+      const int src = __ffs(m) - 1;
+      m &= m - 1;
+      const uint64_t x = shfl64(y[k], src);
+      bits(hn ^ (slot_of((uint32_t)(src + 32 * k)) << 32), x, ov[0], ov[1]);
+    }
+  }
+  for (uint32_t w0 = 32 * DKW; w0 < B; w0 += 32) {          // blocks beyond 128 words
+    const uint64_t xl = w0 + lane < B ? X[w0 + lane] : 0ull;
+    unsigned m = __ballot_sync(FULL, xl != 0);
+    while (m) {
+      const int src = __ffs(m) - 1;
+      m &= m - 1;
+      bits(hn ^ (slot_of(w0 + src) << 32), shfl64(xl, src), ov[0], ov[1]);
+    }
+  }
+  return s;
+}
+
 // (a7) per-node digests d(n) = Σ mix64(mix64(n) ^ (slot<<32 | inst)) (C8).  A warp takes two
 // nodes at a time: both NodeRecs, then the first 128 words of both blocks, are loaded before any
 // bit is hashed (memory-level parallelism; the store is read once, coalesced).  A warp's nodes
@@ -1885,8 +1961,10 @@ __global__ void __launch_bounds__(256) k_digest(Dev D) {
       y2[k] = (has2 && R2.logW == 0 && w < R2.B) ? D.facts[R2.off + w] : 0ull;
     }
     uint32_t pc = 0, pc2 = 0;                               // facts per node (readback sizes)
-    const unsigned long long s = warp_sum64(digest_words(D, R, hn, y, lane, pc));
-    const unsigned long long s2 = has2 ? warp_sum64(digest_words(D, R2, hn2, y2, lane, pc2)) : 0ull;
+    const unsigned long long s = warp_sum64(GD_DIG2 ? digest_words2(D, R, hn, y, lane, pc)
+                                                    : digest_words(D, R, hn, y, lane, pc));
+    const unsigned long long s2 = !has2 ? 0ull : warp_sum64(GD_DIG2 ? digest_words2(D, R2, hn2, y2, lane, pc2)
+                                                                    : digest_words(D, R2, hn2, y2, lane, pc2));
     pc = __reduce_add_sync(FULL, pc);
     pc2 = __reduce_add_sync(FULL, pc2);
     if (lane == 0) {
