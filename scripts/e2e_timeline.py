@@ -11,6 +11,7 @@ from paper_conf_ipps_yuwobby20_b200 import corpus, _binding
 from synth import generator as G
 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 1000
+readback = sys.argv[2] if len(sys.argv) > 2 else "facts"
 sizes = G.corpus_sizes(n)
 wide = [G.corpus_config(i).q_cap > 64 for i in range(n)]
 plan = corpus.plan_corpus(sizes, wide, 1, node_budget=16_000_000)
@@ -30,12 +31,13 @@ def wrap(name):
 _binding.load = w_load
 for k in orig: setattr(_binding.App, k, wrap(k))
 bufs = corpus.ReadbackBuffers()
-corpus.run_pipelined(plan.batches[0], lambda i: apps[i], bufs=bufs)        # warm-up (sizes buffers)
+corpus.run_pipelined(plan.batches[0], lambda i: apps[i], bufs=bufs, readback=readback)   # warm-up (sizes buffers)
 EV.clear()
 torch.cuda.synchronize()
 T0[0] = time.perf_counter()
-corpus.run_pipelined(plan.batches[0], lambda i: apps[i], bufs=bufs)
+res = corpus.run_pipelined(plan.batches[0], lambda i: apps[i], bufs=bufs, readback=readback)
 wall = now()
+build_dev_ms = sum(r.stats["build_ns"] for r in res) / 1e6
 ids = {}
 rows = []
 for ev in EV:
@@ -44,6 +46,7 @@ for ev in EV:
 tot = {}
 for r in rows:
     tot[r["ev"]] = round(tot.get(r["ev"], 0) + r["t1"] - r["t0"], 1)
-print(json.dumps({"wall_ms": wall, "batches": len(plan.batches[0]), "sum_ms": tot}))
+print(json.dumps({"wall_ms": wall, "readback": readback, "batches": len(plan.batches[0]), "sum_ms": tot,
+                  "build_device_ms": round(build_dev_ms, 1)}))
 for r in rows:
     print(json.dumps(r))
