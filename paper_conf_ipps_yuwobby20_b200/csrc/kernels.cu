@@ -128,6 +128,9 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_DYN_NARROW
 #define GD_DYN_NARROW 0      // narrow batches too (A/B)
 #endif
+#ifndef GD_DYN_GRAIN
+#define GD_DYN_GRAIN 8       // narrow batches: items per claim
+#endif
 #ifndef GD_CONT_PF
 #define GD_CONT_PF 0         // light rounds: prefetch the inline successors' records into L1 (A/B: small +6 %, off)
 #endif
@@ -1389,18 +1392,28 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
   // The claim for the item after next is issued one item ahead (lane 0 holds it until the
   // broadcast), so its latency hides behind the current item.  A warp's claims increase, so a
   // claimed index < total is always processed by its claimer.
+  // Narrow rounds claim GD_DYN_GRAIN consecutive items per atomic (one counter for ~100M items
+  // per build is a hotspot at grain 1).
   const bool dyn = GD_DYN && (WIDE || GD_DYN_NARROW) && total > nw;
+  constexpr uint32_t G = WIDE ? 1u : (uint32_t)GD_DYN_GRAIN;
   uint32_t* const ctr = D.counts + cur * CNT_STRIDE + 6;
-  uint32_t item = gw, nitem = gw + nw;
+  uint32_t item = gw, nitem = gw + nw, nend = 0;                     // nend: end of nitem's claim
   if (dyn) {
     uint32_t v = 0;
-    if (lane == 0) v = nw + atomicAdd(ctr, 1u);
+    if (lane == 0) v = nw + G * atomicAdd(ctr, 1u);
     nitem = __shfl_sync(FULL, v, 0);
+    nend = nitem + G;
   }
+  auto advance = [&](uint32_t pend) {                                // item <- nitem <- the one after
+    item = nitem;
+    if (!dyn) nitem += nw;
+    else if (nitem + 1 < nend) ++nitem;
+    else { nitem = __shfl_sync(FULL, pend, 0); nend = nitem + G; }
+  };
   uint32_t entry = item < total ? entry_of(item) : 0u;
   while (item < total) {
-    uint32_t pend = 0;                                                 // lane 0: the item after next
-    if (dyn && lane == 0) pend = nw + atomicAdd(ctr, 1u);
+    uint32_t pend = 0;                          // lane 0: the next claim, issued one item ahead
+    if (dyn && nitem + 1 >= nend && lane == 0) pend = nw + G * atomicAdd(ctr, 1u);
     if (item >= head) {                                                // tail: defer to round+1
       const uint32_t n = entry >> 5;
       uint32_t info = 0;
@@ -1409,8 +1422,7 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
         info = ((uint32_t)R.cls << 2) | ((n_chunks_of(R.e1 - R.e0, R.cls, R.logW) - 1) << 5);
       }
       flush_pushes(D, st, lane, lane == 0, n, info, true, round, nxt);
-      item = nitem;
-      nitem = dyn ? __shfl_sync(FULL, pend, 0) : nitem + nw;
+      advance(pend);
       entry = item < total ? entry_of(item) : 0u;
       continue;
     }
@@ -1454,9 +1466,8 @@ __device__ __forceinline__ uint32_t run_round(const Dev& D, CtaStage& st, uint32
         if (lane == 0) acc.cont += 1;
       }
     }
-    item = nitem;
+    advance(pend);
     entry = nentry;
-    nitem = dyn ? __shfl_sync(FULL, pend, 0) : nitem + nw;
   }
   return total;
 }
