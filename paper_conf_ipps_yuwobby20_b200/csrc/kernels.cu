@@ -122,6 +122,9 @@ constexpr uint32_t LQCAP = 1024;
 #ifndef GD_ITEM3
 #define GD_ITEM3 1           // non-inline narrow items of blocks <= 96 words: 3 words per lane
 #endif
+#ifndef GD_INL4
+#define GD_INL4 1            // inline path for blocks of 97..128 words too (4 words per lane)
+#endif
 #ifndef GD_INL2
 #define GD_INL2 0            // inline items of blocks <= 64 words: 2 words per lane (A/B: corpus +5.7 %, off)
 #endif
@@ -1255,7 +1258,7 @@ __device__ uint32_t process_item(const Dev& D, CtaStage& st, uint32_t n, uint32_
       return cont_v;
     }
   }
-  if (GD_INL && !WIDE && first && R.n_inl) {               // (wide batches: measured slower)
+  if (GD_INL && !WIDE && first && R.n_inl && (GD_INL4 || R.B <= 96u)) {   // (wide batches: measured slower)
     if (GD_INL2 && R.B <= 64u)                             // every row in words 0..63: 2 per lane
       return process_inline<CNT, CD, SB, 2>(D, st, R, me, round, nxt, lane, acc, allow_cont && light, mk0, mk1);
     if (GD_INL3 && R.B <= 96u)                             // every row in words 0..95: 3 per lane
