@@ -38,7 +38,7 @@ constexpr int SCAP = 448 * THREADS / 256;   // staged queue entries per class pe
 #define GD_CONT_DEPTH 8        // longest depth-first continuation per queued item (0 = off)
 #endif
 #ifndef GD_CONT_DEPTH_NARROW
-#define GD_CONT_DEPTH_NARROW 4 // ... in narrow batches (sweep: small 1.51 -> 1.30 ms at 4, corpus flat)
+#define GD_CONT_DEPTH_NARROW 3 // ... in narrow batches (sweeps: small 1.51 / 1.30 / 1.24 / 1.26 ms at 8 / 4 / 3 / 2, corpus flat)
 #endif
 #ifndef GD_CONT_LOAD
 #define GD_CONT_LOAD 4         // continuation allowed in rounds with < GD_CONT_LOAD/4 items per warp
